@@ -1,0 +1,170 @@
+/*
+ * msccl.h — C ABI of the B200-native MSCCL-IR interpreter (libmsccl_b200.so).
+ *
+ * The runtime "is API-compatible with NCCL allowing existing ML workloads to easily
+ * convert" (MSCCLang, ASPLOS '23, §1): entry points, enum values and argument
+ * order mirror nccl.h (2.28). A collective call selects a loaded MSCCL-IR program by
+ * "user configurable size ranges" (§6) and runs it in ONE persistent CUDA
+ * kernel per GPU that interprets the program's instruction lists (§6.2, Fig. 5
+ * P:L1281-1310). Unlike the paper's runtime there is no NCCL fallback: a call with no
+ * matching program returns mscclNoMatchingProgram and launches nothing.
+ *
+ * Conventions for every function:
+ *  - returns mscclResult_t; never throws, never aborts the process;
+ *  - pointers named *buff are DEVICE pointers on the communicator's device, caller-owned,
+ *    valid until the stream reaches the operation; `count`s are ELEMENTS of `datatype`;
+ *  - a communicator is not thread-safe (NCCL rule); all ranks must load the same programs
+ *    in the same order and issue the same collectives with the same count/dtype/op;
+ *  - calls are asynchronous on `stream` and contain no host synchronisation or
+ *    allocation, so they can be captured in a CUDA graph;
+ *  - mscclGetLastError(comm) returns a human-readable reason for the last failure
+ *    (for program errors: rank/thread block/step and the violated rule V1..V9).
+ */
+#ifndef MSCCL_B200_H_
+#define MSCCL_B200_H_
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef struct mscclComm* mscclComm_t;
+typedef struct mscclProgram* mscclProgram_t;
+typedef struct CUstream_st* mscclStream_t; /* == cudaStream_t */
+
+/* 0..7 are numerically identical to ncclResult_t. */
+typedef enum {
+  mscclSuccess = 0,
+  mscclUnhandledCudaError = 1,
+  mscclSystemError = 2,
+  mscclInternalError = 3,
+  mscclInvalidArgument = 4,
+  mscclInvalidUsage = 5,
+  mscclRemoteError = 6,       /* watchdog timeout / peer abort (sticky, async) */
+  mscclInProgress = 7,
+  mscclInvalidProgram = 8,    /* IR failed to parse or validate */
+  mscclNoMatchingProgram = 9  /* no loaded program for (collective, nranks, bytes) */
+} mscclResult_t;
+
+/* Numerically identical to ncclDataType_t. */
+typedef enum {
+  mscclInt8 = 0, mscclUint8 = 1, mscclInt32 = 2, mscclUint32 = 3, mscclInt64 = 4,
+  mscclUint64 = 5, mscclFloat16 = 6, mscclFloat32 = 7, mscclFloat64 = 8, mscclBfloat16 = 9,
+  mscclNumTypes = 10
+} mscclDataType_t;
+
+/* Numerically identical to ncclRedOp_t; ncclAvg (4) is rejected (InvalidArgument). */
+typedef enum { mscclSum = 0, mscclProd = 1, mscclMax = 2, mscclMin = 3, mscclNumOps = 4 } mscclRedOp_t;
+
+/* Size of the opaque handle written by mscclCommExportHandle. */
+#define MSCCL_HANDLE_BYTES 128
+
+/* ---------------------------------------------------------------- communicators */
+
+/* One process drives `ndev` ranks; rank i runs on device devlist[i] (devlist may be NULL:
+ * devices 0..ndev-1). Distinct devices are connected by CUDA peer access over NVLink.
+ * Repeated device ids are VIRTUAL RANKS: several ranks on one GPU, whose buffers and
+ * FIFOs all live in that GPU's HBM (used for correctness work on one GPU). Ranks that
+ * share a device must issue their calls inside mscclGroupStart/End so that they run in
+ * ONE cooperative launch (all thread blocks co-resident, §6.2).
+ * comms[ndev] is written; each must be destroyed with mscclCommDestroy. */
+mscclResult_t mscclCommInitAll(mscclComm_t* comms, int ndev, const int* devlist);
+
+/* One process per GPU: allocate this rank's shared region (FIFOs, flags) on cudaDev.
+ * Then mscclCommExportHandle -> exchange (e.g. torch.distributed all_gather) ->
+ * mscclCommConnect before the first collective. */
+mscclResult_t mscclCommInitRank(mscclComm_t* comm, int nranks, int rank, int cudaDev);
+
+/* Writes MSCCL_HANDLE_BYTES bytes (CUDA IPC handle of the shared region) to `handle`;
+ * *bytes (if not NULL) receives MSCCL_HANDLE_BYTES. */
+mscclResult_t mscclCommExportHandle(mscclComm_t comm, void* handle, size_t* bytes);
+
+/* allHandles: nranks * MSCCL_HANDLE_BYTES bytes, rank order. Opens every peer's region. */
+mscclResult_t mscclCommConnect(mscclComm_t comm, const void* allHandles);
+
+/* Frees the region, programs and IPC mappings (synchronises the device). */
+mscclResult_t mscclCommDestroy(mscclComm_t comm);
+
+mscclResult_t mscclCommCount(const mscclComm_t comm, int* count);
+mscclResult_t mscclCommUserRank(const mscclComm_t comm, int* rank);
+mscclResult_t mscclCommCuDevice(const mscclComm_t comm, int* device);
+
+/* Sticky asynchronous error: mscclRemoteError after a device watchdog timeout (a spin
+ * wait exceeded MSCCL_TIMEOUT_S, default 20 s) or an abort raised by a peer. */
+mscclResult_t mscclCommGetAsyncError(mscclComm_t comm, mscclResult_t* asyncError);
+
+/* ---------------------------------------------------------------- programs */
+
+/* Parse + validate an MSCCL-IR program (text, irBytes bytes; copied) and upload its
+ * instruction tables for this rank (§6.2 "Initialization"). The program is
+ * selected for calls whose byte size (count * element size of the call's datatype) is
+ * in [minBytes, maxBytes); maxBytes == 0 means unbounded. First loaded program wins.
+ * Errors: mscclInvalidProgram (parse/validation, see mscclGetLastError). */
+mscclResult_t mscclLoadProgram(mscclComm_t comm, const char* ir, size_t irBytes, size_t minBytes,
+                               size_t maxBytes, mscclProgram_t* program);
+mscclResult_t mscclUnloadProgram(mscclComm_t comm, mscclProgram_t program);
+
+/* Statistics of a loaded program for this rank: thread blocks (= CTAs launched), total
+ * instructions, and whether it is in place. Any pointer may be NULL. */
+mscclResult_t mscclProgramInfo(mscclProgram_t program, int* nThreadBlocks, int* nInstructions, int* inplace);
+
+/* Comm-free structural validation (rules V1..V9 of DESIGN.md) — needs no GPU.
+ * slots = FIFO slots per connection used by the deadlock check (0 = library default),
+ * maxThreadBlocks = co-residency limit per rank (0 = 148). err (may be NULL) receives a
+ * NUL-terminated reason. Returns mscclSuccess or mscclInvalidProgram. */
+mscclResult_t mscclValidateProgram(const char* ir, size_t irBytes, int nranks, int slots,
+                                   int maxThreadBlocks, char* err, size_t errBytes);
+
+/* ---------------------------------------------------------------- collectives
+ * Semantics (n = count / per-rank block):
+ *   AllReduce     out_r[e]       = (op)_q in_q[e]
+ *   AllGather     out_r[q*n + e] = in_q[e]                          (sendcount = n)
+ *   ReduceScatter out_r[e]       = (op)_q in_q[r*n + e]             (recvcount = n)
+ *   AllToAll      out_r[q*n + e] = in_q[r*n + e]   (count per peer)
+ * In place (NCCL forms): AllReduce sendbuff == recvbuff; AllGather sendbuff ==
+ * recvbuff + rank*n; ReduceScatter recvbuff == sendbuff + rank*n. An in-place program
+ * called out of place gets a device copy send->recv first; an out-of-place program
+ * called in place must be marked aliassafe in its IR, else mscclInvalidUsage.
+ * count == 0 is a no-op. Floating-point results are bit-identical to the CPU oracle
+ * executing the same program (one rounding per reduce instruction). */
+mscclResult_t mscclAllReduce(const void* sendbuff, void* recvbuff, size_t count, mscclDataType_t datatype,
+                             mscclRedOp_t op, mscclComm_t comm, mscclStream_t stream);
+mscclResult_t mscclAllGather(const void* sendbuff, void* recvbuff, size_t sendcount, mscclDataType_t datatype,
+                             mscclComm_t comm, mscclStream_t stream);
+mscclResult_t mscclReduceScatter(const void* sendbuff, void* recvbuff, size_t recvcount,
+                                 mscclDataType_t datatype, mscclRedOp_t op, mscclComm_t comm,
+                                 mscclStream_t stream);
+mscclResult_t mscclAllToAll(const void* sendbuff, void* recvbuff, size_t count, mscclDataType_t datatype,
+                            mscclComm_t comm, mscclStream_t stream);
+
+/* Run a specific loaded program regardless of size ranges (bench / tests). `count` is
+ * interpreted per the program's collective as above. */
+mscclResult_t mscclRunProgram(mscclProgram_t program, const void* sendbuff, void* recvbuff, size_t count,
+                              mscclDataType_t datatype, mscclRedOp_t op, mscclComm_t comm, mscclStream_t stream);
+
+/* Group semantics (ncclGroupStart/End): calls between them are recorded and launched at
+ * mscclGroupEnd, one cooperative kernel per device covering every rank on that device. */
+mscclResult_t mscclGroupStart(void);
+mscclResult_t mscclGroupEnd(void);
+
+/* ---------------------------------------------------------------- misc */
+const char* mscclGetErrorString(mscclResult_t result);
+const char* mscclGetLastError(mscclComm_t comm); /* comm may be NULL: last global error */
+
+/* Tuning knobs (process-wide, read when a communicator is created; env vars of the same
+ * name override at first use): "MSCCL_SLOTS" FIFO slots per connection (1..16, default 4),
+ * "MSCCL_SLOT_BYTES" Simple-protocol slot size (default 262144), "MSCCL_MAX_CHANNELS"
+ * (default 32), "MSCCL_THREADS" threads per CTA (default 512), "MSCCL_TIMEOUT_S"
+ * watchdog (default 20). Returns mscclInvalidArgument for an unknown key. */
+mscclResult_t mscclSetParam(const char* key, int64_t value);
+mscclResult_t mscclGetParam(const char* key, int64_t* value);
+
+/* Number of interpreter kernels this process has launched (for launch accounting). */
+uint64_t mscclLaunchCount(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MSCCL_B200_H_ */

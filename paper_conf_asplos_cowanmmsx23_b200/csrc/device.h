@@ -1,0 +1,68 @@
+// Structures shared by the host runtime and the interpreter kernel.
+//
+// Instruction record = Fig. 5 lines 1-5: opcode, src/dst buffer + chunk
+// offset, count, dependency list (depBid/depStep generalised to a variable-length table,
+// DESIGN.md reading R4) and hasDep.
+#pragma once
+#include <stdint.h>
+
+namespace msccl {
+
+#define MSCCL_MAX_LOCAL 16  // ranks that one kernel launch may cover (virtual ranks)
+
+struct DevInstr {     // 24 bytes
+  uint8_t op, srcBuf, dstBuf, nDeps;
+  uint16_t cnt, hasDep;
+  uint32_t srcOff, dstOff, depStart, pad;
+};
+
+// One thread block of one rank (= one CTA). Connection pointers are resolved at load time
+// from the communicator's peer mapping (receiver-side FIFOs, §6.1).
+struct DevTB {
+  int32_t nSteps;
+  uint32_t instrStart;
+  int32_t tbId;
+  int32_t pad;
+  // send connection (peer = receiver): FIFO and head counter live in the PEER's region
+  char* sendFifo;             // peer FIFO base for (me -> peer, chan); nullptr if no send peer
+  uint64_t* sendHead;         // peer: messages posted by me
+  uint64_t* sendAck;          // mine: messages the peer consumed (written by the peer)
+  uint64_t* sendCnt;          // mine: persistent count of messages I posted
+  // receive connection (peer = sender)
+  char* recvFifo;             // my FIFO base for (peer -> me, chan)
+  uint64_t* recvHead;         // mine: messages the peer posted (written by the peer)
+  uint64_t* recvAck;          // peer: messages I consumed
+  uint64_t* recvCnt;          // mine: persistent count of messages I consumed
+};
+
+struct RankArgs {
+  const DevTB* tbs;
+  const DevInstr* instrs;
+  const uint32_t* deps;       // (tb << 16) | step
+  uint64_t* sem;              // per-TB semaphores (monotone, reading R4)
+  uint64_t* gen;              // per-TB launch generation
+  char* buf[3];               // in, out, scratch base pointers for this call
+  int32_t nTB;
+  int32_t ctaStart;           // first CTA of this rank in the grid
+  uint32_t* abortFlag;        // this rank's abort word (device memory of its region)
+  uint32_t* hostAbort;        // this rank's host-mapped pinned word (watchdog report)
+};
+
+struct KernelArgs {
+  RankArgs rank[MSCCL_MAX_LOCAL];
+  int32_t nLocal;
+  int32_t I;                  // pipeline iterations (reading R3)
+  int64_t n;                  // elements per block
+  int64_t E;                  // elements per chunk
+  int64_t T;                  // tile elements
+  int32_t cb;                 // chunks per block
+  int32_t blocks[3];          // blocks of in / out / scratch (scratch: 1)
+  int32_t slots;              // FIFO slots per connection
+  int32_t proto;              // 0 Simple, 1 LL
+  int64_t slotBytes;
+  int32_t sysScope;           // 1 when any peer is another GPU
+  int32_t pad;
+  uint64_t timeoutNs;
+};
+
+}  // namespace msccl

@@ -1,0 +1,460 @@
+// The MSCCL-IR interpreter kernel for sm_100a (MSCCLang §6.2, Fig. 5).
+//
+// One CTA = one IR thread block; every CTA of every rank on this GPU is co-resident
+// (cooperative launch). Per CTA:
+//
+//   for t in [0, I):                      pipelining loop (Fig. 5 line 10)
+//     for s in [0, nSteps):               instruction loop (line 12)
+//       wait cross-TB deps                (lines 14-16; monotone semaphores, reading R4)
+//       switch (op): primitive            (lines 18-23; one switch case per opcode)
+//       post semaphore if hasDep          (lines 24-27)
+//
+// Primitives move tile t of each of the `cnt` chunks of the instruction (strided tiling,
+// reading R3). Connections are receiver-side FIFOs of `slots` slots (§6.1):
+//  * Simple: the sender waits for a free slot (ack counter), all threads store 16-byte
+//    vectors straight into the receiver's slot (peer memory over NVLink, or the same HBM
+//    for virtual ranks), then one thread fences and bumps the receiver's head counter;
+//    the receiver acquires head, reads the slot with L1-bypassing loads, and acks.
+//  * LL: 16-byte lines {data32, flag, data32, flag}; flag = message sequence number; the
+//    receiver polls lines, no fence and no head counter (latency protocol).
+// Reductions apply one correctly rounded binary op per element (reading R6).
+#pragma once
+#include <cuda_bf16.h>
+#include <cuda_fp16.h>
+#include <stdint.h>
+#include <type_traits>
+
+#include "device.h"
+
+namespace msccl {
+
+enum { R_SUM = 0, R_PROD = 1, R_MAX = 2, R_MIN = 3, R_COPY = 4 };
+enum { DT_I8 = 0, DT_U8 = 1, DT_I32 = 2, DT_U32 = 3, DT_I64 = 4, DT_U64 = 5, DT_F16 = 6, DT_F32 = 7, DT_F64 = 8,
+       DT_BF16 = 9 };
+enum { K_NOP = 0, K_SEND = 1, K_RECV = 2, K_COPY = 3, K_REDUCE = 4, K_RRC = 5, K_RRS = 6, K_RRCS = 7, K_RCS = 8 };
+enum { KB_IN = 0, KB_OUT = 1, KB_SC = 2 };
+
+// ------------------------------------------------------------------ element types
+template <int DT> struct DType;
+#define MSCCL_INT_DTYPE(ID, S, U)                                                          \
+  template <> struct DType<ID> {                                                           \
+    typedef S T;                                                                           \
+    static __device__ __forceinline__ T op(int o, T a, T b) {                              \
+      if (o == R_SUM) return (T)((U)a + (U)b);                                             \
+      if (o == R_PROD) return (T)((U)a * (U)b);                                            \
+      if (o == R_MAX) return a >= b ? a : b;                                               \
+      return a <= b ? a : b;                                                               \
+    }                                                                                      \
+  };
+MSCCL_INT_DTYPE(DT_I8, int8_t, uint8_t)
+MSCCL_INT_DTYPE(DT_U8, uint8_t, uint8_t)
+MSCCL_INT_DTYPE(DT_I32, int32_t, uint32_t)
+MSCCL_INT_DTYPE(DT_U32, uint32_t, uint32_t)
+MSCCL_INT_DTYPE(DT_I64, int64_t, uint64_t)
+MSCCL_INT_DTYPE(DT_U64, uint64_t, uint64_t)
+#undef MSCCL_INT_DTYPE
+
+// IEEE types: max/min follow numpy.maximum/minimum ((a >= b or a is NaN) ? a : b).
+template <typename F>
+__device__ __forceinline__ F fop(int o, F a, F b) {
+  if (o == R_SUM) return a + b;
+  if (o == R_PROD) return a * b;
+  if (o == R_MAX) return (a >= b || a != a) ? a : b;
+  return (a <= b || a != a) ? a : b;
+}
+template <> struct DType<DT_F32> {
+  typedef float T;
+  static __device__ __forceinline__ T op(int o, T a, T b) { return fop<float>(o, a, b); }
+};
+template <> struct DType<DT_F64> {
+  typedef double T;
+  static __device__ __forceinline__ T op(int o, T a, T b) { return fop<double>(o, a, b); }
+};
+template <> struct DType<DT_F16> {  // storage: IEEE binary16 bits
+  typedef uint16_t T;
+  static __device__ __forceinline__ T op(int o, T a, T b) {
+    float x = __half2float(__ushort_as_half(a)), y = __half2float(__ushort_as_half(b));
+    if (o == R_MAX) return (x >= y || x != x) ? a : b;
+    if (o == R_MIN) return (x <= y || x != x) ? a : b;
+    return __half_as_ushort(__float2half_rn(fop<float>(o, x, y)));
+  }
+};
+template <> struct DType<DT_BF16> {  // storage: bf16 bits (top half of an fp32)
+  typedef uint16_t T;
+  static __device__ __forceinline__ float widen(T a) { return __uint_as_float(((uint32_t)a) << 16); }
+  static __device__ __forceinline__ T op(int o, T a, T b) {
+    float x = widen(a), y = widen(b);
+    if (o == R_MAX) return (x >= y || x != x) ? a : b;
+    if (o == R_MIN) return (x <= y || x != x) ? a : b;
+    return __bfloat16_as_ushort(__float2bfloat16_rn(fop<float>(o, x, y)));
+  }
+};
+
+// 16-byte vector op; sum/prod of fp16/bf16 use the packed correctly-rounded instructions.
+template <int DT, int OP>
+__device__ __forceinline__ uint4 vop(uint4 a, uint4 b) {
+  typedef typename DType<DT>::T T;
+  if (DT == DT_BF16 && (OP == R_SUM || OP == R_PROD)) {
+    uint32_t* x = reinterpret_cast<uint32_t*>(&a);
+    const uint32_t* y = reinterpret_cast<const uint32_t*>(&b);
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+      __nv_bfloat162 p = *reinterpret_cast<__nv_bfloat162*>(&x[i]);
+      __nv_bfloat162 q = *reinterpret_cast<const __nv_bfloat162*>(&y[i]);
+      __nv_bfloat162 r = OP == R_SUM ? __hadd2(p, q) : __hmul2(p, q);
+      x[i] = *reinterpret_cast<uint32_t*>(&r);
+    }
+    return a;
+  }
+  if (DT == DT_F16 && (OP == R_SUM || OP == R_PROD)) {
+    uint32_t* x = reinterpret_cast<uint32_t*>(&a);
+    const uint32_t* y = reinterpret_cast<const uint32_t*>(&b);
+#pragma unroll
+    for (int i = 0; i < 4; i++) {
+      __half2 p = *reinterpret_cast<__half2*>(&x[i]);
+      __half2 q = *reinterpret_cast<const __half2*>(&y[i]);
+      __half2 r = OP == R_SUM ? __hadd2(p, q) : __hmul2(p, q);
+      x[i] = *reinterpret_cast<uint32_t*>(&r);
+    }
+    return a;
+  }
+  T* x = reinterpret_cast<T*>(&a);
+  const T* y = reinterpret_cast<const T*>(&b);
+#pragma unroll
+  for (int i = 0; i < (int)(16 / sizeof(T)); i++) x[i] = DType<DT>::op(OP, x[i], y[i]);
+  return a;
+}
+
+// ------------------------------------------------------------------ memory primitives
+__device__ __forceinline__ uint4 ldcg(const void* p) {
+  uint4 v;
+  asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void stg(void* p, uint4 v) {
+  asm volatile("st.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+}
+__device__ __forceinline__ uint4 ldvol(const void* p) {
+  uint4 v;
+  asm volatile("ld.volatile.global.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void stvol(void* p, uint4 v) {
+  asm volatile("st.volatile.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
+}
+__device__ __forceinline__ uint64_t ldAcquireSys(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ uint64_t ldAcquireGpu(const uint64_t* p) {
+  uint64_t v;
+  asm volatile("ld.acquire.gpu.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+  return v;
+}
+__device__ __forceinline__ void stRelaxedSys(uint64_t* p, uint64_t v) {
+  asm volatile("st.relaxed.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void stRelaxedGpu(uint64_t* p, uint64_t v) {
+  asm volatile("st.relaxed.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
+__device__ __forceinline__ void fenceSys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
+__device__ __forceinline__ void fenceGpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+__device__ __forceinline__ uint64_t globaltimer() {
+  uint64_t t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
+// ------------------------------------------------------------------ watchdog + waits
+struct Ctx {
+  const KernelArgs* a;
+  const RankArgs* ra;
+  int tid, nt;
+};
+
+static __device__ __noinline__ void raiseAbort(const KernelArgs& a) {
+  for (int r = 0; r < a.nLocal; r++) {
+    atomicExch(a.rank[r].abortFlag, 1u);
+    *(volatile uint32_t*)a.rank[r].hostAbort = 1u;
+  }
+}
+
+// Spin until *p >= target (acquire). Returns false on watchdog timeout / abort.
+__device__ __forceinline__ bool waitGE(const uint64_t* p, uint64_t target, bool sys, const Ctx& c) {
+  if ((sys ? ldAcquireSys(p) : ldAcquireGpu(p)) >= target) return true;
+  uint64_t t0 = globaltimer();
+  for (uint32_t it = 1;; it++) {
+    if ((sys ? ldAcquireSys(p) : ldAcquireGpu(p)) >= target) return true;
+    if ((it & 1023u) == 0) {
+      if (*(volatile uint32_t*)c.ra->abortFlag) return false;
+      if (globaltimer() - t0 > c.a->timeoutNs) {
+        raiseAbort(*c.a);
+        return false;
+      }
+    }
+  }
+}
+
+// ------------------------------------------------------------------ chunk geometry (reading R1)
+__device__ __forceinline__ void chunkSpan(const KernelArgs& a, int buf, int64_t k, int64_t& start, int64_t& len) {
+  if (buf == KB_SC) {
+    start = k * a.E;
+    len = a.E;
+    return;
+  }
+  int64_t b = k / a.cb, j = k - b * a.cb;
+  start = b * a.n + j * a.E;
+  int64_t rem = a.n - j * a.E;
+  len = rem < 0 ? 0 : (rem < a.E ? rem : a.E);
+}
+
+// ------------------------------------------------------------------ Simple-protocol piece
+// out = RECV&&SRC ? op(recv, src) : REDDST ? op(dst, src) : RECV ? recv : src
+// written to dst (DST) and/or the outgoing slot (SEND).
+template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
+__device__ __forceinline__ void pieceSimple(int64_t m, const char* rslot, const char* src, char* dst, char* sslot,
+                                            const Ctx& c) {
+  typedef typename DType<DT>::T T;
+  constexpr int V = 16 / sizeof(T);
+  constexpr int U = 4;
+  uintptr_t al = (uintptr_t)rslot | (uintptr_t)src | (uintptr_t)dst | (uintptr_t)sslot;
+  int64_t nvec = (al & 15) ? 0 : m / V;
+  const int nt = c.nt;
+  int64_t i = c.tid;
+  for (; i + (U - 1) * nt < nvec; i += U * nt) {
+    uint4 x[U], y[U];
+#pragma unroll
+    for (int u = 0; u < U; u++) {
+      if constexpr (RECV) x[u] = ldcg(rslot + (i + u * nt) * 16);
+      if constexpr (REDDST) x[u] = ldcg(dst + (i + u * nt) * 16);
+      if constexpr (SRC) y[u] = ldcg(src + (i + u * nt) * 16);
+    }
+#pragma unroll
+    for (int u = 0; u < U; u++) {
+      uint4 v;
+      if constexpr ((RECV && SRC) || REDDST) v = vop<DT, OP>(x[u], y[u]);
+      else if constexpr (RECV) v = x[u];
+      else v = y[u];
+      if constexpr (DST) stg(dst + (i + u * nt) * 16, v);
+      if constexpr (SEND) stg(sslot + (i + u * nt) * 16, v);
+    }
+  }
+  for (; i < nvec; i += nt) {
+    uint4 x, y, v;
+    if constexpr (RECV) x = ldcg(rslot + i * 16);
+    if constexpr (REDDST) x = ldcg(dst + i * 16);
+    if constexpr (SRC) y = ldcg(src + i * 16);
+    if constexpr ((RECV && SRC) || REDDST) v = vop<DT, OP>(x, y);
+    else if constexpr (RECV) v = x;
+    else v = y;
+    if constexpr (DST) stg(dst + i * 16, v);
+    if constexpr (SEND) stg(sslot + i * 16, v);
+  }
+  // scalar tail (ragged chunk end or unaligned buffers)
+  for (int64_t e = nvec * V + c.tid; e < m; e += nt) {
+    T x = 0, y = 0, v;
+    if constexpr (RECV) x = *(volatile const T*)(rslot + e * sizeof(T));
+    if constexpr (REDDST) x = *(volatile const T*)(dst + e * sizeof(T));
+    if constexpr (SRC) y = *(volatile const T*)(src + e * sizeof(T));
+    if constexpr ((RECV && SRC) || REDDST) v = DType<DT>::op(OP, x, y);
+    else if constexpr (RECV) v = x;
+    else v = y;
+    if constexpr (DST) *(volatile T*)(dst + e * sizeof(T)) = v;
+    if constexpr (SEND) *(volatile T*)(sslot + e * sizeof(T)) = v;
+  }
+}
+
+// ------------------------------------------------------------------ LL-protocol piece
+// Payload travels in 8-byte units inside 16-byte lines {lo32, flag, hi32, flag}.
+__device__ __forceinline__ uint64_t loadUnit(const char* p, int64_t bytes) {
+  if (bytes == 8 && (((uintptr_t)p) & 7) == 0) return *(volatile const uint64_t*)p;
+  uint64_t v = 0;
+  for (int64_t k = 0; k < bytes; k++) v |= (uint64_t)(*(volatile const uint8_t*)(p + k)) << (8 * k);
+  return v;
+}
+__device__ __forceinline__ void storeUnit(char* p, uint64_t v, int64_t bytes) {
+  if (bytes == 8 && (((uintptr_t)p) & 7) == 0) {
+    *(volatile uint64_t*)p = v;
+    return;
+  }
+  for (int64_t k = 0; k < bytes; k++) *(volatile uint8_t*)(p + k) = (uint8_t)(v >> (8 * k));
+}
+template <int DT, int OP>
+__device__ __forceinline__ uint64_t unitOp(uint64_t a, uint64_t b) {
+  typedef typename DType<DT>::T T;
+  T* x = reinterpret_cast<T*>(&a);
+  const T* y = reinterpret_cast<const T*>(&b);
+#pragma unroll
+  for (int i = 0; i < (int)(8 / sizeof(T)); i++) x[i] = DType<DT>::op(OP, x[i], y[i]);
+  return a;
+}
+
+template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
+__device__ __forceinline__ bool pieceLL(int64_t m, const char* rslot, const char* src, char* dst, char* sslot,
+                                        uint32_t rflag, uint32_t sflag, const Ctx& c) {
+  typedef typename DType<DT>::T T;
+  const int64_t bytes = m * (int64_t)sizeof(T);
+  const int64_t units = (bytes + 7) / 8;
+  bool ok = true;
+  for (int64_t u = c.tid; u < units; u += c.nt) {
+    int64_t off = u * 8;
+    int64_t nb = bytes - off < 8 ? bytes - off : 8;
+    uint64_t x = 0, y = 0, v;
+    if (RECV) {
+      const char* line = rslot + u * 16;
+      uint4 l = ldvol(line);
+      if (l.y != rflag || l.w != rflag) {
+        uint64_t t0 = globaltimer();
+        for (uint32_t it = 1;; it++) {
+          l = ldvol(line);
+          if (l.y == rflag && l.w == rflag) break;
+          if ((it & 1023u) == 0) {
+            if (*(volatile uint32_t*)c.ra->abortFlag) { ok = false; break; }
+            if (globaltimer() - t0 > c.a->timeoutNs) { raiseAbort(*c.a); ok = false; break; }
+          }
+        }
+        if (!ok) break;
+      }
+      x = (uint64_t)l.x | ((uint64_t)l.z << 32);
+    }
+    if (REDDST) x = loadUnit(dst + off, nb);
+    if (SRC) y = loadUnit(src + off, nb);
+    if constexpr ((RECV && SRC) || REDDST) v = unitOp<DT, OP>(x, y);
+    else if constexpr (RECV) v = x;
+    else v = y;
+    if (DST) storeUnit(dst + off, v, nb);
+    if (SEND) stvol(sslot + u * 16, make_uint4((uint32_t)v, sflag, (uint32_t)(v >> 32), sflag));
+  }
+  return ok;
+}
+
+// ------------------------------------------------------------------ one instruction, one tile
+template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
+__device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr& in, int t, uint64_t& sent,
+                                   uint64_t& recvd, volatile int* sAbort) {
+  const KernelArgs& a = *c.a;
+  const RankArgs& ra = *c.ra;
+  const bool ll = a.proto == 1;
+  bool ok = true;
+  if (RECV && !ll && c.tid == 0) ok = waitGE(tb.recvHead, recvd + 1, true, c);
+  // a free slot: at most `slots` messages posted and not yet consumed (§6.1)
+  if (SEND && c.tid == (RECV ? 32 : 0) && sent + 1 > (uint64_t)a.slots)
+    ok = ok && waitGE(tb.sendAck, sent + 1 - (uint64_t)a.slots, true, c);
+  if (!ok) *sAbort = 1;
+  if (RECV || SEND) {
+    __syncthreads();
+    if (*sAbort) return false;
+  }
+  const char* rslot = RECV ? tb.recvFifo + (int64_t)(recvd % (uint64_t)a.slots) * a.slotBytes : nullptr;
+  char* sslot = SEND ? tb.sendFifo + (int64_t)(sent % (uint64_t)a.slots) * a.slotBytes : nullptr;
+  const int64_t w = sizeof(typename DType<DT>::T);
+  const int64_t a0 = (int64_t)t * a.T;
+  for (int j = 0; j < in.cnt; j++) {
+    int64_t ss = 0, sl = INT64_MAX, ds = 0, dl = INT64_MAX;
+    if (SRC) chunkSpan(a, in.srcBuf, (int64_t)in.srcOff + j, ss, sl);
+    if (DST || REDDST) chunkSpan(a, in.dstBuf, (int64_t)in.dstOff + j, ds, dl);
+    int64_t L = sl < dl ? sl : dl;
+    int64_t hi = a0 + a.T < L ? a0 + a.T : L;
+    int64_t m = hi - a0;
+    if (m <= 0) continue;
+    const char* src = SRC ? ra.buf[in.srcBuf] + (ss + a0) * w : nullptr;
+    char* dst = (DST || REDDST) ? ra.buf[in.dstBuf] + (ds + a0) * w : nullptr;
+    if (!ll) {
+      pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, RECV ? rslot + j * a.T * w : nullptr, src, dst,
+                                                       SEND ? sslot + j * a.T * w : nullptr, c);
+    } else {
+      const int64_t lineOff = j * ((a.T * w + 7) / 8) * 16;
+      if (!pieceLL<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, RECV ? rslot + lineOff : nullptr, src, dst,
+                                                         SEND ? sslot + lineOff : nullptr, (uint32_t)(recvd + 1),
+                                                         (uint32_t)(sent + 1), c))
+        *sAbort = 1;
+    }
+  }
+  __syncthreads();
+  if (*sAbort) return false;
+  if (c.tid == 0 && (RECV || SEND)) {
+    if (a.sysScope) fenceSys();
+    else fenceGpu();
+    if (SEND && !ll) stRelaxedSys(tb.sendHead, sent + 1);
+    if (RECV) stRelaxedSys(tb.recvAck, recvd + 1);
+  }
+  if (SEND) sent++;
+  if (RECV) recvd++;
+  return true;
+}
+
+template <int DT, int OP>
+__device__ __forceinline__ bool dispatch(const Ctx& c, const DevTB& tb, const DevInstr& in, int t, uint64_t& sent,
+                                         uint64_t& recvd, volatile int* sAbort) {
+  switch (in.op) {  // Fig. 5 line 18; every case ends (the figure's fall-through is reading R10)
+    case K_SEND: return runOp<DT, OP, false, true, true, false, false>(c, tb, in, t, sent, recvd, sAbort);
+    case K_RECV: return runOp<DT, OP, true, false, false, true, false>(c, tb, in, t, sent, recvd, sAbort);
+    case K_COPY: return runOp<DT, OP, false, false, true, true, false>(c, tb, in, t, sent, recvd, sAbort);
+    case K_RCS: return runOp<DT, OP, true, true, false, true, false>(c, tb, in, t, sent, recvd, sAbort);
+    default: break;
+  }
+  if (OP != R_COPY) {
+    switch (in.op) {
+      case K_REDUCE: return runOp<DT, OP, false, false, true, true, true>(c, tb, in, t, sent, recvd, sAbort);
+      case K_RRC: return runOp<DT, OP, true, false, true, true, false>(c, tb, in, t, sent, recvd, sAbort);
+      case K_RRS: return runOp<DT, OP, true, true, true, false, false>(c, tb, in, t, sent, recvd, sAbort);
+      case K_RRCS: return runOp<DT, OP, true, true, true, true, false>(c, tb, in, t, sent, recvd, sAbort);
+      default: break;
+    }
+  }
+  return true;  // nop
+}
+
+#ifndef MSCCL_MAX_THREADS
+#define MSCCL_MAX_THREADS 512
+#endif
+
+template <int DT, int OP>
+__global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const __grid_constant__ KernelArgs a) {
+  __shared__ int sAbort;
+  int ls = 0;
+  for (int r = 1; r < a.nLocal; r++)
+    if ((int)blockIdx.x >= a.rank[r].ctaStart) ls = r;
+  const RankArgs& ra = a.rank[ls];
+  const int tbi = (int)blockIdx.x - ra.ctaStart;
+  if (tbi >= ra.nTB) return;
+  const DevTB& tb = ra.tbs[tbi];
+  Ctx c{&a, &ra, (int)threadIdx.x, (int)blockDim.x};
+  if (threadIdx.x == 0) sAbort = 0;
+  uint64_t sent = tb.sendFifo ? *(volatile uint64_t*)tb.sendCnt : 0;
+  uint64_t recvd = tb.recvFifo ? *(volatile uint64_t*)tb.recvCnt : 0;
+  const uint64_t gen = *(volatile uint64_t*)&ra.gen[tbi];
+  __syncthreads();
+  for (int t = 0; t < a.I; t++) {
+    for (int s = 0; s < tb.nSteps; s++) {
+      const DevInstr in = ra.instrs[tb.instrStart + s];
+      if (in.nDeps) {  // Fig. 5 lines 15-16; barrier after the waits (reading R10)
+        bool ok = true;
+        for (int d = c.tid; d < in.nDeps && ok; d += c.nt) {
+          uint32_t dep = ra.deps[in.depStart + d];
+          int dtb = (int)(dep >> 16), dstep = (int)(dep & 0xffff);
+          uint64_t target = (gen << 40) | ((uint64_t)t * (uint64_t)ra.tbs[dtb].nSteps + (uint64_t)dstep + 1);
+          ok = waitGE(&ra.sem[dtb], target, false, c);
+        }
+        if (!ok) sAbort = 1;
+        __syncthreads();
+        if (sAbort) return;
+      }
+      if (!dispatch<DT, OP>(c, tb, in, t, sent, recvd, &sAbort)) return;
+      if (in.hasDep) {  // Fig. 5 lines 25-27: the step is complete before the semaphore moves
+        if (c.tid == 0) {
+          fenceGpu();
+          stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)tb.nSteps + (uint64_t)s + 1));
+        }
+      }
+    }
+  }
+  if (threadIdx.x == 0) {
+    if (tb.sendFifo) *(volatile uint64_t*)tb.sendCnt = sent;
+    if (tb.recvFifo) *(volatile uint64_t*)tb.recvCnt = recvd;
+    *(volatile uint64_t*)&ra.gen[tbi] = gen + 1;
+  }
+}
+
+}  // namespace msccl

@@ -1,0 +1,183 @@
+// MSCCL-IR validator (DESIGN.md rules V2..V9). Runs on the host at mscclLoadProgram.
+//
+// V9 is an abstract execution of the program with counters only: each thread block walks
+// its instruction list once per pipeline iteration; a receive needs a posted message on
+// its connection, a send needs a free FIFO slot (at most `slots` outstanding, §6.1
+// P:L1313-1322), a dependency needs the named step done in the same iteration (Fig. 5
+// P:L1294-1307). No progress in a full sweep before completion = deadlock.
+#include <algorithm>
+#include <map>
+#include <sstream>
+#include <tuple>
+
+#include "ir.h"
+
+namespace msccl {
+
+int blocksOf(int coll, int buf, int R) {
+  if (buf == BUF_IN) return (coll == COLL_REDUCESCATTER || coll == COLL_ALLTOALL) ? R : 1;
+  if (buf == BUF_OUT) return (coll == COLL_ALLGATHER || coll == COLL_ALLTOALL) ? R : 1;
+  return 1;
+}
+
+namespace {
+
+[[noreturn]] void fail(const char* rule, const std::string& msg) { throw IRError(std::string(rule) + ": " + msg); }
+
+std::string where(int g, int tb, int s = -1) {
+  std::ostringstream o;
+  o << "rank " << g << " tb " << tb;
+  if (s >= 0) o << " step " << s;
+  return o.str();
+}
+
+typedef std::tuple<int, int, int> ConnKey;  // (src, dst, chan)
+
+void deadlockCheck(const Algo& a, int slots, int iters) {
+  struct TBRef { int g, tb; long long done, total; };
+  std::vector<TBRef> tbs;
+  std::map<ConnKey, long long> posted, consumed;
+  for (auto& g : a.gpus)
+    for (auto& tb : g.tbs) tbs.push_back({g.id, tb.id, 0, (long long)tb.steps.size() * iters});
+  std::map<std::pair<int, int>, long long*> prog;
+  for (auto& r : tbs) prog[{r.g, r.tb}] = &r.done;
+  for (;;) {
+    bool progressed = false, finished = true;
+    for (auto& r : tbs) {
+      const ThreadBlock& tb = a.gpus[r.g].tbs[r.tb];
+      long long n = (long long)tb.steps.size();
+      while (r.done < r.total) {
+        long long t = r.done / n;
+        const Instr& in = tb.steps[r.done % n];
+        OpRole ro = opRole(in.op);
+        bool ok = true;
+        for (auto& d : in.deps) {
+          long long dn = (long long)a.gpus[r.g].tbs[d.first].steps.size();
+          if (*prog[{r.g, d.first}] < t * dn + d.second + 1) { ok = false; break; }
+        }
+        ConnKey rk(tb.recv, r.g, tb.chan), sk(r.g, tb.send, tb.chan);
+        if (ok && ro.recv && posted[rk] <= consumed[rk]) ok = false;
+        if (ok && ro.send && posted[sk] - consumed[sk] >= slots) ok = false;
+        if (!ok) break;
+        if (ro.recv) consumed[rk]++;
+        if (ro.send) posted[sk]++;
+        r.done++;
+        progressed = true;
+      }
+      if (r.done < r.total) finished = false;
+    }
+    if (finished) return;
+    if (!progressed) {
+      std::ostringstream o;
+      o << "deadlock with " << slots << " FIFO slots:";
+      int shown = 0;
+      for (auto& r : tbs)
+        if (r.done < r.total && shown++ < 6) {
+          long long n = (long long)a.gpus[r.g].tbs[r.tb].steps.size();
+          o << " [" << where(r.g, r.tb, (int)(r.done % n)) << " iteration " << r.done / n << "]";
+        }
+      fail("V9", o.str());
+    }
+  }
+}
+
+}  // namespace
+
+void validateIR(Algo& a, int nranks, int slots, int maxTbs, int maxChannels, int iters) {
+  const int R = a.ngpus;
+  if (nranks > 0 && R != nranks) {
+    std::ostringstream o;
+    o << "program is for " << R << " ranks, communicator has " << nranks;
+    fail("V2", o.str());
+  }
+  if ((int)a.gpus.size() != R) fail("V2", "number of <gpu> elements differs from ngpus");
+  std::sort(a.gpus.begin(), a.gpus.end(), [](const GpuProgram& x, const GpuProgram& y) { return x.id < y.id; });
+  for (int i = 0; i < R; i++)
+    if (a.gpus[i].id != i) fail("V2", "gpu ids must be 0..ngpus-1");
+  const GpuProgram& g0 = a.gpus[0];
+  for (auto& g : a.gpus)
+    if (g.iChunks != g0.iChunks || g.oChunks != g0.oChunks) fail("V3", where(g.id, 0) + ": chunk counts differ from rank 0");
+  int ci = g0.iChunks, co = g0.oChunks;
+  bool ok = false;
+  switch (a.coll) {
+    case COLL_ALLREDUCE: ok = ci == co && ci >= 1; break;
+    case COLL_ALLGATHER: ok = co == R * ci && ci >= 1; break;
+    case COLL_REDUCESCATTER: ok = ci == R * co && co >= 1; break;
+    case COLL_ALLTOALL: ok = ci == co && ci >= R && ci % R == 0; break;
+    case COLL_CUSTOM: ok = ci == co && ci >= 1; break;
+  }
+  if (!ok) fail("V3", "chunk counts do not fit the collective");
+  if (a.inplace && a.coll != COLL_ALLREDUCE && a.coll != COLL_CUSTOM) fail("V3", "in-place programs are only defined for allreduce/custom");
+  if (a.proto == PROTO_LL128) fail("V1", "protocol LL128 is not implemented by this runtime");
+
+  std::map<ConnKey, std::pair<int, int>> senders, receivers;  // -> (gpu, tb)
+  for (auto& g : a.gpus) {
+    if ((int)g.tbs.size() > maxTbs) {
+      std::ostringstream o;
+      o << "rank " << g.id << " has " << g.tbs.size() << " thread blocks > " << maxTbs;
+      fail("V4", o.str());
+    }
+    std::sort(g.tbs.begin(), g.tbs.end(), [](const ThreadBlock& x, const ThreadBlock& y) { return x.id < y.id; });
+    for (size_t i = 0; i < g.tbs.size(); i++)
+      if (g.tbs[i].id != (int)i) fail("V1", where(g.id, (int)i) + ": thread block ids must be 0..n-1");
+    int nch[3] = {g.iChunks, g.oChunks, g.sChunks};
+    if (a.inplace) nch[BUF_OUT] = g.iChunks;
+    for (auto& tb : g.tbs) {
+      for (int p : {tb.send, tb.recv})
+        if (p != -1 && (p < 0 || p >= R || p == g.id)) fail("V4", where(g.id, tb.id) + ": bad peer");
+      if (tb.chan < 0 || tb.chan >= maxChannels) fail("V4", where(g.id, tb.id) + ": channel out of range");
+      if (tb.send >= 0) {
+        ConnKey k(g.id, tb.send, tb.chan);
+        if (senders.count(k)) fail("V5", where(g.id, tb.id) + ": connection has two sending thread blocks");
+        senders[k] = {g.id, tb.id};
+      }
+      if (tb.recv >= 0) {
+        ConnKey k(tb.recv, g.id, tb.chan);
+        if (receivers.count(k)) fail("V5", where(g.id, tb.id) + ": connection has two receiving thread blocks");
+        receivers[k] = {g.id, tb.id};
+      }
+      for (size_t s = 0; s < tb.steps.size(); s++) {
+        const Instr& in = tb.steps[s];
+        std::string w = where(g.id, tb.id, (int)s);
+        OpRole ro = opRole(in.op);
+        if (ro.send && tb.send < 0) fail("V6", w + ": instruction sends but the thread block has no send peer");
+        if (ro.recv && tb.recv < 0) fail("V6", w + ": instruction receives but the thread block has no receive peer");
+        if (in.op != OP_NOP && (in.cnt < 1 || in.cnt > 65535)) fail("V6", w + ": cnt out of range");
+        struct { bool used; int buf, off; } acc[2] = {{ro.src, in.srcBuf, in.srcOff}, {ro.dst, in.dstBuf, in.dstOff}};
+        for (auto& x : acc) {
+          if (!x.used) continue;
+          if (x.buf == BUF_NONE) fail("V6", w + ": missing buffer");
+          if (x.off < 0 || (long long)x.off + in.cnt > nch[x.buf]) fail("V6", w + ": chunk range exceeds the buffer");
+        }
+        if (ro.dst && in.dstBuf == BUF_IN && !a.inplace) fail("V3", w + ": out-of-place program writes the input buffer");
+        for (auto& d : in.deps) {
+          if (d.first == tb.id) fail("V8", w + ": depends on its own thread block");
+          if (d.first < 0 || d.first >= (int)g.tbs.size() || d.second < 0 ||
+              d.second >= (int)g.tbs[d.first].steps.size())
+            fail("V8", w + ": dependency names a missing step");
+          if (!g.tbs[d.first].steps[d.second].hasDep) fail("V8", w + ": dependency target does not set hasdep");
+        }
+      }
+    }
+  }
+  for (auto& kv : senders)
+    if (!receivers.count(kv.first)) fail("V5", "connection without a receiving thread block");
+  for (auto& kv : receivers)
+    if (!senders.count(kv.first)) fail("V5", "connection without a sending thread block");
+  for (auto& kv : senders) {
+    const ThreadBlock& st = a.gpus[kv.second.first].tbs[kv.second.second];
+    const auto& rv = receivers[kv.first];
+    const ThreadBlock& rt = a.gpus[rv.first].tbs[rv.second];
+    std::vector<int> sc, rc;
+    for (auto& in : st.steps)
+      if (opRole(in.op).send) sc.push_back(in.cnt);
+    for (auto& in : rt.steps)
+      if (opRole(in.op).recv) rc.push_back(in.cnt);
+    if (sc.size() != rc.size()) fail("V7", "connection: number of sends differs from number of receives");
+    for (size_t k = 0; k < sc.size(); k++)
+      if (sc[k] != rc[k]) fail("V7", "connection: k-th send and k-th receive carry different cnt");
+  }
+  deadlockCheck(a, slots, iters);
+}
+
+}  // namespace msccl

@@ -1,0 +1,94 @@
+"""CPU-side checks of the native library: it loads, exports every symbol include/msccl.h
+declares, and its C++ validator agrees with the independent Python validator of the
+oracle on valid programs and on every IR mutant (no compute calls: no GPU here)."""
+import os
+import re
+
+import pytest
+
+from oracle import irparse
+from oracle import validate as pyval
+from paper_conf_asplos_cowanmmsx23_b200 import programs as P
+
+import irmutate
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def rt():
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    return runtime
+
+
+def test_library_exports_every_declared_symbol(rt):
+    hdr = open(os.path.join(ROOT, "include", "msccl.h")).read()
+    names = set(re.findall(r"^(?:mscclResult_t|const char\*|uint64_t)\s+(msccl\w+)\(", hdr, re.M))
+    assert len(names) >= 25
+    for n in names:
+        assert hasattr(rt.lib, n), n
+    assert set(rt.SIGNATURES) == names
+
+
+def test_error_strings_and_params(rt):
+    assert rt.lib.mscclGetErrorString(8) == b"invalid MSCCL-IR program"
+    assert rt.get_param("MSCCL_SLOTS") >= 1
+    with pytest.raises(rt.MscclError):
+        rt.set_param("NOPE", 1)
+
+
+VALID = [
+    ("ring4", lambda: P.ring_allreduce(4), 4),
+    ("ring8ch", lambda: P.ring_allreduce(8, 8, 2), 8),
+    ("allpairs8", lambda: P.allpairs_allreduce(8), 8),
+    ("oneshot8", lambda: P.oneshot_allreduce(8), 8),
+    ("hier", lambda: P.hierarchical_allreduce(2, 3), 6),
+    ("ag", lambda: P.ring_allgather(4, 2, 2), 4),
+    ("rs", lambda: P.ring_reducescatter(8, 2, 1), 8),
+    ("a2a", lambda: P.alltoall_twostep(2, 4), 8),
+    ("a2n", lambda: P.alltonext(2, 3), 6),
+]
+
+
+@pytest.mark.parametrize("name,build,R", VALID, ids=[v[0] for v in VALID])
+def test_cpp_validator_accepts_shipped_programs(rt, name, build, R):
+    ok, msg = rt.validate(build().to_xml(), R, slots=2)
+    assert ok, msg
+
+
+@pytest.mark.parametrize("name,rule,text", irmutate.mutations(), ids=[m[0] for m in irmutate.mutations()])
+def test_cpp_and_python_validators_agree_on_mutants(rt, name, rule, text):
+    ok, msg = rt.validate(text, 4, slots=8)
+    assert not ok
+    assert msg.startswith(rule), msg
+    with pytest.raises((pyval.ValidationError, irparse.IRError)) as ei:
+        pyval.validate(irparse.parse(text), nranks=4, slots=8)
+    assert str(ei.value)[:2] == msg[:2]
+
+
+def test_cpp_deadlock_fixtures(rt):
+    ring1 = P.ring_allreduce(4, inplace=True).to_xml()
+    ok, msg = rt.validate(ring1, 4, slots=1)
+    assert not ok and msg.startswith("V9")
+    assert rt.validate(ring1, 4, slots=2)[0]
+    assert rt.validate(P.ring_allreduce(8, channels=8, inplace=True).to_xml(), 8, slots=1)[0]
+    ok, msg = rt.validate(irmutate.recv_before_send_ir(), 2, slots=8)
+    assert not ok and msg.startswith("V9")
+    text = irmutate.outstanding_sends_ir()
+    assert not rt.validate(text, 2, slots=2)[0]
+    assert rt.validate(text, 2, slots=3)[0]
+
+
+def test_cpp_thread_block_limit(rt):
+    over, text = irmutate.too_many_tbs(10)
+    ok, msg = rt.validate(text, 8, max_tbs=10)
+    assert not ok and msg.startswith("V4")
+
+
+def test_cpp_parser_rejects_malformed(rt):
+    for bad in ["", "<algo", "<gpu/>", '<algo name="x" coll="nope" ngpus="1" inplace="0"></algo>',
+                '<algo name="x" coll="allreduce" ngpus="1" inplace="0"><gpu id="0" i_chunks="1" o_chunks="1">'
+                '<tb id="0" send="-1" recv="-1" chan="0"><step s="0" type="zz" srcbuf="i" srcoff="0" dstbuf="o" '
+                'dstoff="0" cnt="1" depid="-1" deps="-1" hasdep="0"/></tb></gpu></algo>']:
+        ok, msg = rt.validate(bad, 1)
+        assert not ok and msg.startswith("V1"), (bad, msg)
