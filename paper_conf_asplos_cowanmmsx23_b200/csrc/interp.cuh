@@ -290,41 +290,51 @@ __device__ __forceinline__ uint64_t unitOp(uint64_t a, uint64_t b) {
   return a;
 }
 
+// Every LL piece message has exactly `sendUnits` lines: ceil(min(T, E - t*T) * w / 8), the
+// width of this tile of a FULL chunk, whatever the sender's own chunk length (reading R2:
+// a ragged in/out chunk may be received into a full-length scratch chunk, whose receiver
+// polls more lines than the sender has data for; the sender pads with zeros).
 template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
-__device__ __forceinline__ bool pieceLL(int64_t m, const char* rslot, const char* src, char* dst, char* sslot,
-                                        uint32_t rflag, uint32_t sflag, const Ctx& c) {
+__device__ __forceinline__ bool pieceLL(int64_t m, int64_t sendUnits, const char* rslot, const char* src, char* dst,
+                                        char* sslot, uint32_t rflag, uint32_t sflag, const Ctx& c) {
   typedef typename DType<DT>::T T;
-  const int64_t bytes = m * (int64_t)sizeof(T);
+  const int64_t bytes = m > 0 ? m * (int64_t)sizeof(T) : 0;
   const int64_t units = (bytes + 7) / 8;
+  const int64_t total = SEND ? (units > sendUnits ? units : sendUnits) : units;
   bool ok = true;
-  for (int64_t u = c.tid; u < units; u += c.nt) {
-    int64_t off = u * 8;
-    int64_t nb = bytes - off < 8 ? bytes - off : 8;
-    uint64_t x = 0, y = 0, v;
-    if (RECV) {
-      const char* line = rslot + u * 16;
-      uint4 l = ldvol(line);
-      if (l.y != rflag || l.w != rflag) {
-        uint64_t t0 = globaltimer();
-        for (uint32_t it = 1;; it++) {
-          l = ldvol(line);
-          if (l.y == rflag && l.w == rflag) break;
-          if ((it & 1023u) == 0) {
-            if (*(volatile uint32_t*)c.ra->abortFlag) { ok = false; break; }
-            if (globaltimer() - t0 > c.a->timeoutNs) { raiseAbort(*c.a); ok = false; break; }
+  for (int64_t u = c.tid; u < total; u += c.nt) {
+    const bool has = u < units;
+    const int64_t off = u * 8;
+    const int64_t nb = has ? (bytes - off < 8 ? bytes - off : 8) : 0;
+    uint64_t x = 0, y = 0, v = 0;
+    if constexpr (RECV) {
+      if (has) {
+        const char* line = rslot + u * 16;
+        uint4 l = ldvol(line);
+        if (l.y != rflag || l.w != rflag) {
+          uint64_t t0 = globaltimer();
+          for (uint32_t it = 1;; it++) {
+            l = ldvol(line);
+            if (l.y == rflag && l.w == rflag) break;
+            if ((it & 1023u) == 0) {
+              if (*(volatile uint32_t*)c.ra->abortFlag) { ok = false; break; }
+              if (globaltimer() - t0 > c.a->timeoutNs) { raiseAbort(*c.a); ok = false; break; }
+            }
           }
+          if (!ok) break;
         }
-        if (!ok) break;
+        x = (uint64_t)l.x | ((uint64_t)l.z << 32);
       }
-      x = (uint64_t)l.x | ((uint64_t)l.z << 32);
     }
-    if (REDDST) x = loadUnit(dst + off, nb);
-    if (SRC) y = loadUnit(src + off, nb);
-    if constexpr ((RECV && SRC) || REDDST) v = unitOp<DT, OP>(x, y);
-    else if constexpr (RECV) v = x;
-    else v = y;
-    if (DST) storeUnit(dst + off, v, nb);
-    if (SEND) stvol(sslot + u * 16, make_uint4((uint32_t)v, sflag, (uint32_t)(v >> 32), sflag));
+    if (has) {
+      if constexpr (REDDST) x = loadUnit(dst + off, nb);
+      if constexpr (SRC) y = loadUnit(src + off, nb);
+      if constexpr ((RECV && SRC) || REDDST) v = unitOp<DT, OP>(x, y);
+      else if constexpr (RECV) v = x;
+      else v = y;
+      if constexpr (DST) storeUnit(dst + off, v, nb);
+    }
+    if constexpr (SEND) stvol(sslot + u * 16, make_uint4((uint32_t)v, sflag, (uint32_t)(v >> 32), sflag));
   }
   return ok;
 }
@@ -357,16 +367,17 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
     int64_t L = sl < dl ? sl : dl;
     int64_t hi = a0 + a.T < L ? a0 + a.T : L;
     int64_t m = hi - a0;
-    if (m <= 0) continue;
     const char* src = SRC ? ra.buf[in.srcBuf] + (ss + a0) * w : nullptr;
     char* dst = (DST || REDDST) ? ra.buf[in.dstBuf] + (ds + a0) * w : nullptr;
     if (!ll) {
+      if (m <= 0) continue;
       pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, RECV ? rslot + j * a.T * w : nullptr, src, dst,
                                                        SEND ? sslot + j * a.T * w : nullptr, c);
     } else {
       const int64_t lineOff = j * ((a.T * w + 7) / 8) * 16;
-      if (!pieceLL<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, RECV ? rslot + lineOff : nullptr, src, dst,
-                                                         SEND ? sslot + lineOff : nullptr, (uint32_t)(recvd + 1),
+      const int64_t full = a.E - a0 < a.T ? a.E - a0 : a.T;
+      if (!pieceLL<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, (full * w + 7) / 8, RECV ? rslot + lineOff : nullptr, src,
+                                                         dst, SEND ? sslot + lineOff : nullptr, (uint32_t)(recvd + 1),
                                                          (uint32_t)(sent + 1), c))
         *sAbort = 1;
     }

@@ -524,8 +524,26 @@ class Program:
         heapq.heapify(heap)
         pos = 0
         last = {}
+        # a connection is a FIFO: its k-th receive must be the partner of its k-th send, so a
+        # ready receive waits until every earlier-scheduled send's receive is scheduled.
+        queue, deferred = {}, {}
+
+        def conn(x):
+            return (x.recv_from.rank, x.rank, x.ch)
+
         while heap:
             _, _, _, x = heapq.heappop(heap)
+            if x.recv_from is not None:
+                q = queue[conn(x)]
+                if q[0] is not x:
+                    deferred.setdefault(conn(x), set()).add(x)
+                    continue
+                q.pop(0)
+                if q and q[0] in deferred.get(conn(x), ()):
+                    deferred[conn(x)].discard(q[0])
+                    heapq.heappush(heap, (q[0].depth, -q[0].rdepth, q[0].seq, q[0]))
+            if x.send_to is not None:
+                queue.setdefault(conn(x.send_to), []).append(x.send_to)
             cands = [tb for tb in tbs[x.rank] if _fits(tb, x)]
             if not cands:
                 raise DSLError("rank %d: no thread block for %s" % (x.rank, x.op))
