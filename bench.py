@@ -1,0 +1,446 @@
+#!/usr/bin/env python3
+"""Benchmark of the MSCCL-IR interpreter (MSCCLang, ASPLOS '23) on B200.
+
+Metric (BASELINE.json): AllReduce / AllToAll bus bandwidth (nccl-tests convention,
+busBW = S/t * 2(R-1)/R for AllReduce, S = bytes per rank) — one JSON line on stdout.
+
+Workload of the default run (N=1, one GPU): BASELINE config 1 — ring AllReduce, bf16,
+8 channels, pipelined chunks — executed by R=8 VIRTUAL ranks on one B200 (all ranks'
+buffers and FIFOs in that GPU's HBM, one cooperative interpreter launch per step), at
+S = 256 MiB per rank (inputs 2 GiB > 126 MB L2, so no L2 flush is needed). With one GPU
+the "links" are HBM: the roofline is HBM bandwidth.
+
+Under torchrun (N>1) each process drives one GPU as one rank over CUDA IPC peer memory
+(NVLink/NVSwitch): ring AllReduce over N ranks, S per rank fixed ("weak"), value = busBW
+from the max over ranks of the CUDA-event time.
+
+`--impl reference` times the CPU oracle (oracle/sim.py) executing the same program on a
+bounded sample of the same workload, on the host cores.
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+MIB = 1 << 20
+SEED_SAMPLES = 4096
+
+
+def parse():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=20)
+    ap.add_argument("--warmup", type=int, default=5)
+    ap.add_argument("--impl", default="msccl", choices=["msccl", "reference"])
+    ap.add_argument("--ranks", type=int, default=8, help="virtual ranks when N=1")
+    ap.add_argument("--size-mib", type=float, default=256.0, help="bytes per rank (MiB)")
+    ap.add_argument("--program", default="ring", choices=["ring", "allpairs", "oneshot", "alltoall"])
+    ap.add_argument("--channels", type=int, default=1)
+    ap.add_argument("--instances", type=int, default=16)
+    ap.add_argument("--protocol", default="Simple")
+    ap.add_argument("--threads", type=int, default=512)
+    ap.add_argument("--slots", type=int, default=4)
+    ap.add_argument("--slot-kib", type=int, default=256)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu", action="store_true")
+    ap.add_argument("--quiet-extra", action="store_true")
+    return ap.parse_args()
+
+
+# ----------------------------------------------------------------------------- helpers
+def measured_peak():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        with open(p) as f:
+            return float(json.load(f)["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs)"
+    except Exception:
+        return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+def ncu_traffic():
+    """dram read+write bytes per launch of the interpreter, from the committed ncu summary."""
+    p = os.path.join(ROOT, "profiles", "ncu_summary.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return d.get("dram_bytes_per_launch"), d
+    except Exception:
+        return None, None
+
+
+class Clocks:
+    """nvidia-smi sampling during the timed region (B200_PROFILING.md clocks line)."""
+
+    def __init__(self, index=0):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=clocks.sm,clocks.max.sm,power.draw,"
+                 "clocks_event_reasons.active,clocks_event_reasons.hw_slowdown,"
+                 "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+                 "clocks_event_reasons.sw_power_cap", "--format=csv,noheader,nounits", "-lms", "100"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if not self.proc:
+            return None
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            f = [x.strip() for x in ln.split(",")]
+            if len(f) < 8:
+                continue
+            try:
+                sm.append(float(f[0]))
+                mx.append(float(f[1]))
+            except ValueError:
+                continue
+            for nm_, v in zip(names, f[4:8]):
+                if v.lower() == "active":
+                    reasons.add(nm_)
+        if not sm:
+            return None
+        return {"sm_mhz": statistics.median(sm), "sm_max_mhz": max(mx), "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def busbw(coll, S, t, R):
+    f = 2.0 * (R - 1) / R if coll == "allreduce" else (R - 1) / R
+    return S / t * f / 1e9
+
+
+def build_program(args, R):
+    from paper_conf_asplos_cowanmmsx23_b200 import programs as P
+    if args.program == "ring":
+        return P.ring_allreduce(R, channels=args.channels, instances=args.instances, protocol=args.protocol)
+    if args.program == "allpairs":
+        return P.allpairs_allreduce(R, instances=args.instances, protocol=args.protocol)
+    if args.program == "oneshot":
+        return P.oneshot_allreduce(R, instances=args.instances, protocol=args.protocol)
+    return P.alltoall_twostep(1, R, instances=args.instances, protocol=args.protocol)
+
+
+def simple_bytes_per_rank(algo, rank, S_per_chunk):
+    """Algorithmic HBM bytes of one launch for one rank under the FIFO protocol: each
+    instruction reads/writes its operands once per chunk."""
+    touches = {"s": 2, "r": 2, "cpy": 2, "re": 3, "rrc": 3, "rrs": 3, "rrcs": 4, "rcs": 3, "nop": 0}
+    g = algo.gpus[rank]
+    return sum(touches[st.op] * st.cnt for tb in g.tbs for st in tb.steps) * S_per_chunk
+
+
+# ----------------------------------------------------------------------------- CPU oracle
+def cpu_oracle_run(args, R, algo, sample_bytes, reps=3):
+    """Time oracle.sim.simulate on a bounded sample (same program, same dtype)."""
+    import numpy as np
+    import synth
+    from oracle import irparse, sim
+    dtype = "bfloat16"
+    n = int(sample_bytes // 2)
+    al = irparse.parse(algo.to_xml())
+    xs = [synth.hashed_numpy(q, np.arange(n), dtype) for q in range(R)]
+    times = []
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        sim.simulate(al, xs, n, dtype, "sum")
+        times.append(time.perf_counter() - t0)
+    t = statistics.median(times)
+    return {"value": round(busbw("allreduce", n * 2, t, R), 4), "unit": "GB/s", "cores": 1,
+            "host_cores": len(os.sched_getaffinity(0)), "kind": "oracle",
+            "sample": "ring AllReduce R=%d bf16, %d MiB per rank (median of %d runs of oracle.sim.simulate, "
+                      "numpy, 1 thread), %.2f s per run" % (R, n * 2 // MIB, reps, t)}
+
+
+def run_reference(args):
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    R = args.ranks if args.gpus == 1 else args.gpus
+    algo = build_program(args, R)
+    sample = 16 * MIB
+    import numpy as np
+    import synth
+    from oracle import irparse, sim
+    al = irparse.parse(algo.to_xml())
+    n = sample // 2
+    xs = [synth.hashed_numpy(q, np.arange(n), "bfloat16") for q in range(R)]
+    for _ in range(args.warmup):
+        sim.simulate(al, xs, n, "bfloat16", "sum")
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        sim.simulate(al, xs, n, "bfloat16", "sum")
+    t = (time.perf_counter() - t0) / args.steps
+    v = busbw("allreduce", sample, t, R)
+    cfg = config_dict(args, R, args.gpus)
+    out = {"impl": "reference", "metric": metric_name(), "value": round(v, 4), "unit": "GB/s",
+           "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 3),
+           "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
+           "config": cfg,
+           "cpu_baseline": {"value": round(v, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
+                            "host_cores": len(os.sched_getaffinity(0)),
+                            "sample": "oracle.sim.simulate of the same IR, %d MiB per rank per step" % (sample // MIB)},
+           "e2e": {"value": round(v, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(out), flush=True)
+
+
+def metric_name():
+    return "AllReduce busBW (GB/s), ring MSCCL-IR, bf16"
+
+
+def config_dict(args, R, N):
+    mode = "virtual ranks on 1 GPU" if N == 1 else "1 process per GPU, CUDA IPC peer memory"
+    return {"workload": "BASELINE config 1: ring AllReduce MSCCL-IR, %d channels, %d instances, %s protocol, "
+                        "%d ranks (%s), %d MiB per rank" % (args.channels, args.instances, args.protocol, R, mode,
+                                                            int(args.size_mib)),
+            "program": args.program, "ranks": R, "bytes_per_rank": int(args.size_mib * MIB),
+            "channels": args.channels, "instances": args.instances, "protocol": args.protocol,
+            "threads": args.threads, "slots": args.slots, "slot_bytes": args.slot_kib * 1024,
+            "l2": "inputs (%d MiB total) larger than L2 (126 MB); no flush" % int(args.size_mib * R),
+            "parallelism": "virtual%d" % R if N == 1 else "ranks%d" % N}
+
+
+# ----------------------------------------------------------------------------- GPU runs
+def set_params(rt, args):
+    rt.set_param("MSCCL_SLOTS", args.slots)
+    rt.set_param("MSCCL_SLOT_BYTES", args.slot_kib * 1024)
+    rt.set_param("MSCCL_THREADS", args.threads)
+    rt.set_param("MSCCL_MAX_CHANNELS", max(32, args.channels * args.instances))
+    rt.set_param("MSCCL_TIMEOUT_S", 30)
+
+
+def sampled_parity(algo, recv_list, n, ranks_to_check):
+    """Bit-exact check of sampled outputs against the oracle's reduction trees."""
+    import numpy as np
+    import torch
+    import synth
+    from oracle import irparse, sampled
+    al = irparse.parse(algo.to_xml())
+    g = np.random.default_rng(1)
+    idx = np.unique(np.concatenate([g.integers(0, n, SEED_SAMPLES), [0, n - 1, n // 2]]))
+    bad = 0
+    for q in ranks_to_check:
+        want = sampled.allreduce_at(al, lambda r, i: synth.hashed_numpy(r, i, "bfloat16"), n, "bfloat16", "sum",
+                                    idx, rank=q)
+        got = recv_list[q][torch.from_numpy(idx).to(recv_list[q].device)].view(torch.int16).cpu().numpy() \
+            .view(np.uint16)
+        bad += int(np.count_nonzero(got != want))
+    return bad, idx.size * len(ranks_to_check)
+
+
+def run_virtual(args):
+    import torch
+    import synth
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime as rt
+    R = args.ranks
+    set_params(rt, args)
+    algo = build_program(args, R)
+    ir_text = algo.to_xml()
+    S = int(args.size_mib * MIB)
+    n = S // 2
+    dev = torch.device("cuda:0")
+    comms = rt.Comm.virtual(R, 0)
+    for c in comms:
+        c.load(ir_text)
+    idx = torch.arange(n, device=dev, dtype=torch.int64)
+    send = [synth.hashed(q, idx, "bfloat16") for q in range(R)]
+    del idx
+    recv = [torch.empty(n, dtype=torch.bfloat16, device=dev) for _ in range(R)]
+    stream = torch.cuda.current_stream()
+
+    def step():
+        with rt.group():
+            for q in range(R):
+                comms[q].allreduce(send[q], recv[q], stream=stream)
+
+    for _ in range(args.warmup):
+        step()
+    torch.cuda.synchronize()
+    clocks = Clocks(0)
+    clocks.start()
+    time.sleep(0.3)
+    l0 = rt.launch_count()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    ev0.record(stream)
+    for _ in range(args.steps):
+        step()
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    t = ev0.elapsed_time(ev1) / 1e3 / args.steps
+    launches = rt.launch_count() - l0
+    clk = clocks.stop()
+    for c in comms:
+        if c.async_error():
+            raise RuntimeError("watchdog fired during the bench")
+    bad, total = sampled_parity(algo, recv, n, [0, R - 1])
+    res = {"t": t, "launches": launches, "clocks": clk, "parity_bad": bad, "parity_total": total,
+           "algo": algo, "S": S, "R": R}
+    # end-to-end through the public API with host buffers (pinned), every step
+    if not args.no_e2e:
+        host_in = [s.cpu().pin_memory() for s in send]
+        host_out = [torch.empty(n, dtype=torch.bfloat16).pin_memory() for _ in range(R)]
+        e2e_steps = max(2, min(5, args.steps))
+
+        def e2e_step():
+            for q in range(R):
+                send[q].copy_(host_in[q], non_blocking=True)
+            step()
+            for q in range(R):
+                host_out[q].copy_(recv[q], non_blocking=True)
+
+        e2e_step()
+        torch.cuda.synchronize()
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(e2e_steps):
+            e2e_step()
+        e1.record(stream)
+        torch.cuda.synchronize()
+        te = e0.elapsed_time(e1) / 1e3 / e2e_steps
+        res["e2e"] = {"value": round(busbw("allreduce", S, te, R), 3), "unit": "GB/s",
+                      "h2d_bytes_per_step": S * R, "d2h_bytes_per_step": S * R,
+                      "ms_per_step": round(te * 1e3, 3),
+                      "note": "C-ABI call with pinned host buffers: H2D of all %d ranks' inputs + AllReduce + "
+                              "D2H of all outputs per step (PCIe-bound)" % R}
+    for c in comms:
+        c.destroy()
+    return res
+
+
+def run_multi(args, rank, world, local_rank):
+    import torch
+    import torch.distributed as dist
+    import synth
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime as rt
+    torch.cuda.set_device(local_rank)
+    dist.init_process_group("nccl", rank=rank, world_size=world, device_id=torch.device("cuda", local_rank))
+    set_params(rt, args)
+    R = world
+    algo = build_program(args, R)
+    comm = rt.Comm.init_rank(R, rank, local_rank)
+    h = comm.export_handle()
+    handles = [None] * R
+    dist.all_gather_object(handles, h)
+    comm.connect(handles)
+    comm.load(algo.to_xml())
+    S = int(args.size_mib * MIB)
+    n = S // 2
+    dev = torch.device("cuda", local_rank)
+    send = synth.hashed(rank, torch.arange(n, device=dev, dtype=torch.int64), "bfloat16")
+    recv = torch.empty(n, dtype=torch.bfloat16, device=dev)
+    stream = torch.cuda.current_stream()
+    for _ in range(args.warmup):
+        comm.allreduce(send, recv, stream=stream)
+    torch.cuda.synchronize()
+    dist.barrier()
+    clocks = Clocks(local_rank) if rank == 0 else None
+    if clocks:
+        clocks.start()
+        time.sleep(0.3)
+    l0 = rt.launch_count()
+    ev0, ev1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    torch.cuda.synchronize()
+    dist.barrier()
+    ev0.record(stream)
+    for _ in range(args.steps):
+        comm.allreduce(send, recv, stream=stream)
+    ev1.record(stream)
+    torch.cuda.synchronize()
+    dist.barrier()
+    t = ev0.elapsed_time(ev1) / 1e3 / args.steps
+    tt = torch.tensor([t], device=dev, dtype=torch.float64)
+    dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+    t = float(tt.item())
+    launches = rt.launch_count() - l0
+    clk = clocks.stop() if clocks else None
+    # sampled parity on this rank
+    import numpy as np
+    from oracle import irparse, sampled
+    g = np.random.default_rng(1)
+    idx = np.unique(g.integers(0, n, SEED_SAMPLES))
+    want = sampled.allreduce_at(irparse.parse(algo.to_xml()), lambda r, i: synth.hashed_numpy(r, i, "bfloat16"),
+                                n, "bfloat16", "sum", idx, rank=rank)
+    got = recv[torch.from_numpy(idx).to(dev)].view(torch.int16).cpu().numpy().view(np.uint16)
+    bad = torch.tensor([int(np.count_nonzero(got != want))], device=dev)
+    dist.all_reduce(bad)
+    res = {"t": t, "launches": launches, "clocks": clk, "parity_bad": int(bad.item()),
+           "parity_total": idx.size * R, "algo": algo, "S": S, "R": R}
+    comm.destroy()
+    dist.destroy_process_group()
+    return res if rank == 0 else None
+
+
+def main():
+    args = parse()
+    if args.impl == "reference":
+        run_reference(args)
+        return
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    N = world if world > 1 else args.gpus
+    if world > 1:
+        res = run_multi(args, rank, world, local_rank)
+        if rank != 0:
+            return
+        R = world
+    else:
+        res = run_virtual(args)
+        R = args.ranks
+    S, t, algo = res["S"], res["t"], res["algo"]
+    value = busbw("allreduce", S, t, R)
+    peak, peak_src = measured_peak()
+    per_chunk = S / algo.gpus[0].i_chunks
+    nranks_launch = R if world == 1 else 1
+    alg_bytes = sum(simple_bytes_per_rank(algo, q, per_chunk) for q in range(R)) / R * nranks_launch
+    launches_per_step = max(1, res["launches"] // args.steps)
+    achieved = alg_bytes / t / 1e9
+    traffic, prof = ncu_traffic()
+    out = {
+        "metric": metric_name(), "value": round(value, 3), "unit": "GB/s", "n_gpus": N,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 4),
+        "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
+        "data": "synthetic (counter-based uniform[-1,1) bf16, seed 20230325+rank)",
+        "config": config_dict(args, R, N),
+        "frac_nvlink": round(value / 900.0, 4),
+        "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                     "frac": round(achieved / peak, 4), "traffic": traffic, "peak_source": peak_src,
+                     "kernel": "mscclInterpreter<bf16,sum>", "algorithmic_bytes_per_launch": int(alg_bytes),
+                     "launch_ms": round(t * 1e3 / launches_per_step, 4)},
+        "gpu_launches": res["launches"],
+        "parity": {"sampled_outputs": res["parity_total"], "mismatches": res["parity_bad"],
+                   "against": "oracle reduction trees (oracle/sampled.py), bit-exact"},
+        "clocks": res["clocks"],
+    }
+    if "e2e" in res:
+        out["e2e"] = res["e2e"]
+    if world == 1 and not args.no_cpu:
+        out["cpu_baseline"] = cpu_oracle_run(args, R, algo, 32 * MIB)
+    print(json.dumps(out), flush=True)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,41 @@
+"""Oracle values at sampled output positions (test / bench infrastructure).
+
+For sizes the simulator cannot run in seconds, the AllReduce result at an element e is
+still fixed by the program: the symbolic run (oracle/symbolic.py, §3.2) gives,
+for every output chunk k, its reduction tree over input chunks; element e of chunk k is
+that tree evaluated on element (e - k*E) of each leaf chunk, one rounding per (+)
+(reading R6). The chunk size E follows reading R1 (oracle/geometry.py).
+"""
+import numpy as np
+
+from . import numerics as nm
+from .geometry import Geometry
+from .symbolic import check
+
+
+def _eval(tree, leafval, op, dtype):
+    if tree[0] == "in":
+        return leafval(tree[1], tree[2])
+    _, a, b = tree
+    return nm.reduce(_eval(a, leafval, op, dtype), _eval(b, leafval, op, dtype), op, dtype)
+
+
+def allreduce_at(algo, value_at, count, dtype, op, idx, rank=0):
+    """Output of `rank` at element indices `idx` (AllReduce programs).
+
+    value_at(q, indices) -> numpy array (storage dtype) of rank q's input at `indices`.
+    """
+    assert algo.coll == "allreduce"
+    trees = check(algo)
+    geo = Geometry(algo, count, nm.elem_bytes(dtype))
+    idx = np.asarray(idx, dtype=np.int64)
+    out = np.empty(idx.size, dtype=nm.storage(dtype))
+    k_of = idx // geo.E
+    for k in np.unique(k_of):
+        sel = np.nonzero(k_of == k)[0]
+        pos = idx[sel] - k * geo.E
+
+        def leaf(q, kk, pos=pos):
+            return value_at(q, kk * geo.E + pos)
+        out[sel] = _eval(trees[rank][int(k)], leaf, op, dtype)
+    return out

@@ -57,3 +57,34 @@ def rank_input(rank, n, dtype, dist="uniform", seed=SEED):
 def inputs(R, n, dtype, dist="uniform", seed=SEED):
     """Per-rank input buffers (n elements each) for ranks 0..R-1."""
     return [rank_input(r, n, dtype, dist, seed) for r in range(R)]
+
+
+# ---------------------------------------------------------------------------------------
+# Counter-based generator: value(rank, i) is a pure function of (seed, rank, i), so the GPU
+# can fill multi-GiB buffers directly while the oracle evaluates any sampled index on the
+# host with the same integer arithmetic (torch int64 ops, identical on CPU and CUDA).
+def _mix32(x):
+    x = ((x ^ (x >> 16)) * 0x45D9F3B) & 0xFFFFFFFF
+    x = ((x ^ (x >> 16)) * 0x45D9F3B) & 0xFFFFFFFF
+    return x ^ (x >> 16)
+
+
+def hashed(rank, idx, dtype, seed=SEED):
+    """uniform[-1, 1) (24-bit grid, exact in fp32) cast RNE to `dtype`, for int64 index
+    tensor `idx` (any device). Returns a torch tensor of `dtype` on idx's device."""
+    import torch
+    key = (idx + rank * 0x01000193 + seed) & 0xFFFFFFFF
+    h = _mix32(_mix32(key) ^ 0x5BD1E995)
+    u = (h >> 8).to(torch.float32) * (2.0 ** -23) - 1.0
+    tdt = {"bfloat16": torch.bfloat16, "float16": torch.float16, "float32": torch.float32,
+           "float64": torch.float64}[dtype]
+    return u.to(tdt)
+
+
+def hashed_numpy(rank, idx, dtype, seed=SEED):
+    """Host copy of `hashed` at numpy indices, in the dtype's numpy storage type."""
+    import torch
+    t = hashed(rank, torch.from_numpy(np.asarray(idx, dtype=np.int64)), dtype, seed)
+    if dtype == "bfloat16":
+        return t.view(torch.int16).numpy().view(np.uint16)
+    return t.numpy()
