@@ -47,7 +47,7 @@ def parse():
     ap.add_argument("--protocol", default="Simple")
     ap.add_argument("--threads", type=int, default=512)
     ap.add_argument("--slots", type=int, default=4)
-    ap.add_argument("--slot-kib", type=int, default=256)
+    ap.add_argument("--slot-kib", type=int, default=512)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
     ap.add_argument("--quiet-extra", action="store_true")

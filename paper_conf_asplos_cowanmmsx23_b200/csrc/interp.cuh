@@ -34,6 +34,10 @@ enum { DT_I8 = 0, DT_U8 = 1, DT_I32 = 2, DT_U32 = 3, DT_I64 = 4, DT_U64 = 5, DT_
 enum { K_NOP = 0, K_SEND = 1, K_RECV = 2, K_COPY = 3, K_REDUCE = 4, K_RRC = 5, K_RRS = 6, K_RRCS = 7, K_RCS = 8 };
 enum { KB_IN = 0, KB_OUT = 1, KB_SC = 2 };
 
+struct V32 {  // 32-byte vector (one 256-bit LDG/STG on sm_100)
+  uint4 a, b;
+};
+
 // ------------------------------------------------------------------ element types
 template <int DT> struct DType;
 #define MSCCL_INT_DTYPE(ID, S, U)                                                          \
@@ -125,6 +129,11 @@ __device__ __forceinline__ uint4 vop(uint4 a, uint4 b) {
   return a;
 }
 
+template <int DT, int OP>
+__device__ __forceinline__ V32 vop(V32 a, V32 b) {
+  return V32{vop<DT, OP>(a.a, b.a), vop<DT, OP>(a.b, b.b)};
+}
+
 // ------------------------------------------------------------------ memory primitives
 __device__ __forceinline__ uint4 ldcg(const void* p) {
   uint4 v;
@@ -134,6 +143,53 @@ __device__ __forceinline__ uint4 ldcg(const void* p) {
 __device__ __forceinline__ void stg(void* p, uint4 v) {
   asm volatile("st.global.v4.u32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z), "r"(v.w) : "memory");
 }
+// L2 cache policies: user input/output streams are touched once (evict_first); FIFO
+// slots are written by the sender and read soon after by the receiver (evict_last), then
+// discarded from L2 by the receiver so the dead slot is never written back to HBM.
+__device__ __forceinline__ uint64_t policyEvictFirst() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+__device__ __forceinline__ uint64_t policyEvictLast() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+template <int VB> struct VecT;
+template <> struct VecT<16> { typedef uint4 T; };
+template <> struct VecT<32> { typedef V32 T; };
+
+// stream loads (user buffers): L1 bypass, L2 evict-first
+__device__ __forceinline__ void ldStream(uint4& v, const void* p, uint64_t pol) {
+  asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v4.u32 {%0,%1,%2,%3}, [%4], %5;"
+               : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void ldStream(V32& v, const void* p, uint64_t pol) {
+  asm volatile("ld.global.L1::no_allocate.L2::cache_hint.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8], %9;"
+               : "=r"(v.a.x), "=r"(v.a.y), "=r"(v.a.z), "=r"(v.a.w), "=r"(v.b.x), "=r"(v.b.y), "=r"(v.b.z),
+                 "=r"(v.b.w) : "l"(p), "l"(pol) : "memory");
+}
+// FIFO loads: L2 only (the slot is rewritten by a peer between uses; never trust L1)
+__device__ __forceinline__ void ldFifo(uint4& v, const void* p) {
+  asm volatile("ld.global.cg.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
+}
+__device__ __forceinline__ void ldFifo(V32& v, const void* p) {
+  asm volatile("ld.global.cg.v8.u32 {%0,%1,%2,%3,%4,%5,%6,%7}, [%8];"
+               : "=r"(v.a.x), "=r"(v.a.y), "=r"(v.a.z), "=r"(v.a.w), "=r"(v.b.x), "=r"(v.b.y), "=r"(v.b.z),
+                 "=r"(v.b.w) : "l"(p) : "memory");
+}
+__device__ __forceinline__ void stHint(void* p, const uint4& v, uint64_t pol) {
+  asm volatile("st.global.L2::cache_hint.v4.u32 [%0], {%1,%2,%3,%4}, %5;" ::"l"(p), "r"(v.x), "r"(v.y), "r"(v.z),
+               "r"(v.w), "l"(pol) : "memory");
+}
+__device__ __forceinline__ void stHint(void* p, const V32& v, uint64_t pol) {
+  asm volatile("st.global.L2::cache_hint.v8.u32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8}, %9;" ::"l"(p), "r"(v.a.x),
+               "r"(v.a.y), "r"(v.a.z), "r"(v.a.w), "r"(v.b.x), "r"(v.b.y), "r"(v.b.z), "r"(v.b.w), "l"(pol)
+               : "memory");
+}
+__device__ __forceinline__ void discardL2(const void* p) { asm volatile("discard.global.L2 [%0], 128;" ::"l"(p) : "memory"); }
+
 __device__ __forceinline__ uint4 ldvol(const void* p) {
   uint4 v;
   asm volatile("ld.volatile.global.v4.u32 {%0,%1,%2,%3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
@@ -212,47 +268,89 @@ __device__ __forceinline__ void chunkSpan(const KernelArgs& a, int buf, int64_t 
 // ------------------------------------------------------------------ Simple-protocol piece
 // out = RECV&&SRC ? op(recv, src) : REDDST ? op(dst, src) : RECV ? recv : src
 // written to dst (DST) and/or the outgoing slot (SEND).
+#ifndef MSCCL_UNROLL
+#define MSCCL_UNROLL 4
+#endif
+
+// Main vector loop: VB-byte vectors, U independent vectors in flight per thread.
+// Returns the number of VB-byte vectors processed.
+template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST, int VB>
+__device__ __forceinline__ int64_t vecLoop(int64_t nvec, const char* rslot, const char* src, char* dst, char* sslot,
+                                           const Ctx& c) {
+  typedef typename VecT<VB>::T Vec;
+  constexpr int U = MSCCL_UNROLL;
+  const uint64_t pFirst = policyEvictFirst(), pLast = policyEvictLast();
+  const int nt = c.nt;
+  const bool canDiscard = RECV && ((((uintptr_t)rslot) & 127) == 0);
+  const int lane = c.tid & 31, warp = c.tid >> 5, nw = nt >> 5;
+  // Full blocks of U x 32 vectors, one block per warp-iteration (warp-uniform trip count,
+  // so the __syncwarp below is reached by every lane); each u-row is 32 x VB contiguous bytes.
+  const int64_t nblk = nvec / (U * 32);
+  for (int64_t blk = warp; blk < nblk; blk += nw) {
+    const int64_t base = blk * (U * 32) + lane;
+    Vec x[U], y[U];
+#pragma unroll
+    for (int u = 0; u < U; u++) {
+      if constexpr (RECV) ldFifo(x[u], rslot + (base + u * 32) * VB);
+      if constexpr (REDDST) ldStream(x[u], dst + (base + u * 32) * VB, pFirst);
+      if constexpr (SRC) ldStream(y[u], src + (base + u * 32) * VB, pFirst);
+    }
+#pragma unroll
+    for (int u = 0; u < U; u++) {
+      Vec v;
+      if constexpr ((RECV && SRC) || REDDST) v = vop<DT, OP>(x[u], y[u]);
+      else if constexpr (RECV) v = x[u];
+      else v = y[u];
+      if constexpr (DST) stHint(dst + (base + u * 32) * VB, v, pFirst);
+      if constexpr (SEND) stHint(sslot + (base + u * 32) * VB, v, pLast);
+    }
+    if constexpr (RECV) {
+      // every lane's loads of this block have been consumed: drop the dead slot lines
+      __syncwarp();
+      if (canDiscard && ((lane * VB) & 127) == 0) {
+#pragma unroll
+        for (int u = 0; u < U; u++) discardL2(rslot + (base + u * 32) * VB);
+      }
+    }
+  }
+  for (int64_t i = nblk * (U * 32) + c.tid; i < nvec; i += nt) {
+    Vec x, y, v;
+    if constexpr (RECV) ldFifo(x, rslot + i * VB);
+    if constexpr (REDDST) ldStream(x, dst + i * VB, pFirst);
+    if constexpr (SRC) ldStream(y, src + i * VB, pFirst);
+    if constexpr ((RECV && SRC) || REDDST) v = vop<DT, OP>(x, y);
+    else if constexpr (RECV) v = x;
+    else v = y;
+    if constexpr (DST) stHint(dst + i * VB, v, pFirst);
+    if constexpr (SEND) stHint(sslot + i * VB, v, pLast);
+  }
+  return nvec;
+}
+
+// ------------------------------------------------------------------ Simple-protocol piece
+// out = RECV&&SRC ? op(recv, src) : REDDST ? op(dst, src) : RECV ? recv : src
+// written to dst (DST) and/or the outgoing slot (SEND).
 template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
 __device__ __forceinline__ void pieceSimple(int64_t m, const char* rslot, const char* src, char* dst, char* sslot,
                                             const Ctx& c) {
   typedef typename DType<DT>::T T;
-  constexpr int V = 16 / sizeof(T);
-  constexpr int U = 4;
+  const int64_t bytes = m * (int64_t)sizeof(T);
   uintptr_t al = (uintptr_t)rslot | (uintptr_t)src | (uintptr_t)dst | (uintptr_t)sslot;
-  int64_t nvec = (al & 15) ? 0 : m / V;
-  const int nt = c.nt;
-  int64_t i = c.tid;
-  for (; i + (U - 1) * nt < nvec; i += U * nt) {
-    uint4 x[U], y[U];
-#pragma unroll
-    for (int u = 0; u < U; u++) {
-      if constexpr (RECV) x[u] = ldcg(rslot + (i + u * nt) * 16);
-      if constexpr (REDDST) x[u] = ldcg(dst + (i + u * nt) * 16);
-      if constexpr (SRC) y[u] = ldcg(src + (i + u * nt) * 16);
-    }
-#pragma unroll
-    for (int u = 0; u < U; u++) {
-      uint4 v;
-      if constexpr ((RECV && SRC) || REDDST) v = vop<DT, OP>(x[u], y[u]);
-      else if constexpr (RECV) v = x[u];
-      else v = y[u];
-      if constexpr (DST) stg(dst + (i + u * nt) * 16, v);
-      if constexpr (SEND) stg(sslot + (i + u * nt) * 16, v);
-    }
+  int64_t done = 0;  // bytes handled by the vector paths
+  if ((al & 31) == 0) {
+    done = 32 * vecLoop<DT, OP, RECV, SEND, SRC, DST, REDDST, 32>(bytes / 32, rslot, src, dst, sslot, c);
+  } else if ((al & 15) == 0) {
+    done = 16 * vecLoop<DT, OP, RECV, SEND, SRC, DST, REDDST, 16>(bytes / 16, rslot, src, dst, sslot, c);
   }
-  for (; i < nvec; i += nt) {
-    uint4 x, y, v;
-    if constexpr (RECV) x = ldcg(rslot + i * 16);
-    if constexpr (REDDST) x = ldcg(dst + i * 16);
-    if constexpr (SRC) y = ldcg(src + i * 16);
-    if constexpr ((RECV && SRC) || REDDST) v = vop<DT, OP>(x, y);
-    else if constexpr (RECV) v = x;
-    else v = y;
-    if constexpr (DST) stg(dst + i * 16, v);
-    if constexpr (SEND) stg(sslot + i * 16, v);
+  if ((al & 15) == 0 && bytes - done >= 16) {  // 16-byte remainder after the 32-byte path
+    const int64_t off = done;
+    const int64_t nv = (bytes - done) / 16;
+    done += 16 * vecLoop<DT, OP, RECV, SEND, SRC, DST, REDDST, 16>(
+                     nv, RECV ? rslot + off : nullptr, SRC ? src + off : nullptr, (DST || REDDST) ? dst + off : nullptr,
+                     SEND ? sslot + off : nullptr, c);
   }
   // scalar tail (ragged chunk end or unaligned buffers)
-  for (int64_t e = nvec * V + c.tid; e < m; e += nt) {
+  for (int64_t e = done / (int64_t)sizeof(T) + c.tid; e < m; e += c.nt) {
     T x = 0, y = 0, v;
     if constexpr (RECV) x = *(volatile const T*)(rslot + e * sizeof(T));
     if constexpr (REDDST) x = *(volatile const T*)(dst + e * sizeof(T));
@@ -347,10 +445,11 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
   const RankArgs& ra = *c.ra;
   const bool ll = a.proto == 1;
   bool ok = true;
-  if (RECV && !ll && c.tid == 0) ok = waitGE(tb.recvHead, recvd + 1, true, c);
+  const bool sys = a.sysScope != 0;  // virtual ranks on one GPU only need gpu-scope ordering
+  if (RECV && !ll && c.tid == 0) ok = waitGE(tb.recvHead, recvd + 1, sys, c);
   // a free slot: at most `slots` messages posted and not yet consumed (§6.1)
   if (SEND && c.tid == (RECV ? 32 : 0) && sent + 1 > (uint64_t)a.slots)
-    ok = ok && waitGE(tb.sendAck, sent + 1 - (uint64_t)a.slots, true, c);
+    ok = ok && waitGE(tb.sendAck, sent + 1 - (uint64_t)a.slots, sys, c);
   if (!ok) *sAbort = 1;
   if (RECV || SEND) {
     __syncthreads();
@@ -385,10 +484,15 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
   __syncthreads();
   if (*sAbort) return false;
   if (c.tid == 0 && (RECV || SEND)) {
-    if (a.sysScope) fenceSys();
-    else fenceGpu();
-    if (SEND && !ll) stRelaxedSys(tb.sendHead, sent + 1);
-    if (RECV) stRelaxedSys(tb.recvAck, recvd + 1);
+    if (sys) {
+      fenceSys();
+      if (SEND && !ll) stRelaxedSys(tb.sendHead, sent + 1);
+      if (RECV) stRelaxedSys(tb.recvAck, recvd + 1);
+    } else {
+      fenceGpu();
+      if (SEND && !ll) stRelaxedGpu(tb.sendHead, sent + 1);
+      if (RECV) stRelaxedGpu(tb.recvAck, recvd + 1);
+    }
   }
   if (SEND) sent++;
   if (RECV) recvd++;

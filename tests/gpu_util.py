@@ -8,10 +8,12 @@ _COMMS = {}
 
 
 def comms(R, device=0):
-    """Cached virtual-rank communicator set (one region allocation per R)."""
-    if R not in _COMMS:
-        _COMMS[R] = runtime.Comm.virtual(R, device)
-    return _COMMS[R]
+    """Cached virtual-rank communicator set (one region allocation per R and parameter set)."""
+    key = (R, device) + tuple(runtime.get_param(k) for k in ("MSCCL_SLOTS", "MSCCL_SLOT_BYTES", "MSCCL_THREADS",
+                                                              "MSCCL_MAX_CHANNELS", "MSCCL_TIMEOUT_S"))
+    if key not in _COMMS:
+        _COMMS[key] = runtime.Comm.virtual(R, device)
+    return _COMMS[key]
 
 
 def run_program(ir_text, inputs, count, dtype, op="sum", out_elems=None, inplace=False, device=0):

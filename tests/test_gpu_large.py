@@ -1,0 +1,82 @@
+"""GPU parity at production launch parameters (256 KiB slots, 512 threads, unrolled 256-bit
+vector loops, L2 discard of consumed FIFO lines) with partial last tiles and ragged
+chunks, plus sampled parity at the bench's full size (256 MiB per rank, 8 virtual ranks,
+1 channel x 16 instances) against the oracle's reduction trees (oracle/sampled.py)."""
+import numpy as np
+import pytest
+
+import synth
+from oracle import irparse, sampled, sim
+from paper_conf_asplos_cowanmmsx23_b200 import programs as P
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module", autouse=True)
+def production_params():
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    for k, v in (("MSCCL_SLOT_BYTES", 262144), ("MSCCL_SLOTS", 4), ("MSCCL_THREADS", 512),
+                 ("MSCCL_MAX_CHANNELS", 32), ("MSCCL_TIMEOUT_S", 10)):
+        runtime.set_param(k, v)
+    yield
+
+
+@pytest.mark.parametrize("r,extra", [(4, 12345), (3, 7), (2, 131072 * 2 + 999)])
+def test_ring_partial_tiles_default_slots(r, extra):
+    import gpu_util
+    R = 8
+    n = R * r * 131072 * 2 + extra
+    ir = P.ring_allreduce(R, instances=r).to_xml()
+    xs = synth.inputs(R, n, "bfloat16", "uniform")
+    want = sim.simulate(irparse.parse(ir), xs, n, "bfloat16", "sum")
+    got = gpu_util.run_program(ir, xs, n, "bfloat16", "sum")
+    for g, w in zip(got, want):
+        assert np.array_equal(g, w)
+
+
+def test_alltoall_and_allgather_default_slots():
+    import gpu_util
+    from oracle import mpi_ref
+    R, n = 8, 300001
+    xs = synth.inputs(R, R * n, "bfloat16", "pattern")
+    got = gpu_util.run_program(P.alltoall_twostep(1, R, 1).to_xml(), xs, n, "bfloat16", out_elems=R * n)
+    assert all(np.array_equal(g, e) for g, e in zip(got, mpi_ref.alltoall(xs, n)))
+    xs = synth.inputs(R, n, "int32", "pattern")
+    got = gpu_util.run_program(P.ring_allgather(R, 1, 4).to_xml(), xs, n, "int32", out_elems=R * n)
+    assert all(np.array_equal(g, e) for g, e in zip(got, mpi_ref.allgather(xs)))
+
+
+@pytest.mark.parametrize("instances", [16, 18])
+def test_bench_size_sampled_parity(instances):
+    """The bench workload (launch configuration of bench.py) at full size; outputs
+    sampled on every rank and compared bit-exactly with the oracle's reduction trees."""
+    import torch
+    import gpu_util
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    R, n = 8, (256 << 20) // 2
+    algo = P.ring_allreduce(R, instances=instances)
+    ir = algo.to_xml()
+    cs = gpu_util.comms(R)
+    progs = [c.load(ir) for c in cs]
+    try:
+        dev = torch.device("cuda:0")
+        idx = torch.arange(n, device=dev, dtype=torch.int64)
+        send = [synth.hashed(q, idx, "bfloat16") for q in range(R)]
+        del idx
+        recv = [torch.empty(n, dtype=torch.bfloat16, device=dev) for _ in range(R)]
+        for _ in range(2):
+            with runtime.group():
+                for q in range(R):
+                    cs[q].allreduce(send[q], recv[q])
+        torch.cuda.synchronize()
+        al = irparse.parse(ir)
+        g = np.random.default_rng(5)
+        sample = np.unique(np.concatenate([g.integers(0, n, 2048), [0, n - 1]]))
+        for q in range(R):
+            want = sampled.allreduce_at(al, lambda rr, i: synth.hashed_numpy(rr, i, "bfloat16"), n, "bfloat16", "sum",
+                                        sample, rank=q)
+            got = recv[q][torch.from_numpy(sample).to(dev)].view(torch.int16).cpu().numpy().view(np.uint16)
+            assert np.array_equal(got, want), "rank %d" % q
+    finally:
+        for c, p in zip(cs, progs):
+            c.unload(p)
