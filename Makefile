@@ -4,13 +4,14 @@ NVCC    ?= nvcc
 ARCH    ?= -gencode arch=compute_100a,code=sm_100a
 PKG     := paper_conf_asplos_cowanmmsx23_b200
 SRC     := $(PKG)/csrc
-OBJDIR  := build/obj
-NVFLAGS := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -Wall -Iinclude -I$(SRC)
+OBJDIR  ?= build/obj
+EXTRA   ?=
+NVFLAGS := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -Wall -Iinclude -I$(SRC) $(EXTRA)
 CXXSRCS := $(wildcard $(SRC)/*.cpp)
 CUSRCS  := $(wildcard $(SRC)/*.cu)
 OBJS    := $(patsubst $(SRC)/%.cpp,$(OBJDIR)/%.o,$(CXXSRCS)) $(patsubst $(SRC)/%.cu,$(OBJDIR)/%.o,$(CUSRCS))
 HDRS    := $(wildcard $(SRC)/*.h) $(wildcard $(SRC)/*.cuh) include/msccl.h
-LIB     := $(PKG)/libmsccl_b200.so
+LIB     ?= $(PKG)/libmsccl_b200.so
 
 all: $(LIB)
 

@@ -43,14 +43,14 @@ def parse():
     ap.add_argument("--size-mib", type=float, default=256.0, help="bytes per rank (MiB)")
     ap.add_argument("--program", default="ring", choices=["ring", "allpairs", "oneshot", "alltoall"])
     ap.add_argument("--channels", type=int, default=1)
-    ap.add_argument("--instances", type=int, default=16)
+    ap.add_argument("--instances", type=int, default=32)
     ap.add_argument("--protocol", default="Simple")
-    ap.add_argument("--threads", type=int, default=512)
+    ap.add_argument("--threads", type=int, default=256)
     ap.add_argument("--slots", type=int, default=4)
-    ap.add_argument("--slot-kib", type=int, default=512)
+    ap.add_argument("--slot-kib", type=int, default=256)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--quiet-extra", action="store_true")
+    ap.add_argument("--quiet-extra", action="store_true", help="skip the small-message and AllToAll extras")
     return ap.parse_args()
 
 
@@ -325,9 +325,99 @@ def run_virtual(args):
                       "ms_per_step": round(te * 1e3, 3),
                       "note": "C-ABI call with pinned host buffers: H2D of all %d ranks' inputs + AllReduce + "
                               "D2H of all outputs per step (PCIe-bound)" % R}
+    if not args.quiet_extra:
+        del send, recv
+        torch.cuda.empty_cache()
+        res["extras"] = virtual_extras(comms, R, stream)
     for c in comms:
         c.destroy()
     return res
+
+
+def _timed(fn, iters, stream, graph=True):
+    """Mean device time per call of fn(); CUDA-graph replay of `iters` calls when possible."""
+    import torch
+    fn()
+    torch.cuda.synchronize()
+    mode = "eager"
+    if graph:
+        try:
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=stream):
+                for _ in range(iters):
+                    fn()
+            g.replay()
+            torch.cuda.synchronize()
+            run = g.replay
+            mode = "cuda-graph"
+        except Exception:
+            torch.cuda.synchronize()
+            run = None
+    if mode == "eager":
+        def run():
+            for _ in range(iters):
+                fn()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    run()
+    torch.cuda.synchronize()
+    e0.record(stream)
+    for _ in range(5):
+        run()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    return e0.elapsed_time(e1) / 1e3 / (5 * iters), mode
+
+
+def virtual_extras(comms, R, stream):
+    """BASELINE configs 3 and 4 on the same virtual ranks: 1 KB AllReduce latency (LL
+    one-shot / two-shot / ring) and AllToAll busBW at 256 MiB per rank."""
+    import torch
+    import synth
+    from paper_conf_asplos_cowanmmsx23_b200 import programs as P
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime as rt
+    dev = torch.device("cuda:0")
+    out = {}
+    lat = {}
+    n = 512  # 1 KiB of fp16 per rank
+    send = [synth.hashed(q, torch.arange(n, device=dev), "float16") for q in range(R)]
+    recv = [torch.empty_like(x) for x in send]
+    for name, algo in (("oneshot_LL", P.oneshot_allreduce(R, protocol="LL")),
+                       ("allpairs_LL", P.allpairs_allreduce(R, protocol="LL")),
+                       ("ring_LL", P.ring_allreduce(R, protocol="LL"))):
+        progs = [c.load(algo.to_xml()) for c in comms]
+
+        def call():
+            with rt.group():
+                for q in range(R):
+                    comms[q].run(progs[q], send[q], recv[q], n, stream=stream)
+        try:
+            t, mode = _timed(call, 50, stream)
+            lat[name] = round(t * 1e6, 2)
+            lat["mode"] = mode
+        except Exception as e:
+            lat[name] = "error: %s" % str(e)[:120]
+        for c, p in zip(comms, progs):
+            c.unload(p)
+    out["allreduce_1KiB_fp16_latency_us"] = lat
+    # AllToAll (direct, N=1 two-step), 256 MiB per rank, bf16
+    S = 256 * MIB
+    n = S // 2
+    algo = P.alltoall_twostep(1, R)
+    progs = [c.load(algo.to_xml()) for c in comms]
+    send = [synth.hashed(q, torch.arange(n, device=dev), "bfloat16") for q in range(R)]
+    recv = [torch.empty_like(x) for x in send]
+
+    def a2a():
+        with rt.group():
+            for q in range(R):
+                comms[q].run(progs[q], send[q], recv[q], n // R, stream=stream)
+    t, mode = _timed(a2a, 3, stream, graph=False)
+    ok = all(torch.equal(recv[q].view(R, -1)[p], send[p].view(R, -1)[q]) for q in (0, R - 1) for p in range(R))
+    out["alltoall_bf16_256MiB"] = {"busbw_GBps": round(busbw("alltoall", S, t, R), 2), "ms": round(t * 1e3, 3),
+                                   "ctas": sum(p.info()["thread_blocks"] for p in progs), "bit_exact": bool(ok)}
+    for c, p in zip(comms, progs):
+        c.unload(p)
+    return out
 
 
 def run_multi(args, rank, world, local_rank):
@@ -340,11 +430,8 @@ def run_multi(args, rank, world, local_rank):
     set_params(rt, args)
     R = world
     algo = build_program(args, R)
-    comm = rt.Comm.init_rank(R, rank, local_rank)
-    h = comm.export_handle()
-    handles = [None] * R
-    dist.all_gather_object(handles, h)
-    comm.connect(handles)
+    from paper_conf_asplos_cowanmmsx23_b200 import dist as mdist
+    comm = mdist.init_from_process_group(local_rank)
     comm.load(algo.to_xml())
     S = int(args.size_mib * MIB)
     n = S // 2
@@ -437,6 +524,8 @@ def main():
     }
     if "e2e" in res:
         out["e2e"] = res["e2e"]
+    if "extras" in res:
+        out["extras"] = res["extras"]
     if world == 1 and not args.no_cpu:
         out["cpu_baseline"] = cpu_oracle_run(args, R, algo, 32 * MIB)
     print(json.dumps(out), flush=True)

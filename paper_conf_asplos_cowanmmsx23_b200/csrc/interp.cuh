@@ -268,6 +268,9 @@ __device__ __forceinline__ void chunkSpan(const KernelArgs& a, int buf, int64_t 
 // ------------------------------------------------------------------ Simple-protocol piece
 // out = RECV&&SRC ? op(recv, src) : REDDST ? op(dst, src) : RECV ? recv : src
 // written to dst (DST) and/or the outgoing slot (SEND).
+#ifndef MSCCL_FENCE_MODE
+#define MSCCL_FENCE_MODE 0
+#endif
 #ifndef MSCCL_UNROLL
 #define MSCCL_UNROLL 4
 #endif
@@ -489,9 +492,17 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
       if (SEND && !ll) stRelaxedSys(tb.sendHead, sent + 1);
       if (RECV) stRelaxedSys(tb.recvAck, recvd + 1);
     } else {
+#if MSCCL_FENCE_MODE == 1
+      if (SEND && !ll) asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(tb.sendHead), "l"(sent + 1) : "memory");
+      if (RECV) asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(tb.recvAck), "l"(recvd + 1) : "memory");
+#elif MSCCL_FENCE_MODE == 2
+      if (SEND && !ll) stRelaxedGpu(tb.sendHead, sent + 1);
+      if (RECV) stRelaxedGpu(tb.recvAck, recvd + 1);
+#else
       fenceGpu();
       if (SEND && !ll) stRelaxedGpu(tb.sendHead, sent + 1);
       if (RECV) stRelaxedGpu(tb.recvAck, recvd + 1);
+#endif
     }
   }
   if (SEND) sent++;

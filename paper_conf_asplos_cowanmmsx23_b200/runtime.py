@@ -12,7 +12,7 @@ import ctypes
 import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIBPATH = os.path.join(_HERE, "libmsccl_b200.so")
+LIBPATH = os.environ.get("MSCCL_LIB") or os.path.join(_HERE, "libmsccl_b200.so")
 
 if not os.path.exists(LIBPATH):
     raise ImportError("libmsccl_b200.so not built (run `make` or __graft_entry__.build()); "
