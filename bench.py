@@ -343,15 +343,16 @@ def _timed(fn, iters, stream, graph=True):
     if graph:
         try:
             g = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(g, stream=stream):
+            with torch.cuda.graph(g):
                 for _ in range(iters):
                     fn()
             g.replay()
             torch.cuda.synchronize()
             run = g.replay
             mode = "cuda-graph"
-        except Exception:
+        except Exception as e:
             torch.cuda.synchronize()
+            print("graph capture failed: %s" % e, file=sys.stderr)
             run = None
     if mode == "eager":
         def run():
@@ -389,7 +390,7 @@ def virtual_extras(comms, R, stream):
         def call():
             with rt.group():
                 for q in range(R):
-                    comms[q].run(progs[q], send[q], recv[q], n, stream=stream)
+                    comms[q].run(progs[q], send[q], recv[q], n)  # current stream (graph capture)
         try:
             t, mode = _timed(call, 50, stream)
             lat[name] = round(t * 1e6, 2)
