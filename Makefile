@@ -6,7 +6,7 @@ PKG     := paper_conf_asplos_cowanmmsx23_b200
 SRC     := $(PKG)/csrc
 OBJDIR  ?= build/obj
 EXTRA   ?=
-NVFLAGS := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -Wall -Iinclude -I$(SRC) $(EXTRA)
+NVFLAGS := $(ARCH) -O3 -lineinfo -std=c++17 -Xcompiler -fPIC -Xcompiler -Wall -diag-suppress 177 -Iinclude -I$(SRC) $(EXTRA)
 CXXSRCS := $(wildcard $(SRC)/*.cpp)
 CUSRCS  := $(wildcard $(SRC)/*.cu)
 OBJS    := $(patsubst $(SRC)/%.cpp,$(OBJDIR)/%.o,$(CXXSRCS)) $(patsubst $(SRC)/%.cu,$(OBJDIR)/%.o,$(CUSRCS))

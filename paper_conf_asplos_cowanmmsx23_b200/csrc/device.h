@@ -61,8 +61,9 @@ struct KernelArgs {
   int32_t proto;              // 0 Simple, 1 LL
   int64_t slotBytes;
   int32_t sysScope;           // 1 when any peer is another GPU
-  int32_t pad;
+  int32_t useTma;             // Simple protocol: bulk-copy (TMA) pipeline through shared memory
   uint64_t timeoutNs;
+  uint64_t* trace;            // MSCCL_TRACE builds: per-CTA phase times (ns), else null
 };
 
 }  // namespace msccl

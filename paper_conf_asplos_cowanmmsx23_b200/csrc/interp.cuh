@@ -223,10 +223,12 @@ __device__ __forceinline__ uint64_t globaltimer() {
 }
 
 // ------------------------------------------------------------------ watchdog + waits
+struct TmaState;  // tma_pipe.cuh (MSCCL_ENABLE_TMA builds)
 struct Ctx {
   const KernelArgs* a;
   const RankArgs* ra;
   int tid, nt;
+  TmaState* tma;  // shared-memory pipeline state (Simple protocol with TMA), or null
 };
 
 static __device__ __noinline__ void raiseAbort(const KernelArgs& a) {
@@ -268,6 +270,9 @@ __device__ __forceinline__ void chunkSpan(const KernelArgs& a, int buf, int64_t 
 // ------------------------------------------------------------------ Simple-protocol piece
 // out = RECV&&SRC ? op(recv, src) : REDDST ? op(dst, src) : RECV ? recv : src
 // written to dst (DST) and/or the outgoing slot (SEND).
+#ifndef MSCCL_TRACE
+#define MSCCL_TRACE 0
+#endif
 #ifndef MSCCL_FENCE_MODE
 #define MSCCL_FENCE_MODE 0
 #endif
@@ -366,8 +371,29 @@ __device__ __forceinline__ void pieceSimple(int64_t m, const char* rslot, const 
   }
 }
 
+#ifndef MSCCL_ENABLE_TMA
+#define MSCCL_ENABLE_TMA 0
+#endif
+#if MSCCL_ENABLE_TMA
+#include "tma_pipe.cuh"
+#endif
+
 // ------------------------------------------------------------------ LL-protocol piece
 // Payload travels in 8-byte units inside 16-byte lines {lo32, flag, hi32, flag}.
+// user-buffer units for LL128 (not concurrently written by peers): plain cached accesses
+__device__ __forceinline__ uint64_t loadUnitPlain(const char* p, int64_t bytes) {
+  if (bytes == 8 && (((uintptr_t)p) & 7) == 0) return *(const uint64_t*)p;
+  uint64_t v = 0;
+  for (int64_t k = 0; k < bytes; k++) v |= (uint64_t)(*(const uint8_t*)(p + k)) << (8 * k);
+  return v;
+}
+__device__ __forceinline__ void storeUnitPlain(char* p, uint64_t v, int64_t bytes) {
+  if (bytes == 8 && (((uintptr_t)p) & 7) == 0) {
+    *(uint64_t*)p = v;
+    return;
+  }
+  for (int64_t k = 0; k < bytes; k++) *(uint8_t*)(p + k) = (uint8_t)(v >> (8 * k));
+}
 __device__ __forceinline__ uint64_t loadUnit(const char* p, int64_t bytes) {
   if (bytes == 8 && (((uintptr_t)p) & 7) == 0) return *(volatile const uint64_t*)p;
   uint64_t v = 0;
@@ -440,16 +466,233 @@ __device__ __forceinline__ bool pieceLL(int64_t m, int64_t sendUnits, const char
   return ok;
 }
 
-// ------------------------------------------------------------------ one instruction, one tile
+// ------------------------------------------------------------------ LL128-protocol piece
+// 128-byte lines written by 8 lanes x 16 bytes in one warp store: lanes 0-6 carry 16 payload
+// bytes, lane 7 carries 8 payload bytes and the 64-bit flag (message sequence number), so a
+// line holds 120 payload bytes (LL128 sits between LL and Simple). A line is
+// read by the same 8 lanes in one warp load and accepted when its flag matches; no fence and
+// no separate head counter are needed. Lines per piece message: ceil(min(T, E - t*T)*w/120)
+// (the sender pads, reading R2).
+#ifndef MSCCL_LL128_UNROLL
+#define MSCCL_LL128_UNROLL 4
+#endif
 template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
+__device__ __forceinline__ bool pieceLL128(int64_t m, int64_t sendLines, const char* rslot, const char* src, char* dst,
+                                           char* sslot, uint64_t rflag, uint64_t sflag, const Ctx& c) {
+  typedef typename DType<DT>::T T;
+  constexpr int U = MSCCL_LL128_UNROLL;
+  const int64_t bytes = m > 0 ? m * (int64_t)sizeof(T) : 0;
+  const int64_t lines = (bytes + 119) / 120;
+  const int64_t total = SEND ? (lines > sendLines ? lines : sendLines) : lines;
+  const int lane = c.tid & 31, warp = c.tid >> 5, nw = c.nt >> 5;
+  const int g = lane & 7, sub = lane >> 3;
+  bool ok = true;
+  for (int64_t base = (int64_t)warp * 4 * U; base < total; base += (int64_t)nw * 4 * U) {
+    uint64_t x0[U], x1[U];
+    if constexpr (RECV) {
+      uint4 l[U];
+      uint64_t t0 = 0;
+      for (uint32_t it = 0;; it++) {
+        bool mine = true;
+#pragma unroll
+        for (int u = 0; u < U; u++) {
+          const int64_t L = base + u * 4 + sub;
+          if (L < lines) {
+            l[u] = ldvol(rslot + L * 128 + g * 16);
+            if (g == 7 && ((uint64_t)l[u].z | ((uint64_t)l[u].w << 32)) != rflag) mine = false;
+          }
+        }
+        if (__all_sync(0xffffffffu, mine)) break;
+        if ((it & 1023u) == 1023u) {
+          uint64_t now = globaltimer();
+          if (t0 == 0) t0 = now;
+          if (*(volatile uint32_t*)c.ra->abortFlag) { ok = false; break; }
+          if (now - t0 > c.a->timeoutNs) { raiseAbort(*c.a); ok = false; break; }
+        }
+      }
+      if (!ok) break;
+#pragma unroll
+      for (int u = 0; u < U; u++) {
+        x0[u] = (uint64_t)l[u].x | ((uint64_t)l[u].y << 32);
+        x1[u] = (uint64_t)l[u].z | ((uint64_t)l[u].w << 32);
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; u++) {
+      const int64_t L = base + u * 4 + sub;
+      if (L >= total) continue;
+      const int64_t po = L * 120 + g * 16;                 // payload offset of this lane
+      const int64_t lb = g == 7 ? 8 : 16;                  // payload bytes of this lane
+      int64_t nb = bytes - po;
+      nb = nb < 0 ? 0 : (nb > lb ? lb : nb);
+      const int64_t nb0 = nb > 8 ? 8 : nb, nb1 = nb - nb0;
+      uint64_t v0 = 0, v1 = 0;
+      if (nb > 0) {
+        uint64_t a0 = 0, a1 = 0, b0 = 0, b1 = 0;
+        if constexpr (RECV) {
+          a0 = x0[u];
+          a1 = x1[u];
+        }
+        if constexpr (REDDST) {
+          a0 = loadUnitPlain(dst + po, nb0);
+          if (nb1) a1 = loadUnitPlain(dst + po + 8, nb1);
+        }
+        if constexpr (SRC) {
+          b0 = loadUnitPlain(src + po, nb0);
+          if (nb1) b1 = loadUnitPlain(src + po + 8, nb1);
+        }
+        if constexpr ((RECV && SRC) || REDDST) {
+          v0 = unitOp<DT, OP>(a0, b0);
+          v1 = nb1 ? unitOp<DT, OP>(a1, b1) : 0;
+        } else if constexpr (RECV) {
+          v0 = a0;
+          v1 = a1;
+        } else {
+          v0 = b0;
+          v1 = b1;
+        }
+        if constexpr (DST) {
+          storeUnitPlain(dst + po, v0, nb0);
+          if (nb1) storeUnitPlain(dst + po + 8, v1, nb1);
+        }
+      }
+      if constexpr (SEND) {
+        if (g == 7) v1 = sflag;
+        stvol(sslot + L * 128 + g * 16, make_uint4((uint32_t)v0, (uint32_t)(v0 >> 32), (uint32_t)v1, (uint32_t)(v1 >> 32)));
+      }
+    }
+  }
+  return ok;
+}
+
+// ------------------------------------------------------------------ per-protocol piece loops
+#define MSCCL_PIECE_GEOM                                                                  \
+  const KernelArgs& a = *c.a;                                                             \
+  const RankArgs& ra = *c.ra;                                                             \
+  const int64_t w = sizeof(typename DType<DT>::T);                                        \
+  const int64_t a0 = (int64_t)t * a.T;
+
+// piece j of the instruction at tile t: element count m and src/dst pointers (reading R2)
+template <int DT, bool SRC, bool DST, bool REDDST>
+__device__ __forceinline__ int64_t pieceGeom(const Ctx& c, const DevInstr& in, int t, int j, const char*& src, char*& dst) {
+  MSCCL_PIECE_GEOM
+  int64_t ss = 0, sl = INT64_MAX, ds = 0, dl = INT64_MAX;
+  if (SRC) chunkSpan(a, in.srcBuf, (int64_t)in.srcOff + j, ss, sl);
+  if (DST || REDDST) chunkSpan(a, in.dstBuf, (int64_t)in.dstOff + j, ds, dl);
+  int64_t L = sl < dl ? sl : dl;
+  int64_t hi = a0 + a.T < L ? a0 + a.T : L;
+  src = SRC ? ra.buf[in.srcBuf] + (ss + a0) * w : nullptr;
+  dst = (DST || REDDST) ? ra.buf[in.dstBuf] + (ds + a0) * w : nullptr;
+  return hi - a0;
+}
+
+template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
+__device__ __noinline__ void movePiecesSimple(const Ctx& c, const DevInstr& in, int t, const char* rslot, char* sslot) {
+  MSCCL_PIECE_GEOM
+  (void)a0;
+  for (int j = 0; j < in.cnt; j++) {
+    const char* src;
+    char* dst;
+    const int64_t m = pieceGeom<DT, SRC, DST, REDDST>(c, in, t, j, src, dst);
+    if (m <= 0) continue;
+    pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, RECV ? rslot + j * a.T * w : nullptr, src, dst,
+                                                     SEND ? sslot + j * a.T * w : nullptr, c);
+  }
+}
+
+template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
+__device__ __noinline__ bool movePiecesLL(const Ctx& c, const DevInstr& in, int t, const char* rslot, char* sslot,
+                                          uint64_t rseq, uint64_t sseq) {
+  MSCCL_PIECE_GEOM
+  bool ok = true;
+  for (int j = 0; j < in.cnt; j++) {
+    const char* src;
+    char* dst;
+    const int64_t m = pieceGeom<DT, SRC, DST, REDDST>(c, in, t, j, src, dst);
+    const int64_t lineOff = j * ((a.T * w + 7) / 8) * 16;
+    const int64_t full = a.E - a0 < a.T ? a.E - a0 : a.T;
+    ok &= pieceLL<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, (full * w + 7) / 8, RECV ? rslot + lineOff : nullptr, src, dst,
+                                                      SEND ? sslot + lineOff : nullptr, (uint32_t)rseq, (uint32_t)sseq, c);
+  }
+  return ok;
+}
+
+template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
+__device__ __noinline__ bool movePiecesLL128(const Ctx& c, const DevInstr& in, int t, const char* rslot, char* sslot,
+                                             uint64_t rseq, uint64_t sseq) {
+  MSCCL_PIECE_GEOM
+  bool ok = true;
+  const int64_t linesPer = (a.T * w + 119) / 120;
+  const int64_t full = a.E - a0 < a.T ? a.E - a0 : a.T;
+  for (int j = 0; j < in.cnt; j++) {
+    const char* src;
+    char* dst;
+    const int64_t m = pieceGeom<DT, SRC, DST, REDDST>(c, in, t, j, src, dst);
+    ok &= pieceLL128<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, (full * w + 119) / 120,
+                                                         RECV ? rslot + j * linesPer * 128 : nullptr, src, dst,
+                                                         SEND ? sslot + j * linesPer * 128 : nullptr, rseq, sseq, c);
+  }
+  return ok;
+}
+
+#if MSCCL_ENABLE_TMA
+// TMA path; returns false (nothing moved) when a piece is not 16-byte aligned
+template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
+__device__ __noinline__ bool movePiecesTma(const Ctx& c, const DevInstr& in, int t, const char* rslot, char* sslot) {
+  MSCCL_PIECE_GEOM
+  (void)a0;
+  constexpr int MAXP = 8;
+  if (in.cnt > MAXP) return false;
+  TmaPiece ps[MAXP];
+  int64_t ms[MAXP];
+  bool aligned = true;
+  for (int j = 0; j < in.cnt; j++) {
+    const char* src;
+    char* dst;
+    int64_t m = pieceGeom<DT, SRC, DST, REDDST>(c, in, t, j, src, dst);
+    m = m > 0 ? m : 0;
+    ms[j] = m;
+    TmaPiece& p = ps[j];
+    p.inA = RECV ? rslot + j * a.T * w : (REDDST ? dst : src);
+    p.inB = (RECV && SRC) || REDDST ? src : nullptr;
+    p.out0 = DST ? dst : nullptr;
+    p.out1 = SEND ? sslot + j * a.T * w : nullptr;
+    p.bytes = (m * w) & ~(int64_t)15;
+    uintptr_t al = (uintptr_t)p.inA | (uintptr_t)p.inB | (uintptr_t)p.out0 | (uintptr_t)p.out1;
+    if (m > 0 && (al & 15)) aligned = false;
+  }
+  if (!aligned) return false;
+  tmaMessage<DT, OP, (RECV && SRC) || REDDST, MAXP>(*c.tma, ps, in.cnt, RECV, c.tid, c.nt);
+  for (int j = 0; j < in.cnt; j++) {  // < 16-byte tails of ragged pieces
+    const int64_t e0 = ps[j].bytes / w;
+    if (e0 >= ms[j]) continue;
+    const int64_t k = e0 * w;
+    const char* srcp = (RECV && SRC) || REDDST ? ps[j].inB : ps[j].inA;
+    pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(
+        ms[j] - e0, RECV ? ps[j].inA + k : nullptr, SRC ? srcp + k : nullptr,
+        (DST || REDDST) ? (REDDST ? (char*)ps[j].inA : ps[j].out0) + k : nullptr, SEND ? ps[j].out1 + k : nullptr, c);
+  }
+  return true;
+}
+
+#endif  // MSCCL_ENABLE_TMA
+
+// ------------------------------------------------------------------ one instruction, one tile
+template <int DT, int OP, int PROTO, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
 __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr& in, int t, uint64_t& sent,
                                    uint64_t& recvd, volatile int* sAbort) {
   const KernelArgs& a = *c.a;
   const RankArgs& ra = *c.ra;
-  const bool ll = a.proto == 1;
+  constexpr bool ll = PROTO != 0;  // LL / LL128: the flags travel inside the data lines
   bool ok = true;
   const bool sys = a.sysScope != 0;  // virtual ranks on one GPU only need gpu-scope ordering
+#if MSCCL_TRACE
+  uint64_t tr0 = c.tid == 0 ? globaltimer() : 0, tr1 = 0, tr2 = 0, tr3 = 0, tr4 = 0;
+#endif
   if (RECV && !ll && c.tid == 0) ok = waitGE(tb.recvHead, recvd + 1, sys, c);
+#if MSCCL_TRACE
+  if (c.tid == 0) tr1 = globaltimer();
+#endif
   // a free slot: at most `slots` messages posted and not yet consumed (§6.1)
   if (SEND && c.tid == (RECV ? 32 : 0) && sent + 1 > (uint64_t)a.slots)
     ok = ok && waitGE(tb.sendAck, sent + 1 - (uint64_t)a.slots, sys, c);
@@ -458,38 +701,37 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
     __syncthreads();
     if (*sAbort) return false;
   }
+#if MSCCL_TRACE
+  if (c.tid == 0) tr2 = globaltimer();
+#endif
   const char* rslot = RECV ? tb.recvFifo + (int64_t)(recvd % (uint64_t)a.slots) * a.slotBytes : nullptr;
   char* sslot = SEND ? tb.sendFifo + (int64_t)(sent % (uint64_t)a.slots) * a.slotBytes : nullptr;
-  const int64_t w = sizeof(typename DType<DT>::T);
-  const int64_t a0 = (int64_t)t * a.T;
-  for (int j = 0; j < in.cnt; j++) {
-    int64_t ss = 0, sl = INT64_MAX, ds = 0, dl = INT64_MAX;
-    if (SRC) chunkSpan(a, in.srcBuf, (int64_t)in.srcOff + j, ss, sl);
-    if (DST || REDDST) chunkSpan(a, in.dstBuf, (int64_t)in.dstOff + j, ds, dl);
-    int64_t L = sl < dl ? sl : dl;
-    int64_t hi = a0 + a.T < L ? a0 + a.T : L;
-    int64_t m = hi - a0;
-    const char* src = SRC ? ra.buf[in.srcBuf] + (ss + a0) * w : nullptr;
-    char* dst = (DST || REDDST) ? ra.buf[in.dstBuf] + (ds + a0) * w : nullptr;
-    if (!ll) {
-      if (m <= 0) continue;
-      pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, RECV ? rslot + j * a.T * w : nullptr, src, dst,
-                                                       SEND ? sslot + j * a.T * w : nullptr, c);
-    } else {
-      const int64_t lineOff = j * ((a.T * w + 7) / 8) * 16;
-      const int64_t full = a.E - a0 < a.T ? a.E - a0 : a.T;
-      if (!pieceLL<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, (full * w + 7) / 8, RECV ? rslot + lineOff : nullptr, src,
-                                                         dst, SEND ? sslot + lineOff : nullptr, (uint32_t)(recvd + 1),
-                                                         (uint32_t)(sent + 1), c))
-        *sAbort = 1;
-    }
+  // each protocol's data path is its own non-inlined function (separate register allocation)
+  if constexpr (!ll || (!RECV && !SEND)) {
+#if MSCCL_ENABLE_TMA
+    if (c.tma == nullptr || !movePiecesTma<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, in, t, rslot, sslot))
+#endif
+      movePiecesSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, in, t, rslot, sslot);
+  } else if constexpr (PROTO == 2) {
+    if (!movePiecesLL128<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, in, t, rslot, sslot, recvd + 1, sent + 1)) *sAbort = 1;
+  } else {
+    if (!movePiecesLL<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, in, t, rslot, sslot, recvd + 1, sent + 1)) *sAbort = 1;
   }
+#if MSCCL_TRACE
+  if (c.tid == 0) tr3 = globaltimer();
+#endif
   __syncthreads();
   if (*sAbort) return false;
-  if (c.tid == 0 && (RECV || SEND)) {
+#if MSCCL_TRACE
+  if (c.tid == 0) tr4 = globaltimer();
+#endif
+  if (c.tid == 0 && ll && RECV) {  // LL/LL128: data carried its own flags; the ack frees the slot
+    if (sys) stRelaxedSys(tb.recvAck, recvd + 1);
+    else stRelaxedGpu(tb.recvAck, recvd + 1);
+  } else if (c.tid == 0 && (RECV || SEND) && !ll) {
     if (sys) {
       fenceSys();
-      if (SEND && !ll) stRelaxedSys(tb.sendHead, sent + 1);
+      if (SEND) stRelaxedSys(tb.sendHead, sent + 1);
       if (RECV) stRelaxedSys(tb.recvAck, recvd + 1);
     } else {
 #if MSCCL_FENCE_MODE == 1
@@ -505,27 +747,39 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
 #endif
     }
   }
+#if MSCCL_TRACE
+  if (c.tid == 0 && a.trace) {
+    uint64_t* tr = a.trace + (size_t)blockIdx.x * 8;
+    uint64_t tr5 = globaltimer();
+    tr[0] += tr1 - tr0;  // waiting for the incoming head
+    tr[1] += tr2 - tr1;  // barrier (incl. the credit wait of thread 32)
+    tr[2] += tr3 - tr2;  // thread 0's own data work
+    tr[3] += tr4 - tr3;  // barrier after the data loop (slowest thread)
+    tr[4] += tr5 - tr4;  // fence + flag stores
+    tr[5] += 1;
+  }
+#endif
   if (SEND) sent++;
   if (RECV) recvd++;
   return true;
 }
 
-template <int DT, int OP>
+template <int DT, int OP, int PROTO>
 __device__ __forceinline__ bool dispatch(const Ctx& c, const DevTB& tb, const DevInstr& in, int t, uint64_t& sent,
                                          uint64_t& recvd, volatile int* sAbort) {
   switch (in.op) {  // Fig. 5 line 18; every case ends (the figure's fall-through is reading R10)
-    case K_SEND: return runOp<DT, OP, false, true, true, false, false>(c, tb, in, t, sent, recvd, sAbort);
-    case K_RECV: return runOp<DT, OP, true, false, false, true, false>(c, tb, in, t, sent, recvd, sAbort);
-    case K_COPY: return runOp<DT, OP, false, false, true, true, false>(c, tb, in, t, sent, recvd, sAbort);
-    case K_RCS: return runOp<DT, OP, true, true, false, true, false>(c, tb, in, t, sent, recvd, sAbort);
+    case K_SEND: return runOp<DT, OP, PROTO, false, true, true, false, false>(c, tb, in, t, sent, recvd, sAbort);
+    case K_RECV: return runOp<DT, OP, PROTO, true, false, false, true, false>(c, tb, in, t, sent, recvd, sAbort);
+    case K_COPY: return runOp<DT, OP, PROTO, false, false, true, true, false>(c, tb, in, t, sent, recvd, sAbort);
+    case K_RCS: return runOp<DT, OP, PROTO, true, true, false, true, false>(c, tb, in, t, sent, recvd, sAbort);
     default: break;
   }
   if (OP != R_COPY) {
     switch (in.op) {
-      case K_REDUCE: return runOp<DT, OP, false, false, true, true, true>(c, tb, in, t, sent, recvd, sAbort);
-      case K_RRC: return runOp<DT, OP, true, false, true, true, false>(c, tb, in, t, sent, recvd, sAbort);
-      case K_RRS: return runOp<DT, OP, true, true, true, false, false>(c, tb, in, t, sent, recvd, sAbort);
-      case K_RRCS: return runOp<DT, OP, true, true, true, true, false>(c, tb, in, t, sent, recvd, sAbort);
+      case K_REDUCE: return runOp<DT, OP, PROTO, false, false, true, true, true>(c, tb, in, t, sent, recvd, sAbort);
+      case K_RRC: return runOp<DT, OP, PROTO, true, false, true, true, false>(c, tb, in, t, sent, recvd, sAbort);
+      case K_RRS: return runOp<DT, OP, PROTO, true, true, true, false, false>(c, tb, in, t, sent, recvd, sAbort);
+      case K_RRCS: return runOp<DT, OP, PROTO, true, true, true, true, false>(c, tb, in, t, sent, recvd, sAbort);
       default: break;
     }
   }
@@ -536,9 +790,13 @@ __device__ __forceinline__ bool dispatch(const Ctx& c, const DevTB& tb, const De
 #define MSCCL_MAX_THREADS 512
 #endif
 
-template <int DT, int OP>
+template <int DT, int OP, int PROTO>
 __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const __grid_constant__ KernelArgs a) {
   __shared__ int sAbort;
+#if MSCCL_ENABLE_TMA
+  __shared__ TmaState sTma;
+  extern __shared__ __align__(128) uint8_t dynSmem[];
+#endif
   int ls = 0;
   for (int r = 1; r < a.nLocal; r++)
     if ((int)blockIdx.x >= a.rank[r].ctaStart) ls = r;
@@ -546,7 +804,25 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
   const int tbi = (int)blockIdx.x - ra.ctaStart;
   if (tbi >= ra.nTB) return;
   const DevTB& tb = ra.tbs[tbi];
-  Ctx c{&a, &ra, (int)threadIdx.x, (int)blockDim.x};
+  Ctx c{&a, &ra, (int)threadIdx.x, (int)blockDim.x, nullptr};
+#if MSCCL_ENABLE_TMA
+  if (a.useTma && PROTO == 0) {
+    c.tma = &sTma;
+    if (threadIdx.x == 0) {
+      sTma.A = dynSmem;
+      sTma.B = dynSmem + TMA_NST * TMA_CB;
+      sTma.full = reinterpret_cast<uint64_t*>(dynSmem + 2 * TMA_NST * TMA_CB);
+      sTma.comp = sTma.full + TMA_NST;
+      sTma.gc = 0;
+      for (int i = 0; i < TMA_NST; i++) {
+        mbarInit(&sTma.full[i], 1);
+        mbarInit(&sTma.comp[i], blockDim.x / 32 - 1);
+      }
+      // make the initialised barriers visible to the async proxy (TMA complete_tx)
+      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+  }
+#endif
   if (threadIdx.x == 0) sAbort = 0;
   uint64_t sent = tb.sendFifo ? *(volatile uint64_t*)tb.sendCnt : 0;
   uint64_t recvd = tb.recvFifo ? *(volatile uint64_t*)tb.recvCnt : 0;
@@ -567,7 +843,7 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
         __syncthreads();
         if (sAbort) return;
       }
-      if (!dispatch<DT, OP>(c, tb, in, t, sent, recvd, &sAbort)) return;
+      if (!dispatch<DT, OP, PROTO>(c, tb, in, t, sent, recvd, &sAbort)) return;
       if (in.hasDep) {  // Fig. 5 lines 25-27: the step is complete before the semaphore moves
         if (c.tid == 0) {
           fenceGpu();

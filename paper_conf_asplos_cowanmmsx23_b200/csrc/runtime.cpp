@@ -12,6 +12,7 @@
 #include <mutex>
 #include <sstream>
 #include <string>
+#include <tuple>
 #include <vector>
 
 #include "../../include/msccl.h"
@@ -25,7 +26,7 @@ using namespace msccl;
 namespace {
 
 struct Params {
-  int64_t slots = 4, slotBytes = 262144, maxChannels = 32, threads = 512, timeoutS = 20;
+  int64_t slots = 4, slotBytes = 262144, maxChannels = 32, threads = 512, timeoutS = 20, tma = 0;
 };
 
 std::mutex gMu;
@@ -40,6 +41,7 @@ int64_t* paramRef(Params& p, const std::string& k) {
   if (k == "MSCCL_MAX_CHANNELS") return &p.maxChannels;
   if (k == "MSCCL_THREADS") return &p.threads;
   if (k == "MSCCL_TIMEOUT_S") return &p.timeoutS;
+  if (k == "MSCCL_TMA") return &p.tma;
   return nullptr;
 }
 
@@ -47,7 +49,8 @@ Params currentParams() {
   std::lock_guard<std::mutex> g(gMu);
   if (!gEnvRead) {
     gEnvRead = true;
-    for (const char* k : {"MSCCL_SLOTS", "MSCCL_SLOT_BYTES", "MSCCL_MAX_CHANNELS", "MSCCL_THREADS", "MSCCL_TIMEOUT_S"}) {
+    for (const char* k : {"MSCCL_SLOTS", "MSCCL_SLOT_BYTES", "MSCCL_MAX_CHANNELS", "MSCCL_THREADS", "MSCCL_TIMEOUT_S",
+                          "MSCCL_TMA"}) {
       const char* v = getenv(k);
       if (v && *v) *paramRef(gParams, k) = atoll(v);
     }
@@ -167,7 +170,7 @@ mscclResult_t allocRegion(mscclComm* c) {
   c->peerBase[c->rank] = c->region;
   int nsm = 0, nb = 0;
   CUDACHECK(c, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, c->dev));
-  CUDACHECK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, interpreterKernel(9, 0), (int)c->prm.threads, 0));
+  CUDACHECK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, interpreterKernel(9, 0, 0), (int)c->prm.threads, 0));
   c->maxCoResident = nsm * nb;
   return mscclSuccess;
 }
@@ -181,6 +184,43 @@ void freeProgram(mscclProgram* p) {
   cudaFree(p->dSem);
   cudaFree(p->dScratch);
   delete p;
+}
+
+// Debug: per-CTA phase timers of MSCCL_TRACE builds (host-mapped; enabled by env MSCCL_TRACE)
+uint64_t* gTraceHost = nullptr;
+uint64_t* gTraceDev = nullptr;
+uint64_t* traceBuffer() {
+  static bool init = false;
+  if (!init) {
+    init = true;
+    const char* v = getenv("MSCCL_TRACE");
+    if (v && *v == '1' && cudaHostAlloc(&gTraceHost, 4096 * 8 * sizeof(uint64_t), cudaHostAllocMapped) == cudaSuccess) {
+      memset(gTraceHost, 0, 4096 * 8 * sizeof(uint64_t));
+      cudaHostGetDevicePointer((void**)&gTraceDev, gTraceHost, 0);
+    }
+  }
+  return gTraceDev;
+}
+
+// co-resident CTAs per device for (kernel, threads, dynamic smem); sets the smem attribute
+mscclResult_t coResident(mscclComm* c, const void* fn, int threads, int smem, int& out) {
+  static std::mutex mu;
+  static std::map<std::tuple<const void*, int, int, int>, int> cache;
+  std::lock_guard<std::mutex> g(mu);
+  auto key = std::make_tuple(fn, threads, smem, c->dev);
+  auto it = cache.find(key);
+  if (it != cache.end()) {
+    out = it->second;
+    return mscclSuccess;
+  }
+  DeviceGuard dg(c->dev);
+  if (smem > 48 * 1024) CUDACHECK(c, cudaFuncSetAttribute(fn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  int nsm = 0, nb = 0;
+  CUDACHECK(c, cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, c->dev));
+  CUDACHECK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, threads, smem));
+  out = nsm * nb;
+  cache[key] = out;
+  return mscclSuccess;
 }
 
 // ------------------------------------------------------------------ groups and launches
@@ -209,8 +249,11 @@ mscclResult_t geometry(mscclComm* c, const mscclProgram* p, int dtype, int64_t n
   g.cb = p->algo.gpus[0].iChunks / blocksOf(p->algo.coll, BUF_IN, R);
   int64_t e = (n + g.cb - 1) / g.cb;
   g.E = (e + V - 1) / V * V;
-  int64_t payload = p->algo.proto == PROTO_LL ? c->prm.slotBytes / 2 : c->prm.slotBytes;
-  int64_t t = payload / ((int64_t)p->maxCnt * w) / V * V;
+  int64_t t;
+  if (p->algo.proto == PROTO_LL128)  // whole 128-byte lines (120 payload bytes) per piece
+    t = (c->prm.slotBytes / 128 / p->maxCnt) * 120 / w / V * V;
+  else
+    t = (p->algo.proto == PROTO_LL ? c->prm.slotBytes / 2 : c->prm.slotBytes) / ((int64_t)p->maxCnt * w) / V * V;
   if (t < V) return setErr(c, mscclInvalidUsage, "FIFO slot too small for the program's largest count");
   g.T = std::min<int64_t>(t, g.E);
   g.I = (int)((g.E + g.T - 1) / g.T);
@@ -265,9 +308,10 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
     ka.T = g.T;
     ka.cb = g.cb;
     ka.slots = (int)c0->prm.slots;
-    ka.proto = p0->algo.proto == PROTO_LL ? 1 : 0;
+    ka.proto = p0->algo.proto == PROTO_LL ? 1 : (p0->algo.proto == PROTO_LL128 ? 2 : 0);
     ka.slotBytes = c0->prm.slotBytes;
     ka.timeoutNs = (uint64_t)c0->prm.timeoutS * 1000000000ull;
+    ka.trace = traceBuffer();
     int cta = 0;
     for (int i = 0; i < (int)v.size(); i++) {
       Call* cl = v[i];
@@ -292,20 +336,27 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
       if (cl->comm->sysScope) ka.sysScope = 1;
     }
     if (cta == 0) continue;
-    if (cta > c0->maxCoResident) {
+    const void* fn = p0->hasReduce ? interpreterKernel(v[0]->dtype, v[0]->op, ka.proto)
+                                   : copyKernel(elemBytes(v[0]->dtype), ka.proto);
+    ka.useTma = (ka.proto == 0 && c0->prm.tma && tmaSmemBytes() > 0) ? 1 : 0;
+    const int smem = ka.useTma ? tmaSmemBytes() : 0;
+    int maxCta = 0;
+    r = coResident(c0, fn, (int)c0->prm.threads, smem, maxCta);
+    if (r != mscclSuccess) return r;
+    if (cta > maxCta) {
       std::ostringstream o;
-      o << "program needs " << cta << " co-resident CTAs on device " << c0->dev << " but at most "
-        << c0->maxCoResident << " fit (lower MSCCL_THREADS or use fewer instances/channels)";
+      o << "program needs " << cta << " co-resident CTAs on device " << c0->dev << " but at most " << maxCta
+        << " fit (use fewer instances/channels, or MSCCL_TMA=0 / fewer MSCCL_THREADS for more CTAs per SM)";
       return setErr(c0, mscclInvalidUsage, o.str());
     }
-    const void* fn = p0->hasReduce ? interpreterKernel(v[0]->dtype, v[0]->op) : copyKernel(elemBytes(v[0]->dtype));
     DeviceGuard dg(c0->dev);
     void* args[] = {&ka};
     if (debugOn())
       fprintf(stderr, "[msccl] launch dev %d ranks %d program %s ctas %d threads %d n %lld E %lld T %lld I %d\n",
               c0->dev, ka.nLocal, p0->algo.name.c_str(), cta, (int)c0->prm.threads, (long long)g.n,
               (long long)g.E, (long long)g.T, g.I);
-    CUDACHECK(c0, cudaLaunchCooperativeKernel(fn, dim3(cta), dim3((unsigned)c0->prm.threads), args, 0, v[0]->stream));
+    CUDACHECK(c0, cudaLaunchCooperativeKernel(fn, dim3(cta), dim3((unsigned)c0->prm.threads), args, (size_t)smem,
+                                              v[0]->stream));
     gLaunches++;
   }
   return mscclSuccess;
@@ -435,6 +486,9 @@ mscclResult_t mscclGetParam(const char* key, int64_t* value) {
 }
 
 uint64_t mscclLaunchCount(void) { return gLaunches.load(); }
+
+// not part of msccl.h: debug access to the MSCCL_TRACE phase timers (4096 CTAs x 8)
+uint64_t* msccl_debug_trace(void) { return gTraceHost; }
 
 mscclResult_t mscclCommInitAll(mscclComm_t* comms, int ndev, const int* devlist) {
   if (!comms || ndev < 1) return setErr(nullptr, mscclInvalidArgument, "bad arguments to mscclCommInitAll");

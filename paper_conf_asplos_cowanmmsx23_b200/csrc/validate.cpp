@@ -108,7 +108,6 @@ void validateIR(Algo& a, int nranks, int slots, int maxTbs, int maxChannels, int
   }
   if (!ok) fail("V3", "chunk counts do not fit the collective");
   if (a.inplace && a.coll != COLL_ALLREDUCE && a.coll != COLL_CUSTOM) fail("V3", "in-place programs are only defined for allreduce/custom");
-  if (a.proto == PROTO_LL128) fail("V1", "protocol LL128 is not implemented by this runtime");
 
   std::map<ConnKey, std::pair<int, int>> senders, receivers;  // -> (gpu, tb)
   for (auto& g : a.gpus) {

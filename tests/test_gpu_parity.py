@@ -69,6 +69,8 @@ AR = [
     ("ring_inplace", lambda R: P.ring_allreduce(R, inplace=True)),
     ("ring_channels_instances", lambda R: P.ring_allreduce(R, channels=R, instances=2)),
     ("ring_LL", lambda R: P.ring_allreduce(R, protocol="LL")),
+    ("ring_LL128", lambda R: P.ring_allreduce(R, instances=2, protocol="LL128")),
+    ("allpairs_LL128", lambda R: P.allpairs_allreduce(R, protocol="LL128")),
     ("allpairs_LL", lambda R: P.allpairs_allreduce(R)),
     ("allpairs_simple", lambda R: P.allpairs_allreduce(R, protocol="Simple")),
     ("oneshot_LL", lambda R: P.oneshot_allreduce(R)),
