@@ -423,6 +423,8 @@ def virtual_extras(comms, R, stream):
 
 def run_multi(args, rank, world, local_rank):
     import torch
+    if os.environ.get("MSCCL_FORCE_DEVICE"):  # testing the multi-process path on one GPU only
+        local_rank = int(os.environ["MSCCL_FORCE_DEVICE"])
     import torch.distributed as dist
     import synth
     from paper_conf_asplos_cowanmmsx23_b200 import runtime as rt
