@@ -429,7 +429,10 @@ def run_multi(args, rank, world, local_rank):
     import synth
     from paper_conf_asplos_cowanmmsx23_b200 import runtime as rt
     torch.cuda.set_device(local_rank)
-    dist.init_process_group("nccl", rank=rank, world_size=world, device_id=torch.device("cuda", local_rank))
+    if os.environ.get("MSCCL_FORCE_DEVICE"):  # NCCL refuses two ranks on one GPU; plumbing only anyway
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+    else:
+        dist.init_process_group("nccl", rank=rank, world_size=world, device_id=torch.device("cuda", local_rank))
     set_params(rt, args)
     R = world
     algo = build_program(args, R)
@@ -461,7 +464,9 @@ def run_multi(args, rank, world, local_rank):
     torch.cuda.synchronize()
     dist.barrier()
     t = ev0.elapsed_time(ev1) / 1e3 / args.steps
-    tt = torch.tensor([t], device=dev, dtype=torch.float64)
+    tt = torch.tensor([t], dtype=torch.float64)  # host tensor: works with any plumbing backend
+    if dist.get_backend() == "nccl":
+        tt = tt.to(dev)
     dist.all_reduce(tt, op=dist.ReduceOp.MAX)
     t = float(tt.item())
     launches = rt.launch_count() - l0
@@ -474,7 +479,9 @@ def run_multi(args, rank, world, local_rank):
     want = sampled.allreduce_at(irparse.parse(algo.to_xml()), lambda r, i: synth.hashed_numpy(r, i, "bfloat16"),
                                 n, "bfloat16", "sum", idx, rank=rank)
     got = recv[torch.from_numpy(idx).to(dev)].view(torch.int16).cpu().numpy().view(np.uint16)
-    bad = torch.tensor([int(np.count_nonzero(got != want))], device=dev)
+    bad = torch.tensor([int(np.count_nonzero(got != want))])
+    if dist.get_backend() == "nccl":
+        bad = bad.to(dev)
     dist.all_reduce(bad)
     res = {"t": t, "launches": launches, "clocks": clk, "parity_bad": int(bad.item()),
            "parity_total": idx.size * R, "algo": algo, "S": S, "R": R}
@@ -509,6 +516,23 @@ def main():
     launches_per_step = max(1, res["launches"] // args.steps)
     achieved = alg_bytes / t / 1e9
     traffic, prof = ncu_traffic()
+    if world > 1:
+        # one rank per GPU: the ring's bytes cross NVLink; roofline = measured peer copy 770 GB/s
+        # per direction (B200_PROFILING.md; 900 nominal). Egress per rank per step = busBW * t.
+        roof = {"bound": "nvlink", "achieved": round(value, 1), "peak": 770.0, "unit": "GB/s",
+                "frac": round(value / 770.0, 4), "traffic": None,
+                "peak_source": "measured peer copy per direction (B200_PROFILING.md)",
+                "kernel": "mscclInterpreter<bf16,sum>", "algorithmic_bytes_per_launch": int(S * 2 * (R - 1) / R),
+                "launch_ms": round(t * 1e3 / launches_per_step, 4)}
+    else:
+        roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(achieved / peak, 4), "traffic": traffic, "peak_source": peak_src,
+                "kernel": "mscclInterpreter<bf16,sum>", "algorithmic_bytes_per_launch": int(alg_bytes),
+                "launch_ms": round(t * 1e3 / launches_per_step, 4),
+                "compulsory_bytes_per_launch": int(2 * S * R),
+                "note": "algorithmic = per-instruction FIFO-protocol bytes (5.5 S per rank, SURVEY 8d), part of "
+                        "which stays in L2; traffic = ncu DRAM bytes per launch; compulsory = inputs read + "
+                        "outputs written"}
     out = {
         "metric": metric_name(), "value": round(value, 3), "unit": "GB/s", "n_gpus": N,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 4),
@@ -516,10 +540,7 @@ def main():
         "data": "synthetic (counter-based uniform[-1,1) bf16, seed 20230325+rank)",
         "config": config_dict(args, R, N),
         "frac_nvlink": round(value / 900.0, 4),
-        "roofline": {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                     "frac": round(achieved / peak, 4), "traffic": traffic, "peak_source": peak_src,
-                     "kernel": "mscclInterpreter<bf16,sum>", "algorithmic_bytes_per_launch": int(alg_bytes),
-                     "launch_ms": round(t * 1e3 / launches_per_step, 4)},
+        "roofline": roof,
         "gpu_launches": res["launches"],
         "parity": {"sampled_outputs": res["parity_total"], "mismatches": res["parity_bad"],
                    "against": "oracle reduction trees (oracle/sampled.py), bit-exact"},
