@@ -262,8 +262,9 @@ def run_virtual(args):
     n = S // 2
     dev = torch.device("cuda:0")
     comms = rt.Comm.virtual(R, 0)
-    for c in comms:
-        c.load(ir_text)
+    progs = [c.load(ir_text) for c in comms]
+    direct = rt.get_param("MSCCL_DIRECT") != 0 and args.protocol == "Simple"
+    touches = [p.touches(direct) for p in progs]
     idx = torch.arange(n, device=dev, dtype=torch.int64)
     send = [synth.hashed(q, idx, "bfloat16") for q in range(R)]
     del idx
@@ -297,7 +298,7 @@ def run_virtual(args):
             raise RuntimeError("watchdog fired during the bench")
     bad, total = sampled_parity(algo, recv, n, [0, R - 1])
     res = {"t": t, "launches": launches, "clocks": clk, "parity_bad": bad, "parity_total": total,
-           "algo": algo, "S": S, "R": R}
+           "algo": algo, "S": S, "R": R, "touches": touches, "direct": direct}
     # end-to-end through the public API with host buffers (pinned), every step
     if not args.no_e2e:
         host_in = [s.cpu().pin_memory() for s in send]
@@ -403,7 +404,7 @@ def virtual_extras(comms, R, stream):
     # AllToAll (direct, N=1 two-step), 256 MiB per rank, bf16
     S = 256 * MIB
     n = S // 2
-    algo = P.alltoall_twostep(1, R)
+    algo = P.alltoall_twostep(1, R, instances=2)
     progs = [c.load(algo.to_xml()) for c in comms]
     send = [synth.hashed(q, torch.arange(n, device=dev), "bfloat16") for q in range(R)]
     recv = [torch.empty_like(x) for x in send]
@@ -512,7 +513,10 @@ def main():
     peak, peak_src = measured_peak()
     per_chunk = S / algo.gpus[0].i_chunks
     nranks_launch = R if world == 1 else 1
-    alg_bytes = sum(simple_bytes_per_rank(algo, q, per_chunk) for q in range(R)) / R * nranks_launch
+    if "touches" in res:
+        alg_bytes = sum(res["touches"]) * per_chunk
+    else:
+        alg_bytes = sum(simple_bytes_per_rank(algo, q, per_chunk) for q in range(R)) / R * nranks_launch
     launches_per_step = max(1, res["launches"] // args.steps)
     achieved = alg_bytes / t / 1e9
     traffic, prof = ncu_traffic()
@@ -530,9 +534,10 @@ def main():
                 "kernel": "mscclInterpreter<bf16,sum>", "algorithmic_bytes_per_launch": int(alg_bytes),
                 "launch_ms": round(t * 1e3 / launches_per_step, 4),
                 "compulsory_bytes_per_launch": int(2 * S * R),
-                "note": "algorithmic = per-instruction FIFO-protocol bytes (5.5 S per rank, SURVEY 8d), part of "
-                        "which stays in L2; traffic = ncu DRAM bytes per launch; compulsory = inputs read + "
-                        "outputs written"}
+                "direct_placement": res.get("direct"),
+                "note": "algorithmic = per-instruction bytes of the program under the protocol (FIFO: 5.5 S per "
+                        "rank, SURVEY 8d; with direct placement 4.5 S), part of which stays in L2; traffic = ncu "
+                        "DRAM bytes per launch; compulsory = inputs read + outputs written"}
     out = {
         "metric": metric_name(), "value": round(value, 3), "unit": "GB/s", "n_gpus": N,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 4),

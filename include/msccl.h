@@ -110,6 +110,13 @@ mscclResult_t mscclUnloadProgram(mscclComm_t comm, mscclProgram_t program);
  * instructions, and whether it is in place. Any pointer may be NULL. */
 mscclResult_t mscclProgramInfo(mscclProgram_t program, int* nThreadBlocks, int* nInstructions, int* inplace);
 
+/* Algorithmic memory traffic of this rank's program, in chunk-sized touches per pipeline
+ * pass (bytes per launch = touches * chunk bytes): each instruction reads/writes its
+ * operands once per chunk — send 2, recv 2, copy 2, reduce 3, rrc 3, rrs 3, rrcs 4, rcs 3 —
+ * and with direct placement (directPlacement != 0, reading R15) a direct recv costs 0 and
+ * a direct rcs 2 (the data arrived in dst). */
+mscclResult_t mscclProgramTouches(mscclProgram_t program, int directPlacement, int64_t* touches);
+
 /* Comm-free structural validation (rules V1..V9 of DESIGN.md) — needs no GPU.
  * slots = FIFO slots per connection used by the deadlock check (0 = library default),
  * maxThreadBlocks = co-residency limit per rank (0 = 148). err (may be NULL) receives a

@@ -10,10 +10,18 @@ namespace msccl {
 
 #define MSCCL_MAX_LOCAL 16  // ranks that one kernel launch may cover (virtual ranks)
 
-struct DevInstr {     // 24 bytes
+enum { DI_SEND_DIRECT = 1, DI_RECV_DIRECT = 2 };
+
+struct DevInstr {     // 32 bytes
   uint8_t op, srcBuf, dstBuf, nDeps;
   uint16_t cnt, hasDep;
-  uint32_t srcOff, dstOff, depStart, pad;
+  uint32_t srcOff, dstOff, depStart;
+  // direct placement (reading R15): the message lands in the receiver's destination chunk
+  // instead of its FIFO slot. flags: DI_SEND_DIRECT (this send writes peer rdstBuf/rdstOff),
+  // DI_RECV_DIRECT (the data of this receive is already in dst when its head arrives).
+  uint8_t flags, rdstBuf;
+  uint16_t pad0;
+  uint32_t rdstOff, pad1;
 };
 
 // One thread block of one rank (= one CTA). Connection pointers are resolved at load time
@@ -22,7 +30,7 @@ struct DevTB {
   int32_t nSteps;
   uint32_t instrStart;
   int32_t tbId;
-  int32_t pad;
+  int32_t sendPeer;           // rank of the send peer (-1 if none)
   // send connection (peer = receiver): FIFO and head counter live in the PEER's region
   char* sendFifo;             // peer FIFO base for (me -> peer, chan); nullptr if no send peer
   uint64_t* sendHead;         // peer: messages posted by me
@@ -62,6 +70,8 @@ struct KernelArgs {
   int64_t slotBytes;
   int32_t sysScope;           // 1 when any peer is another GPU
   int32_t useTma;             // Simple protocol: bulk-copy (TMA) pipeline through shared memory
+  int32_t direct;             // honour DI_*_DIRECT flags (all ranks in this launch, rank == slot)
+  int32_t pad2;
   uint64_t timeoutNs;
   uint64_t* trace;            // MSCCL_TRACE builds: per-CTA phase times (ns), else null
 };

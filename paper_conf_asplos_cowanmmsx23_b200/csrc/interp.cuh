@@ -587,16 +587,28 @@ __device__ __forceinline__ int64_t pieceGeom(const Ctx& c, const DevInstr& in, i
 }
 
 template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
-__device__ __noinline__ void movePiecesSimple(const Ctx& c, const DevInstr& in, int t, const char* rslot, char* sslot) {
+__device__ __noinline__ void movePiecesSimple(const Ctx& c, const DevTB& tb, const DevInstr& in, int t,
+                                              const char* rslot, char* sslot) {
   MSCCL_PIECE_GEOM
-  (void)a0;
+  const bool sdirect = SEND && a.direct && (in.flags & DI_SEND_DIRECT);
+  const bool rdirect = RECV && a.direct && (in.flags & DI_RECV_DIRECT);
   for (int j = 0; j < in.cnt; j++) {
     const char* src;
     char* dst;
-    const int64_t m = pieceGeom<DT, SRC, DST, REDDST>(c, in, t, j, src, dst);
+    int64_t m = pieceGeom<DT, SRC, DST, REDDST>(c, in, t, j, src, dst);
+    char* so = SEND ? sslot + j * a.T * w : nullptr;
+    if (sdirect) {  // reading R15: write straight into the receiver's destination chunk
+      int64_t rs, rl;
+      chunkSpan(a, in.rdstBuf, (int64_t)in.rdstOff + j, rs, rl);
+      so = a.rank[tb.sendPeer].buf[in.rdstBuf] + (rs + a0) * w;
+      if (rl - a0 < m) m = rl - a0;
+    }
     if (m <= 0) continue;
-    pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, RECV ? rslot + j * a.T * w : nullptr, src, dst,
-                                                     SEND ? sslot + j * a.T * w : nullptr, c);
+    if (rdirect) {  // the data is already in dst (the sender wrote it there)
+      if (SEND) pieceSimple<DT, OP, false, true, true, false, false>(m, nullptr, dst, nullptr, so, c);
+      continue;
+    }
+    pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, RECV ? rslot + j * a.T * w : nullptr, src, dst, so, c);
   }
 }
 
@@ -694,7 +706,8 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
   if (c.tid == 0) tr1 = globaltimer();
 #endif
   // a free slot: at most `slots` messages posted and not yet consumed (§6.1)
-  if (SEND && c.tid == (RECV ? 32 : 0) && sent + 1 > (uint64_t)a.slots)
+  // (a direct message uses no slot: no credit needed, reading R15)
+  if (SEND && c.tid == (RECV ? 32 : 0) && sent + 1 > (uint64_t)a.slots && !(a.direct && (in.flags & DI_SEND_DIRECT)))
     ok = ok && waitGE(tb.sendAck, sent + 1 - (uint64_t)a.slots, sys, c);
   if (!ok) *sAbort = 1;
   if (RECV || SEND) {
@@ -711,7 +724,7 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
 #if MSCCL_ENABLE_TMA
     if (c.tma == nullptr || !movePiecesTma<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, in, t, rslot, sslot))
 #endif
-      movePiecesSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, in, t, rslot, sslot);
+      movePiecesSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, tb, in, t, rslot, sslot);
   } else if constexpr (PROTO == 2) {
     if (!movePiecesLL128<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, in, t, rslot, sslot, recvd + 1, sent + 1)) *sAbort = 1;
   } else {

@@ -70,6 +70,16 @@ Algo parseIR(const char* text, size_t len);  // throws IRError (rule V1)
 // Throws IRError("Vn: ...") on the first violated rule (V1..V9).
 void validateIR(Algo& a, int nranks, int slots, int maxTbs, int maxChannels, int iters = 2);
 
+// Direct placement analysis (reading R15). For rank `rank`: recvDirect[tb][step] = the
+// receive may find its data already in its destination (op r / rcs whose destination
+// chunks no other instruction of the rank touches unless ordered after it);
+// sendDirect[tb][step] = the matching receive on the peer is direct (+ its dst buf/off).
+struct DirectInfo {
+  std::vector<std::vector<char>> recvDirect, sendDirect;
+  std::vector<std::vector<int>> rdstBuf, rdstOff;
+};
+DirectInfo directPlacement(const Algo& a, int rank);
+
 // blocks per buffer for a collective (reading R1)
 int blocksOf(int coll, int buf, int R);
 

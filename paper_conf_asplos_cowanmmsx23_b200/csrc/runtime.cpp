@@ -26,7 +26,7 @@ using namespace msccl;
 namespace {
 
 struct Params {
-  int64_t slots = 4, slotBytes = 262144, maxChannels = 32, threads = 512, timeoutS = 20, tma = 0;
+  int64_t slots = 4, slotBytes = 262144, maxChannels = 32, threads = 512, timeoutS = 20, tma = 0, direct = 1;
 };
 
 std::mutex gMu;
@@ -42,6 +42,7 @@ int64_t* paramRef(Params& p, const std::string& k) {
   if (k == "MSCCL_THREADS") return &p.threads;
   if (k == "MSCCL_TIMEOUT_S") return &p.timeoutS;
   if (k == "MSCCL_TMA") return &p.tma;
+  if (k == "MSCCL_DIRECT") return &p.direct;
   return nullptr;
 }
 
@@ -50,7 +51,7 @@ Params currentParams() {
   if (!gEnvRead) {
     gEnvRead = true;
     for (const char* k : {"MSCCL_SLOTS", "MSCCL_SLOT_BYTES", "MSCCL_MAX_CHANNELS", "MSCCL_THREADS", "MSCCL_TIMEOUT_S",
-                          "MSCCL_TMA"}) {
+                          "MSCCL_TMA", "MSCCL_DIRECT"}) {
       const char* v = getenv(k);
       if (v && *v) *paramRef(gParams, k) = atoll(v);
     }
@@ -339,6 +340,9 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
     const void* fn = p0->hasReduce ? interpreterKernel(v[0]->dtype, v[0]->op, ka.proto)
                                    : copyKernel(elemBytes(v[0]->dtype), ka.proto);
     ka.useTma = (ka.proto == 0 && c0->prm.tma && tmaSmemBytes() > 0) ? 1 : 0;
+    // direct placement needs every rank's buffers in this launch (rank r at slot r) and the
+    // Simple protocol; one launch covering all ranks also orders it against earlier launches
+    ka.direct = (ka.proto == 0 && c0->prm.direct && ka.nLocal == p0->algo.ngpus && !ka.useTma) ? 1 : 0;
     const int smem = ka.useTma ? tmaSmemBytes() : 0;
     int maxCta = 0;
     r = coResident(c0, fn, (int)c0->prm.threads, smem, maxCta);
@@ -659,6 +663,7 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
   p->hasReduce = p->algo.hasReduce();
   const GpuProgram& g = p->algo.gpus[c->rank];
   p->nTB = (int)g.tbs.size();
+  const DirectInfo dinfo = directPlacement(p->algo, c->rank);
   std::vector<DevTB> tbs(p->nTB);
   std::vector<DevInstr> ins;
   std::vector<uint32_t> deps;
@@ -669,6 +674,7 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
     d.nSteps = (int)tb.steps.size();
     d.instrStart = (uint32_t)ins.size();
     d.tbId = tb.id;
+    d.sendPeer = tb.send;
     if (tb.send >= 0) {
       d.sendFifo = c->peerBase[tb.send] + c->fifoOff(c->rank, tb.chan);
       d.sendHead = (uint64_t*)(c->peerBase[tb.send] + c->flagOff(0, c->rank, tb.chan));
@@ -681,7 +687,8 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
       d.recvAck = (uint64_t*)(c->peerBase[tb.recv] + c->flagOff(1, c->rank, tb.chan));
       d.recvCnt = (uint64_t*)(c->region + c->flagOff(3, tb.recv, tb.chan));
     }
-    for (auto& in : tb.steps) {
+    for (size_t si = 0; si < tb.steps.size(); si++) {
+      const Instr& in = tb.steps[si];
       DevInstr di;
       memset(&di, 0, sizeof(di));
       di.op = (uint8_t)in.op;
@@ -695,6 +702,12 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
       di.dstOff = (uint32_t)std::max(in.dstOff, 0);
       di.depStart = (uint32_t)deps.size();
       for (auto& dp : in.deps) deps.push_back(((uint32_t)dp.first << 16) | (uint32_t)dp.second);
+      if (dinfo.recvDirect[t][si]) di.flags |= DI_RECV_DIRECT;
+      if (dinfo.sendDirect[t][si]) {
+        di.flags |= DI_SEND_DIRECT;
+        di.rdstBuf = (uint8_t)dinfo.rdstBuf[t][si];
+        di.rdstOff = (uint32_t)dinfo.rdstOff[t][si];
+      }
       ins.push_back(di);
     }
   }
@@ -738,6 +751,23 @@ mscclResult_t mscclProgramInfo(mscclProgram_t p, int* nTB, int* nInstr, int* inp
   if (nTB) *nTB = p->nTB;
   if (nInstr) *nInstr = p->nInstr;
   if (inplace) *inplace = p->algo.inplace ? 1 : 0;
+  return mscclSuccess;
+}
+
+mscclResult_t mscclProgramTouches(mscclProgram_t p, int direct, int64_t* touches) {
+  if (!p || !touches) return mscclInvalidArgument;
+  static const int cost[OP_COUNT] = {0, 2, 2, 2, 3, 3, 3, 4, 3};
+  const DirectInfo di = directPlacement(p->algo, p->comm->rank);
+  int64_t n = 0;
+  const GpuProgram& g = p->algo.gpus[p->comm->rank];
+  for (size_t t = 0; t < g.tbs.size(); t++)
+    for (size_t s = 0; s < g.tbs[t].steps.size(); s++) {
+      const Instr& in = g.tbs[t].steps[s];
+      int c = cost[in.op];
+      if (direct && di.recvDirect[t][s]) c = in.op == OP_RCS ? 2 : 0;
+      n += (int64_t)c * in.cnt;
+    }
+  *touches = n;
   return mscclSuccess;
 }
 

@@ -179,4 +179,78 @@ void validateIR(Algo& a, int nranks, int slots, int maxTbs, int maxChannels, int
   deadlockCheck(a, slots, iters);
 }
 
+namespace {
+
+// may receive step (tb, s) of rank g write its destination before its turn?
+bool recvCanBeDirect(const Algo& a, int g, int tb, int s) {
+  const GpuProgram& gp = a.gpus[g];
+  const Instr& q = gp.tbs[tb].steps[s];
+  if (q.op != OP_RECV && q.op != OP_RCS) return false;  // data must land unchanged
+  auto canon = [&](int buf) { return (a.inplace && buf == BUF_OUT) ? BUF_IN : buf; };
+  const int qb = canon(q.dstBuf);
+  auto overlaps = [&](int buf, int off, int cnt) {
+    return canon(buf) == qb && off < q.dstOff + q.cnt && q.dstOff < off + cnt;
+  };
+  for (auto& t : gp.tbs) {
+    for (size_t k = 0; k < t.steps.size(); k++) {
+      if (t.id == tb && (int)k == s) continue;
+      const Instr& x = t.steps[k];
+      OpRole ro = opRole(x.op);
+      bool touches = (ro.src && overlaps(x.srcBuf, x.srcOff, x.cnt)) ||
+                     ((ro.dst || x.op == OP_REDUCE) && overlaps(x.dstBuf, x.dstOff, x.cnt));
+      if (!touches) continue;
+      if (t.id == tb && (int)k > s) continue;  // same thread block, later in program order
+      bool ordered = false;                     // waits on this receive (or a later step of its tb)
+      for (auto& d : x.deps)
+        if (d.first == tb && d.second >= s) ordered = true;
+      if (!ordered) return false;
+    }
+  }
+  return true;
+}
+
+}  // namespace
+
+DirectInfo directPlacement(const Algo& a, int rank) {
+  DirectInfo di;
+  const GpuProgram& g = a.gpus[rank];
+  di.recvDirect.resize(g.tbs.size());
+  di.sendDirect.resize(g.tbs.size());
+  di.rdstBuf.resize(g.tbs.size());
+  di.rdstOff.resize(g.tbs.size());
+  for (size_t t = 0; t < g.tbs.size(); t++) {
+    const ThreadBlock& tb = g.tbs[t];
+    di.recvDirect[t].assign(tb.steps.size(), 0);
+    di.sendDirect[t].assign(tb.steps.size(), 0);
+    di.rdstBuf[t].assign(tb.steps.size(), 0);
+    di.rdstOff[t].assign(tb.steps.size(), 0);
+    for (size_t s = 0; s < tb.steps.size(); s++)
+      if (opRole(tb.steps[s].op).recv) di.recvDirect[t][s] = recvCanBeDirect(a, rank, (int)t, (int)s);
+    if (tb.send < 0) continue;
+    // pair the k-th send of (rank -> peer, chan) with the k-th receive of the peer's receiving tb
+    const GpuProgram& pg = a.gpus[tb.send];
+    const ThreadBlock* rt = nullptr;
+    for (auto& x : pg.tbs)
+      if (x.recv == rank && x.chan == tb.chan) rt = &x;
+    if (!rt) continue;
+    std::vector<int> rsteps;
+    for (size_t k = 0; k < rt->steps.size(); k++)
+      if (opRole(rt->steps[k].op).recv) rsteps.push_back((int)k);
+    int k = 0;
+    for (size_t s = 0; s < tb.steps.size(); s++) {
+      if (!opRole(tb.steps[s].op).send) continue;
+      if (k < (int)rsteps.size()) {
+        int rs = rsteps[k];
+        if (recvCanBeDirect(a, tb.send, rt->id, rs)) {
+          di.sendDirect[t][s] = 1;
+          di.rdstBuf[t][s] = rt->steps[rs].dstBuf;
+          di.rdstOff[t][s] = rt->steps[rs].dstOff;
+        }
+      }
+      k++;
+    }
+  }
+  return di;
+}
+
 }  // namespace msccl

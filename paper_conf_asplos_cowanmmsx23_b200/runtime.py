@@ -42,6 +42,7 @@ SIGNATURES = {
     "mscclUnloadProgram": (_i, [_vp, _vp]),
     "mscclProgramInfo": (_i, [_vp, _c.POINTER(_i), _c.POINTER(_i), _c.POINTER(_i)]),
     "mscclValidateProgram": (_i, [_c.c_char_p, _sz, _i, _i, _i, _c.c_char_p, _sz]),
+    "mscclProgramTouches": (_i, [_vp, _i, _c.POINTER(_i64)]),
     "mscclAllReduce": (_i, [_vp, _vp, _sz, _i, _i, _vp, _vp]),
     "mscclAllGather": (_i, [_vp, _vp, _sz, _i, _vp, _vp]),
     "mscclReduceScatter": (_i, [_vp, _vp, _sz, _i, _i, _vp, _vp]),
@@ -134,6 +135,12 @@ class Program:
         a, b, c = _i(), _i(), _i()
         _check(lib.mscclProgramInfo(self.handle, _c.byref(a), _c.byref(b), _c.byref(c)), self.comm.handle)
         return {"thread_blocks": a.value, "instructions": b.value, "inplace": bool(c.value)}
+
+    def touches(self, direct=True):
+        """Algorithmic chunk-sized memory touches of this rank's program (mscclProgramTouches)."""
+        v = _i64()
+        _check(lib.mscclProgramTouches(self.handle, int(direct), _c.byref(v)), self.comm.handle)
+        return v.value
 
 
 class Comm:
