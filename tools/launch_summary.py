@@ -1,6 +1,7 @@
 """Summarise an ncu --metrics gpu__time_duration.sum launch list (csv) into profiles/."""
 import csv, sys
-rows = list(csv.reader(open(sys.argv[1])))
+lines = [l for l in open(sys.argv[1]) if l.startswith('"')]
+rows = list(csv.reader(lines))
 hdr = rows[0]
 ki, vi = hdr.index("Kernel Name"), hdr.index("Metric Value")
 allk, interp = [], []
