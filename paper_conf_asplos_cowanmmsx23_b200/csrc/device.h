@@ -10,7 +10,7 @@ namespace msccl {
 
 #define MSCCL_MAX_LOCAL 16  // ranks that one kernel launch may cover (virtual ranks)
 
-enum { DI_SEND_DIRECT = 1, DI_RECV_DIRECT = 2 };
+enum { DI_SEND_DIRECT = 1, DI_RECV_DIRECT = 2, DI_CHAIN_HEAD = 4 };
 
 struct DevInstr {     // 32 bytes
   uint8_t op, srcBuf, dstBuf, nDeps;
@@ -20,7 +20,7 @@ struct DevInstr {     // 32 bytes
   // instead of its FIFO slot. flags: DI_SEND_DIRECT (this send writes peer rdstBuf/rdstOff),
   // DI_RECV_DIRECT (the data of this receive is already in dst when its head arrives).
   uint8_t flags, rdstBuf;
-  uint16_t pad0;
+  uint16_t chainLen;          // DI_CHAIN_HEAD: this and the next chainLen-1 local ops fold into one pass
   uint32_t rdstOff, pad1;
 };
 

@@ -799,6 +799,71 @@ __device__ __forceinline__ bool dispatch(const Ctx& c, const DevTB& tb, const De
   return true;  // nop
 }
 
+// ------------------------------------------------------------------ fused local reduce chains
+// A run of local instructions [cpy(src0 -> D)] re(src1 -> D) re(src2 -> D) ... on one
+// destination D (marked by the loader, reading R16) is executed in ONE pass: acc = src0
+// (or D), acc = acc (+) src_k in program order, one store — the same operations in the same
+// order as the sequential instructions (bit-identical), without a global round trip and a
+// barrier per instruction. Pieces whose members disagree on length fall back to the
+// sequential instructions.
+#define MSCCL_MAX_CHAIN 16
+template <int DT, int OP>
+__device__ __noinline__ void chainExec(const Ctx& c, const DevInstr* mem, int L, int t) {
+  typedef typename DType<DT>::T T;
+  const KernelArgs& a = *c.a;
+  const RankArgs& ra = *c.ra;
+  const int64_t w = sizeof(T);
+  const int64_t a0 = (int64_t)t * a.T;
+  const bool headCopy = mem[0].op == K_COPY;
+  for (int j = 0; j < mem[0].cnt; j++) {
+    int64_t ds, dl;
+    chunkSpan(a, mem[0].dstBuf, (int64_t)mem[0].dstOff + j, ds, dl);
+    const char* srcs[MSCCL_MAX_CHAIN];
+    int64_t m = -1;
+    bool same = true;
+    uintptr_t al = 0;
+    for (int k = 0; k < L; k++) {
+      int64_t ss, sl;
+      chunkSpan(a, mem[k].srcBuf, (int64_t)mem[k].srcOff + j, ss, sl);
+      int64_t Lk = sl < dl ? sl : dl;
+      int64_t mk = (a0 + a.T < Lk ? a0 + a.T : Lk) - a0;
+      if (m < 0) m = mk;
+      else if (mk != m) same = false;
+      srcs[k] = ra.buf[mem[k].srcBuf] + (ss + a0) * w;
+      al |= (uintptr_t)srcs[k];
+    }
+    char* dst = ra.buf[mem[0].dstBuf] + (ds + a0) * w;
+    al |= (uintptr_t)dst;
+    if (!same) {  // sequential fallback (a barrier between members: element->thread maps differ)
+      for (int k = 0; k < L; k++) {
+        int64_t ss, sl;
+        chunkSpan(a, mem[k].srcBuf, (int64_t)mem[k].srcOff + j, ss, sl);
+        int64_t Lk = sl < dl ? sl : dl;
+        int64_t mk = (a0 + a.T < Lk ? a0 + a.T : Lk) - a0;
+        if (mk > 0) {
+          if (mem[k].op == K_COPY) pieceSimple<DT, OP, false, false, true, true, false>(mk, nullptr, srcs[k], dst, nullptr, c);
+          else pieceSimple<DT, OP, false, false, true, true, true>(mk, nullptr, srcs[k], dst, nullptr, c);
+        }
+        __syncthreads();
+      }
+      continue;
+    }
+    if (m <= 0) continue;
+    const int64_t bytes = m * w;
+    int64_t nvec = (al & 15) ? 0 : bytes / 16;
+    for (int64_t i = c.tid; i < nvec; i += c.nt) {
+      uint4 acc = headCopy ? ldcg(srcs[0] + i * 16) : ldcg(dst + i * 16);
+      for (int k = headCopy ? 1 : 0; k < L; k++) acc = vop<DT, OP>(acc, ldcg(srcs[k] + i * 16));
+      stg(dst + i * 16, acc);
+    }
+    for (int64_t e = nvec * 16 / w + c.tid; e < m; e += c.nt) {
+      T acc = headCopy ? *(const T*)(srcs[0] + e * w) : *(const T*)(dst + e * w);
+      for (int k = headCopy ? 1 : 0; k < L; k++) acc = DType<DT>::op(OP, acc, *(const T*)(srcs[k] + e * w));
+      *(T*)(dst + e * w) = acc;
+    }
+  }
+}
+
 #ifndef MSCCL_MAX_THREADS
 #define MSCCL_MAX_THREADS 512
 #endif
@@ -844,6 +909,32 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
   for (int t = 0; t < a.I; t++) {
     for (int s = 0; s < tb.nSteps; s++) {
       const DevInstr in = ra.instrs[tb.instrStart + s];
+      if constexpr (OP != R_COPY) {
+        if (in.flags & DI_CHAIN_HEAD) {  // reading R16: fused local reduce chain
+          const int L = in.chainLen;
+          bool ok = true;
+          for (int k = 0; k < L && ok; k++) {  // all members' dependencies first
+            const DevInstr& mk = ra.instrs[tb.instrStart + s + k];
+            for (int d = c.tid; d < mk.nDeps && ok; d += c.nt) {
+              uint32_t dep = ra.deps[mk.depStart + d];
+              int dtb = (int)(dep >> 16), dstep = (int)(dep & 0xffff);
+              uint64_t target = (gen << 40) | ((uint64_t)t * (uint64_t)ra.tbs[dtb].nSteps + (uint64_t)dstep + 1);
+              ok = waitGE(&ra.sem[dtb], target, false, c);
+            }
+          }
+          if (!ok) sAbort = 1;
+          __syncthreads();
+          if (sAbort) return;
+          chainExec<DT, OP>(c, ra.instrs + tb.instrStart + s, L, t);
+          __syncthreads();
+          s += L - 1;
+          if (ra.instrs[tb.instrStart + s].hasDep && c.tid == 0) {
+            fenceGpu();
+            stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)tb.nSteps + (uint64_t)s + 1));
+          }
+          continue;
+        }
+      }
       if (in.nDeps) {  // Fig. 5 lines 15-16; barrier after the waits (reading R10)
         bool ok = true;
         for (int d = c.tid; d < in.nDeps && ok; d += c.nt) {

@@ -710,6 +710,36 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
       }
       ins.push_back(di);
     }
+    // reading R16: mark runs [cpy ->D] re ->D re ->D ... (same D and cnt, no hasDep before the
+    // last member, sources distinct from D) as one fused chain for the interpreter
+    size_t base = d.instrStart;
+    for (size_t s0 = 0; s0 < tb.steps.size();) {
+      const Instr& h = tb.steps[s0];
+      size_t e = s0;
+      if (h.op == OP_COPY || h.op == OP_REDUCE) {
+        auto sameDst = [&](const Instr& x) {
+          return x.op == OP_REDUCE && x.dstBuf == h.dstBuf && x.dstOff == h.dstOff && x.cnt == h.cnt &&
+                 !(x.srcBuf == h.dstBuf && x.srcOff < h.dstOff + h.cnt && h.dstOff < x.srcOff + x.cnt);
+        };
+        bool headOk = !(h.srcBuf == h.dstBuf && h.srcOff < h.dstOff + h.cnt && h.dstOff < h.srcOff + h.cnt);
+        if (headOk && !h.hasDep) {
+          e = s0 + 1;
+          while (e < tb.steps.size() && e - s0 < 16 && sameDst(tb.steps[e])) {
+            if (tb.steps[e].hasDep) {
+              e++;
+              break;
+            }
+            e++;
+          }
+        }
+      }
+      size_t len = e > s0 ? e - s0 : 1;
+      if (len >= 2) {
+        ins[base + s0].flags |= DI_CHAIN_HEAD;
+        ins[base + s0].chainLen = (uint16_t)len;
+      }
+      s0 += len;
+    }
   }
   p->nInstr = (int)ins.size();
   DeviceGuard dg(c->dev);

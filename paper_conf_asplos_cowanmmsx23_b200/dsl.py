@@ -550,7 +550,15 @@ class Program:
             if x.sp >= 0 or x.rp >= 0:
                 tb = cands[0]
             else:
-                tb = min(cands, key=lambda t: (last.get(id(t), -1), t.id))
+                # a local op that depends on the last instruction of some thread block stays on
+                # that block (program order replaces a cross-block dependency and keeps chains of
+                # local reduces together, reading R16); otherwise the paper's rule: the block
+                # whose latest instruction is earliest
+                chained = [t for t in cands if t.ins and t.ins[-1] in x.deps]
+                if chained:
+                    tb = chained[0]
+                else:
+                    tb = min(cands, key=lambda t: (last.get(id(t), -1), t.id))
             x.tb, x.step = tb.id, len(tb.ins)
             tb.ins.append(x)
             last[id(tb)] = pos
