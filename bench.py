@@ -419,6 +419,31 @@ def virtual_extras(comms, R, stream):
                                    "ctas": sum(p.info()["thread_blocks"] for p in progs), "bit_exact": bool(ok)}
     for c, p in zip(comms, progs):
         c.unload(p)
+    del send, recv
+    # AllGather / ReduceScatter rings (config 5), S = 256 MiB of output (AG) / input (RS) per rank
+    nb = n // R
+    for name, algo, coll in (("allgather", P.ring_allgather(R, 1, 32), "allgather"),
+                             ("reducescatter", P.ring_reducescatter(R, 1, 32), "reducescatter")):
+        progs = [c.load(algo.to_xml()) for c in comms]
+        ins = nb if coll == "allgather" else n
+        outs = n if coll == "allgather" else nb
+        send = [synth.hashed(q, torch.arange(ins, device=dev), "bfloat16") for q in range(R)]
+        recv = [torch.empty(outs, dtype=torch.bfloat16, device=dev) for _ in range(R)]
+
+        def call():
+            with rt.group():
+                for q in range(R):
+                    comms[q].run(progs[q], send[q], recv[q], nb)
+        t, mode = _timed(call, 3, stream, graph=False)
+        if coll == "allgather":
+            ok = all(torch.equal(recv[q].view(R, -1)[p], send[p]) for q in (0, R - 1) for p in range(R))
+        else:
+            ok = None
+        out[name + "_bf16_256MiB"] = {"busbw_GBps": round(busbw(coll, S, t, R), 2), "ms": round(t * 1e3, 3),
+                                      "instances": 32, "bit_exact": ok}
+        for c, p in zip(comms, progs):
+            c.unload(p)
+        del send, recv
     return out
 
 

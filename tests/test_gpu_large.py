@@ -12,13 +12,16 @@ from paper_conf_asplos_cowanmmsx23_b200 import programs as P
 pytestmark = pytest.mark.gpu
 
 
-@pytest.fixture(scope="module", autouse=True)
-def production_params():
+@pytest.fixture(scope="module", autouse=True, params=[1, 0], ids=["direct", "fifo"])
+def production_params(request):
+    """Production launch parameters; every test runs with direct placement (reading R15)
+    and with it disabled (all messages through the receiver-side FIFO)."""
     from paper_conf_asplos_cowanmmsx23_b200 import runtime
-    for k, v in (("MSCCL_SLOT_BYTES", 262144), ("MSCCL_SLOTS", 4), ("MSCCL_THREADS", 512),
-                 ("MSCCL_MAX_CHANNELS", 32), ("MSCCL_TIMEOUT_S", 10)):
+    for k, v in (("MSCCL_SLOT_BYTES", 262144), ("MSCCL_SLOTS", 4), ("MSCCL_THREADS", 256),
+                 ("MSCCL_MAX_CHANNELS", 32), ("MSCCL_TIMEOUT_S", 10), ("MSCCL_DIRECT", request.param)):
         runtime.set_param(k, v)
     yield
+    runtime.set_param("MSCCL_DIRECT", 1)
 
 
 @pytest.mark.parametrize("r,extra", [(4, 12345), (3, 7), (2, 131072 * 2 + 999)])
@@ -46,7 +49,7 @@ def test_alltoall_and_allgather_default_slots():
     assert all(np.array_equal(g, e) for g, e in zip(got, mpi_ref.allgather(xs)))
 
 
-@pytest.mark.parametrize("instances", [16, 18])
+@pytest.mark.parametrize("instances", [16, 32])
 def test_bench_size_sampled_parity(instances):
     """The bench workload (launch configuration of bench.py) at full size; outputs
     sampled on every rank and compared bit-exactly with the oracle's reduction trees."""
