@@ -198,9 +198,10 @@ class _Ins:
 class Program:
     """Context in which a DSL program is traced and lowered (Fig. 2 architecture)."""
 
-    def __init__(self, name, collective, protocol="Simple", instances=1, topology=None):
+    def __init__(self, name, collective, protocol="Simple", instances=1, topology=None, pair_tbs=False):
         if protocol not in ("Simple", "LL", "LL128"):
             raise DSLError("unknown protocol %r" % protocol)
+        self.pair_tbs = pair_tbs  # merge send-only (p,-1,ch) with recv-only (-1,p,ch) blocks (R17)
         self.name = name
         self.collective = collective
         self.protocol = protocol
@@ -499,7 +500,18 @@ class Program:
                                    "thread block" % (x.rank, x.sp, x.rp, x.ch))
         tbs = []
         for r in range(self.R):
-            lst = [_TB(t[0], t[1], t[2]) for t in states[r].final()]
+            tuples = states[r].final()
+            if self.pair_tbs:  # reading R17: one block per peer and channel for both directions
+                recv_only = {(t[1], t[2]): t for t in tuples if t[0] < 0 <= t[1]}
+                merged = []
+                for t in tuples:
+                    if t[0] >= 0 and t[1] < 0 and (t[0], t[2]) in recv_only:
+                        merged.append((t[0], t[0], t[2]))
+                        recv_only.pop((t[0], t[2]))
+                    elif not (t[0] < 0 <= t[1]):
+                        merged.append(t)
+                tuples = merged + list(recv_only.values())
+            lst = [_TB(t[0], t[1], t[2]) for t in tuples]
             if not lst and any(x.rank == r for x in ins):
                 lst.append(_TB(-1, -1, 0))
             for i, tb in enumerate(lst):

@@ -91,7 +91,7 @@ def mutations():
 
 
 def too_many_tbs(limit):
-    a = P.allpairs_allreduce(8)
+    a = P.allpairs_allreduce(8, pair_tbs=False)
     return a.max_tbs() > limit, a.to_xml()
 
 
