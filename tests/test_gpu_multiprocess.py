@@ -79,3 +79,55 @@ def test_two_processes_ipc(prog_name):
         y, err = res[r]
         assert err == 0, y
         assert np.array_equal(np.asarray(y).view(np.uint32), want[r].view(np.uint32))
+
+
+def _silent_peer_worker(rank, world, port, q):
+    import torch
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_asplos_cowanmmsx23_b200 import dist as mdist
+        from paper_conf_asplos_cowanmmsx23_b200 import programs, runtime
+        runtime.set_param("MSCCL_TIMEOUT_S", 3)
+        runtime.set_param("MSCCL_SLOT_BYTES", 16384)
+        runtime.set_param("MSCCL_MAX_CHANNELS", 2)
+        runtime.set_param("MSCCL_THREADS", 64)
+        comm = mdist.init_from_process_group(0)
+        comm.load(programs.ring_allreduce(world).to_xml())
+        res = None
+        if rank == 0:  # rank 1 never joins the collective: rank 0's kernel must not hang
+            x = torch.ones(4096, device="cuda")
+            y = torch.empty_like(x)
+            comm.allreduce(x, y)
+            torch.cuda.synchronize()
+            err = comm.async_error()
+            try:
+                comm.allreduce(x, y)
+                again = "no error"
+            except runtime.MscclError as e:
+                again = e.code
+            res = (err, again)
+        dist.barrier()
+        q.put((rank, res))
+    except Exception as e:
+        q.put((rank, repr(e)))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_watchdog_turns_a_missing_peer_into_an_error():
+    """A peer that never launches: the spin waits time out (MSCCL_TIMEOUT_S), the kernel
+    exits, and the communicator reports mscclRemoteError (sticky) instead of hanging."""
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_silent_peer_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = dict(q.get(timeout=180) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+    assert res[0] == (6, 6), res  # async error RemoteError, and the next call refuses
