@@ -146,14 +146,25 @@ __device__ __forceinline__ void stg(void* p, uint4 v) {
 // L2 cache policies: user input/output streams are touched once (evict_first); FIFO
 // slots are written by the sender and read soon after by the receiver (evict_last), then
 // discarded from L2 by the receiver so the dead slot is never written back to HBM.
+#ifndef MSCCL_NO_HINTS
+#define MSCCL_NO_HINTS 0
+#endif
 __device__ __forceinline__ uint64_t policyEvictFirst() {
   uint64_t p;
+#if MSCCL_NO_HINTS
+  asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+#else
   asm volatile("createpolicy.fractional.L2::evict_first.b64 %0, 1.0;" : "=l"(p));
+#endif
   return p;
 }
 __device__ __forceinline__ uint64_t policyEvictLast() {
   uint64_t p;
+#if MSCCL_NO_HINTS
+  asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+#else
   asm volatile("createpolicy.fractional.L2::evict_last.b64 %0, 1.0;" : "=l"(p));
+#endif
   return p;
 }
 template <int VB> struct VecT;
@@ -188,7 +199,14 @@ __device__ __forceinline__ void stHint(void* p, const V32& v, uint64_t pol) {
                "r"(v.a.y), "r"(v.a.z), "r"(v.a.w), "r"(v.b.x), "r"(v.b.y), "r"(v.b.z), "r"(v.b.w), "l"(pol)
                : "memory");
 }
-__device__ __forceinline__ void discardL2(const void* p) { asm volatile("discard.global.L2 [%0], 128;" ::"l"(p) : "memory"); }
+#ifndef MSCCL_NO_DISCARD
+#define MSCCL_NO_DISCARD 0
+#endif
+__device__ __forceinline__ void discardL2(const void* p) {
+#if !MSCCL_NO_DISCARD
+  asm volatile("discard.global.L2 [%0], 128;" ::"l"(p) : "memory");
+#endif
+}
 
 __device__ __forceinline__ uint4 ldvol(const void* p) {
   uint4 v;
