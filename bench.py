@@ -64,6 +64,17 @@ def measured_peak():
         return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
 
 
+def l2_peak():
+    """Measured L2-resident copy throughput (tools/l2bw.cu), committed under profiles/."""
+    p = os.path.join(ROOT, "profiles", "l2_peak.json")
+    try:
+        with open(p) as f:
+            d = json.load(f)
+        return float(d["l2_gbs"]), "measured (profiles/l2_peak.json: %s)" % d.get("how", "")
+    except Exception:
+        return None, "unmeasured"
+
+
 def ncu_traffic():
     """dram read+write bytes per launch of the interpreter, from the committed ncu summary."""
     p = os.path.join(ROOT, "profiles", "ncu_summary.json")
@@ -206,15 +217,19 @@ def run_reference(args):
     print(json.dumps(out), flush=True)
 
 
-def metric_name():
+def metric_name(coll="allreduce"):
+    if coll == "alltoall":
+        return "AllToAll busBW (GB/s), direct MSCCL-IR (two-step N=1), bf16"
     return "AllReduce busBW (GB/s), ring MSCCL-IR, bf16"
 
 
 def config_dict(args, R, N):
     mode = "virtual ranks on 1 GPU" if N == 1 else "1 process per GPU, CUDA IPC peer memory"
-    return {"workload": "BASELINE config 1: ring AllReduce MSCCL-IR, %d channels, %d instances, %s protocol, "
-                        "%d ranks (%s), %d MiB per rank" % (args.channels, args.instances, args.protocol, R, mode,
-                                                            int(args.size_mib)),
+    what = {"ring": "BASELINE config 1: ring AllReduce", "allpairs": "BASELINE config 2: all-pairs AllReduce",
+            "oneshot": "BASELINE config 2: one-shot AllReduce",
+            "alltoall": "BASELINE config 3: direct AllToAll"}[args.program]
+    return {"workload": "%s MSCCL-IR, %d channels, %d instances, %s protocol, %d ranks (%s), %d MiB per rank"
+                        % (what, args.channels, args.instances, args.protocol, R, mode, int(args.size_mib)),
             "program": args.program, "ranks": R, "bytes_per_rank": int(args.size_mib * MIB),
             "channels": args.channels, "instances": args.instances, "protocol": args.protocol,
             "threads": args.threads, "slots": args.slots, "slot_bytes": args.slot_kib * 1024,
@@ -271,10 +286,15 @@ def run_virtual(args):
     recv = [torch.empty(n, dtype=torch.bfloat16, device=dev) for _ in range(R)]
     stream = torch.cuda.current_stream()
 
+    coll = "alltoall" if args.program == "alltoall" else "allreduce"
+
     def step():
         with rt.group():
             for q in range(R):
-                comms[q].allreduce(send[q], recv[q], stream=stream)
+                if coll == "alltoall":
+                    comms[q].alltoall(send[q], recv[q], stream=stream)
+                else:
+                    comms[q].allreduce(send[q], recv[q], stream=stream)
 
     for _ in range(args.warmup):
         step()
@@ -296,8 +316,13 @@ def run_virtual(args):
     for c in comms:
         if c.async_error():
             raise RuntimeError("watchdog fired during the bench")
-    bad, total = sampled_parity(algo, recv, n, [0, R - 1])
-    res = {"t": t, "launches": launches, "clocks": clk, "parity_bad": bad, "parity_total": total,
+    if coll == "alltoall":  # bit-exact block permutation on the first and last rank
+        bad = sum(int(torch.count_nonzero(recv[q].view(R, -1)[p] != send[p].view(R, -1)[q]))
+                  for q in (0, R - 1) for p in range(R))
+        total = 2 * n
+    else:
+        bad, total = sampled_parity(algo, recv, n, [0, R - 1])
+    res = {"t": t, "coll": coll, "launches": launches, "clocks": clk, "parity_bad": bad, "parity_total": total,
            "algo": algo, "S": S, "R": R, "touches": touches, "direct": direct}
     # end-to-end through the public API with host buffers (pinned), every step
     if not args.no_e2e:
@@ -534,7 +559,8 @@ def main():
         res = run_virtual(args)
         R = args.ranks
     S, t, algo = res["S"], res["t"], res["algo"]
-    value = busbw("allreduce", S, t, R)
+    coll = res.get("coll", "allreduce")
+    value = busbw(coll, S, t, R)
     peak, peak_src = measured_peak()
     per_chunk = S / algo.gpus[0].i_chunks
     nranks_launch = R if world == 1 else 1
@@ -554,17 +580,31 @@ def main():
                 "kernel": "mscclInterpreter<bf16,sum>", "algorithmic_bytes_per_launch": int(S * 2 * (R - 1) / R),
                 "launch_ms": round(t * 1e3 / launches_per_step, 4)}
     else:
-        roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peak, "unit": "GB/s",
-                "frac": round(achieved / peak, 4), "traffic": traffic, "peak_source": peak_src,
-                "kernel": "mscclInterpreter<bf16,sum>", "algorithmic_bytes_per_launch": int(alg_bytes),
-                "launch_ms": round(t * 1e3 / launches_per_step, 4),
-                "compulsory_bytes_per_launch": int(2 * S * R),
-                "direct_placement": res.get("direct"),
-                "note": "algorithmic = per-instruction bytes of the program under the protocol (FIFO: 5.5 S per "
-                        "rank, SURVEY 8d; with direct placement 4.5 S), part of which stays in L2; traffic = ncu "
-                        "DRAM bytes per launch; compulsory = inputs read + outputs written"}
+        # All R ranks run in one launch on one GPU: the HBM bytes any implementation must move are
+        # every rank's input read once and its output written once.
+        launch_s = t / launches_per_step
+        compulsory = 2 * S * R
+        hbm_achieved = compulsory / launch_s / 1e9
+        l2peak, l2src = l2_peak()
+        is_default = (args.program, args.instances, args.channels, args.slot_kib, args.threads, args.protocol) == \
+            ("ring", 32, 1, 256, 256, "Simple")
+        roof = {"bound": "hbm", "achieved": round(hbm_achieved, 1), "peak": peak, "unit": "GB/s",
+                "frac": round(hbm_achieved / peak, 4), "traffic": traffic if is_default else None,
+                "peak_source": peak_src,
+                "kernel": "mscclInterpreter<bf16,%s,Simple>" % ("copy" if coll == "alltoall" else "sum"),
+                "algorithmic_bytes_per_launch": int(compulsory), "launch_ms": round(launch_s * 1e3, 4),
+                "note": "algorithmic = compulsory HBM bytes of one launch covering all %d ranks: every input read "
+                        "once + every output written once (2 S R); traffic = ncu dram read+write bytes per launch "
+                        "(profiles/ncu_summary.json, default config only)" % R,
+                "l2": {"touched_bytes_per_launch": int(alg_bytes), "achieved": round(achieved, 1),
+                       "peak": l2peak, "frac": round(achieved / l2peak, 4) if l2peak else None,
+                       "peak_source": l2src,
+                       "note": "touched = the program's per-instruction operand bytes (send 2, recv 2, copy 2, "
+                               "reduce/rrc/rrs 3, rrcs 4, rcs 3 chunks; a direct recv 0, a direct rcs 2), i.e. "
+                               "the L2-level traffic of the interpreter; FIFO slots live mostly in L2"},
+                "direct_placement": res.get("direct")}
     out = {
-        "metric": metric_name(), "value": round(value, 3), "unit": "GB/s", "n_gpus": N,
+        "metric": metric_name(coll), "value": round(value, 3), "unit": "GB/s", "n_gpus": N,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 4),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
         "data": "synthetic (counter-based uniform[-1,1) bf16, seed 20230325+rank)",

@@ -9,6 +9,7 @@
 namespace msccl {
 
 #define MSCCL_MAX_LOCAL 16  // ranks that one kernel launch may cover (virtual ranks)
+#define MSCCL_FLAG_WORDS 16 // u64 flag words per connection counter: one per warp (<= 512 threads)
 
 enum { DI_SEND_DIRECT = 1, DI_RECV_DIRECT = 2, DI_CHAIN_HEAD = 4 };
 
@@ -31,7 +32,10 @@ struct DevTB {
   uint32_t instrStart;
   int32_t tbId;
   int32_t sendPeer;           // rank of the send peer (-1 if none)
-  // send connection (peer = receiver): FIFO and head counter live in the PEER's region
+  // send connection (peer = receiver): FIFO and head counter live in the PEER's region.
+  // head/ack are arrays of MSCCL_FLAG_WORDS words: with warp flags (Simple protocol) warp w
+  // of the sender and warp w of the receiver own word w (reading R18); block-level protocols
+  // wait on word 0 and post every word.
   char* sendFifo;             // peer FIFO base for (me -> peer, chan); nullptr if no send peer
   uint64_t* sendHead;         // peer: messages posted by me
   uint64_t* sendAck;          // mine: messages the peer consumed (written by the peer)
@@ -71,7 +75,9 @@ struct KernelArgs {
   int32_t sysScope;           // 1 when any peer is another GPU
   int32_t useTma;             // Simple protocol: bulk-copy (TMA) pipeline through shared memory
   int32_t direct;             // honour DI_*_DIRECT flags (all ranks in this launch, rank == slot)
-  int32_t pad2;
+  int32_t warpFlags;          // Simple protocol: per-warp head/ack flags, no block barrier per message (R18)
+  int32_t prefetch;           // Simple protocol: bulk L2 prefetch of the local operand before a receive wait
+  int32_t pad3;
   uint64_t timeoutNs;
   uint64_t* trace;            // MSCCL_TRACE builds: per-CTA phase times (ns), else null
 };

@@ -234,6 +234,14 @@ __device__ __forceinline__ void stRelaxedGpu(uint64_t* p, uint64_t v) {
 }
 __device__ __forceinline__ void fenceSys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
 __device__ __forceinline__ void fenceGpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+// store v to every flag word of a connection counter (block-level protocols, DevTB comment)
+__device__ __forceinline__ void postWords(uint64_t* p, uint64_t v, bool sys) {
+#pragma unroll
+  for (int k = 0; k < MSCCL_FLAG_WORDS; k++) {
+    if (sys) stRelaxedSys(p + k, v);
+    else stRelaxedGpu(p + k, v);
+  }
+}
 __device__ __forceinline__ uint64_t globaltimer() {
   uint64_t t;
   asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
@@ -247,6 +255,7 @@ struct Ctx {
   const RankArgs* ra;
   int tid, nt;
   TmaState* tma;  // shared-memory pipeline state (Simple protocol with TMA), or null
+  uint64_t sent0; // messages posted on the send connection before this launch
 };
 
 static __device__ __noinline__ void raiseAbort(const KernelArgs& a) {
@@ -295,20 +304,22 @@ __device__ __forceinline__ void chunkSpan(const KernelArgs& a, int buf, int64_t 
 #define MSCCL_FENCE_MODE 0
 #endif
 #ifndef MSCCL_UNROLL
-#define MSCCL_UNROLL 4
+#define MSCCL_UNROLL 4   // vectors in flight per lane and input stream (two input streams)
+#endif
+#ifndef MSCCL_UNROLL1
+#define MSCCL_UNROLL1 8  // ... when the op reads one stream (copies, sends, receives): same registers
 #endif
 
 // Main vector loop: VB-byte vectors, U independent vectors in flight per thread.
 // Returns the number of VB-byte vectors processed.
 template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST, int VB>
 __device__ __forceinline__ int64_t vecLoop(int64_t nvec, const char* rslot, const char* src, char* dst, char* sslot,
-                                           const Ctx& c) {
+                                           int ti, int nt) {
   typedef typename VecT<VB>::T Vec;
-  constexpr int U = MSCCL_UNROLL;
+  constexpr int U = ((int)RECV + (int)SRC + (int)REDDST) >= 2 ? MSCCL_UNROLL : MSCCL_UNROLL1;
   const uint64_t pFirst = policyEvictFirst(), pLast = policyEvictLast();
-  const int nt = c.nt;
   const bool canDiscard = RECV && ((((uintptr_t)rslot) & 127) == 0);
-  const int lane = c.tid & 31, warp = c.tid >> 5, nw = nt >> 5;
+  const int lane = ti & 31, warp = ti >> 5, nw = nt >> 5;
   // Full blocks of U x 32 vectors, one block per warp-iteration (warp-uniform trip count,
   // so the __syncwarp below is reached by every lane); each u-row is 32 x VB contiguous bytes.
   const int64_t nblk = nvec / (U * 32);
@@ -339,7 +350,7 @@ __device__ __forceinline__ int64_t vecLoop(int64_t nvec, const char* rslot, cons
       }
     }
   }
-  for (int64_t i = nblk * (U * 32) + c.tid; i < nvec; i += nt) {
+  for (int64_t i = nblk * (U * 32) + ti; i < nvec; i += nt) {
     Vec x, y, v;
     if constexpr (RECV) ldFifo(x, rslot + i * VB);
     if constexpr (REDDST) ldStream(x, dst + i * VB, pFirst);
@@ -355,28 +366,29 @@ __device__ __forceinline__ int64_t vecLoop(int64_t nvec, const char* rslot, cons
 
 // ------------------------------------------------------------------ Simple-protocol piece
 // out = RECV&&SRC ? op(recv, src) : REDDST ? op(dst, src) : RECV ? recv : src
-// written to dst (DST) and/or the outgoing slot (SEND).
+// written to dst (DST) and/or the outgoing slot (SEND). Threads ti of [0, nt): the whole
+// block (nt = blockDim) or one warp (nt = 32, warp flags).
 template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
 __device__ __forceinline__ void pieceSimple(int64_t m, const char* rslot, const char* src, char* dst, char* sslot,
-                                            const Ctx& c) {
+                                            int ti, int nt) {
   typedef typename DType<DT>::T T;
   const int64_t bytes = m * (int64_t)sizeof(T);
   uintptr_t al = (uintptr_t)rslot | (uintptr_t)src | (uintptr_t)dst | (uintptr_t)sslot;
   int64_t done = 0;  // bytes handled by the vector paths
   if ((al & 31) == 0) {
-    done = 32 * vecLoop<DT, OP, RECV, SEND, SRC, DST, REDDST, 32>(bytes / 32, rslot, src, dst, sslot, c);
+    done = 32 * vecLoop<DT, OP, RECV, SEND, SRC, DST, REDDST, 32>(bytes / 32, rslot, src, dst, sslot, ti, nt);
   } else if ((al & 15) == 0) {
-    done = 16 * vecLoop<DT, OP, RECV, SEND, SRC, DST, REDDST, 16>(bytes / 16, rslot, src, dst, sslot, c);
+    done = 16 * vecLoop<DT, OP, RECV, SEND, SRC, DST, REDDST, 16>(bytes / 16, rslot, src, dst, sslot, ti, nt);
   }
   if ((al & 15) == 0 && bytes - done >= 16) {  // 16-byte remainder after the 32-byte path
     const int64_t off = done;
     const int64_t nv = (bytes - done) / 16;
     done += 16 * vecLoop<DT, OP, RECV, SEND, SRC, DST, REDDST, 16>(
                      nv, RECV ? rslot + off : nullptr, SRC ? src + off : nullptr, (DST || REDDST) ? dst + off : nullptr,
-                     SEND ? sslot + off : nullptr, c);
+                     SEND ? sslot + off : nullptr, ti, nt);
   }
   // scalar tail (ragged chunk end or unaligned buffers)
-  for (int64_t e = done / (int64_t)sizeof(T) + c.tid; e < m; e += c.nt) {
+  for (int64_t e = done / (int64_t)sizeof(T) + ti; e < m; e += nt) {
     T x = 0, y = 0, v;
     if constexpr (RECV) x = *(volatile const T*)(rslot + e * sizeof(T));
     if constexpr (REDDST) x = *(volatile const T*)(dst + e * sizeof(T));
@@ -604,6 +616,24 @@ __device__ __forceinline__ int64_t pieceGeom(const Ctx& c, const DevInstr& in, i
   return hi - a0;
 }
 
+// Bulk L2 prefetch (the TMA engine, no registers) of the local operand of an instruction that
+// is about to wait for its incoming message: the HBM reads of the source tile overlap the
+// wait instead of following it. Issued by one thread; purely a cache hint.
+template <int DT, bool SRC, bool DST, bool REDDST>
+__device__ __noinline__ void prefetchLocal(const Ctx& c, const DevInstr& in, int t) {
+  MSCCL_PIECE_GEOM
+  (void)a0;
+  for (int j = 0; j < in.cnt; j++) {
+    const char* src;
+    char* dst;
+    const int64_t m = pieceGeom<DT, SRC, DST, REDDST>(c, in, t, j, src, dst);
+    const char* p = SRC ? src : dst;
+    if (m * w < 16 || (((uintptr_t)p) & 15)) continue;
+    const uint32_t bytes = (uint32_t)((m * w) & ~(int64_t)15);
+    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+  }
+}
+
 template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
 __device__ __noinline__ void movePiecesSimple(const Ctx& c, const DevTB& tb, const DevInstr& in, int t,
                                               const char* rslot, char* sslot) {
@@ -623,10 +653,10 @@ __device__ __noinline__ void movePiecesSimple(const Ctx& c, const DevTB& tb, con
     }
     if (m <= 0) continue;
     if (rdirect) {  // the data is already in dst (the sender wrote it there)
-      if (SEND) pieceSimple<DT, OP, false, true, true, false, false>(m, nullptr, dst, nullptr, so, c);
+      if (SEND) pieceSimple<DT, OP, false, true, true, false, false>(m, nullptr, dst, nullptr, so, c.tid, c.nt);
       continue;
     }
-    pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, RECV ? rslot + j * a.T * w : nullptr, src, dst, so, c);
+    pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, RECV ? rslot + j * a.T * w : nullptr, src, dst, so, c.tid, c.nt);
   }
 }
 
@@ -700,12 +730,130 @@ __device__ __noinline__ bool movePiecesTma(const Ctx& c, const DevInstr& in, int
     const char* srcp = (RECV && SRC) || REDDST ? ps[j].inB : ps[j].inA;
     pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(
         ms[j] - e0, RECV ? ps[j].inA + k : nullptr, SRC ? srcp + k : nullptr,
-        (DST || REDDST) ? (REDDST ? (char*)ps[j].inA : ps[j].out0) + k : nullptr, SEND ? ps[j].out1 + k : nullptr, c);
+        (DST || REDDST) ? (REDDST ? (char*)ps[j].inA : ps[j].out0) + k : nullptr, SEND ? ps[j].out1 + k : nullptr, c.tid,
+        c.nt);
   }
   return true;
 }
 
 #endif  // MSCCL_ENABLE_TMA
+
+// ------------------------------------------------------------------ warp flags (reading R18)
+// Simple protocol without a block barrier per message. A piece of a tile (T elements) is cut
+// into nw contiguous byte ranges of P = ceil(T*w/nw) rounded up to 1 KiB (32 lanes x 32
+// bytes); warp w of every thread block moves range w of every piece, and head/ack word w of a
+// connection carries only warp w's progress. Sender warp w and receiver warp w therefore
+// form their own pipeline: a warp starts on its part of a message as soon as the upstream
+// warp with the same index has posted it, and the other warps on the SM keep the memory
+// system busy while it waits. The partition depends only on (T, nw), fixed for a launch:
+// every message that passes through a slot during a launch is cut the same way (so word w's
+// ack frees exactly the bytes sender warp w overwrites), and the program-order hazards of one
+// thread block (an instruction reading what an earlier one wrote, same chunk and tile) stay
+// inside one warp. A slot whose previous message belongs to an earlier launch (possibly cut
+// differently) is reused only when every word has acknowledged it.
+template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
+__device__ __noinline__ void movePiecesWarp(const Ctx& c, const DevTB& tb, const DevInstr& in, int t,
+                                            const char* rslot, char* sslot) {
+  MSCCL_PIECE_GEOM
+  const int lane = c.tid & 31, warp = c.tid >> 5, nw = c.nt >> 5;
+  const int64_t P = ((a.T * w + nw - 1) / nw + 1023) / 1024 * 1024;
+  const int64_t lo = (int64_t)warp * P;
+  if (lo >= (a.E - a0 < a.T ? a.E - a0 : a.T) * w) return;  // beyond tile t of a full chunk
+  const int64_t hiw = lo + P;
+  const bool sdirect = SEND && a.direct && (in.flags & DI_SEND_DIRECT);
+  const bool rdirect = RECV && a.direct && (in.flags & DI_RECV_DIRECT);
+  for (int j = 0; j < in.cnt; j++) {
+    const char* src;
+    char* dst;
+    int64_t m = pieceGeom<DT, SRC, DST, REDDST>(c, in, t, j, src, dst);
+    char* so = SEND ? sslot + j * a.T * w : nullptr;
+    if (sdirect) {  // reading R15: write straight into the receiver's destination chunk
+      int64_t rs, rl;
+      chunkSpan(a, in.rdstBuf, (int64_t)in.rdstOff + j, rs, rl);
+      so = a.rank[tb.sendPeer].buf[in.rdstBuf] + (rs + a0) * w;
+      if (rl - a0 < m) m = rl - a0;
+    }
+    const int64_t hi = hiw < m * w ? hiw : m * w;
+    if (hi <= lo) continue;
+    const int64_t mw = (hi - lo) / w;
+    if (rdirect) {  // the data is already in dst (the sender wrote it there)
+      if (SEND) pieceSimple<DT, OP, false, true, true, false, false>(mw, nullptr, dst + lo, nullptr, so + lo, lane, 32);
+      continue;
+    }
+    pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(mw, RECV ? rslot + j * a.T * w + lo : nullptr,
+                                                      SRC ? src + lo : nullptr, (DST || REDDST) ? dst + lo : nullptr,
+                                                      SEND ? so + lo : nullptr, lane, 32);
+  }
+}
+
+template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
+__device__ __noinline__ bool runOpWarp(const Ctx& c, const DevTB& tb, const DevInstr& in, int t, uint64_t& sent,
+                                       uint64_t& recvd) {
+  const KernelArgs& a = *c.a;
+  const int lane = c.tid & 31, warp = c.tid >> 5;
+  const bool sys = a.sysScope != 0;
+  bool ok = true;
+  if constexpr (RECV && (SRC || REDDST)) {
+    if (a.prefetch && c.tid == 32) prefetchLocal<DT, SRC, DST, REDDST>(c, in, t);
+  }
+  if (RECV && lane == 0) ok = waitGE(tb.recvHead + warp, recvd + 1, sys, c);
+  // a free slot for this warp's part (a direct message uses none, reading R15): the slot's
+  // previous message must be consumed -- by receiver warp w if this launch posted it, by every
+  // receiver warp if an earlier launch did (lanes 0..15 wait on one word each)
+  if (SEND && sent + 1 > (uint64_t)a.slots && !(a.direct && (in.flags & DI_SEND_DIRECT))) {
+    const uint64_t target = sent + 1 - (uint64_t)a.slots;
+    if (target > c.sent0) {
+      if (lane == 0) ok = ok && waitGE(tb.sendAck + warp, target, sys, c);
+    } else if (lane < MSCCL_FLAG_WORDS) {
+      ok = ok && waitGE(tb.sendAck + lane, target, sys, c);
+    }
+  }
+  if (!__all_sync(0xffffffffu, ok)) return false;
+  __syncwarp();  // lane 0's acquire orders the other lanes' reads (bar.warp.sync is a memory barrier among the warp)
+  const char* rslot = RECV ? tb.recvFifo + (int64_t)(recvd % (uint64_t)a.slots) * a.slotBytes : nullptr;
+  char* sslot = SEND ? tb.sendFifo + (int64_t)(sent % (uint64_t)a.slots) * a.slotBytes : nullptr;
+  movePiecesWarp<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, tb, in, t, rslot, sslot);
+  if (RECV || SEND) {
+    __syncwarp();
+    if (lane == 0) {  // release: this warp's stores (and consumed reads) before its flag words
+      if (sys) fenceSys();
+      else fenceGpu();
+      if (SEND) {
+        if (sys) stRelaxedSys(tb.sendHead + warp, sent + 1);
+        else stRelaxedGpu(tb.sendHead + warp, sent + 1);
+      }
+      if (RECV) {
+        if (sys) stRelaxedSys(tb.recvAck + warp, recvd + 1);
+        else stRelaxedGpu(tb.recvAck + warp, recvd + 1);
+      }
+    }
+  }
+  if (SEND) sent++;
+  if (RECV) recvd++;
+  return true;
+}
+
+template <int DT, int OP>
+__device__ __forceinline__ bool dispatchWarp(const Ctx& c, const DevTB& tb, const DevInstr& in, int t, uint64_t& sent,
+                                             uint64_t& recvd) {
+  switch (in.op) {
+    case K_SEND: return runOpWarp<DT, OP, false, true, true, false, false>(c, tb, in, t, sent, recvd);
+    case K_RECV: return runOpWarp<DT, OP, true, false, false, true, false>(c, tb, in, t, sent, recvd);
+    case K_COPY: return runOpWarp<DT, OP, false, false, true, true, false>(c, tb, in, t, sent, recvd);
+    case K_RCS: return runOpWarp<DT, OP, true, true, false, true, false>(c, tb, in, t, sent, recvd);
+    default: break;
+  }
+  if (OP != R_COPY) {
+    switch (in.op) {
+      case K_REDUCE: return runOpWarp<DT, OP, false, false, true, true, true>(c, tb, in, t, sent, recvd);
+      case K_RRC: return runOpWarp<DT, OP, true, false, true, true, false>(c, tb, in, t, sent, recvd);
+      case K_RRS: return runOpWarp<DT, OP, true, true, true, false, false>(c, tb, in, t, sent, recvd);
+      case K_RRCS: return runOpWarp<DT, OP, true, true, true, true, false>(c, tb, in, t, sent, recvd);
+      default: break;
+    }
+  }
+  return true;  // nop
+}
 
 // ------------------------------------------------------------------ one instruction, one tile
 template <int DT, int OP, int PROTO, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
@@ -719,14 +867,19 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
 #if MSCCL_TRACE
   uint64_t tr0 = c.tid == 0 ? globaltimer() : 0, tr1 = 0, tr2 = 0, tr3 = 0, tr4 = 0;
 #endif
+  if constexpr (!ll && RECV && (SRC || REDDST)) {
+    if (a.prefetch && c.tid == 64) prefetchLocal<DT, SRC, DST, REDDST>(c, in, t);
+  }
   if (RECV && !ll && c.tid == 0) ok = waitGE(tb.recvHead, recvd + 1, sys, c);
 #if MSCCL_TRACE
   if (c.tid == 0) tr1 = globaltimer();
 #endif
   // a free slot: at most `slots` messages posted and not yet consumed (§6.1)
   // (a direct message uses no slot: no credit needed, reading R15)
-  if (SEND && c.tid == (RECV ? 32 : 0) && sent + 1 > (uint64_t)a.slots && !(a.direct && (in.flags & DI_SEND_DIRECT)))
-    ok = ok && waitGE(tb.sendAck, sent + 1 - (uint64_t)a.slots, sys, c);
+  // (every ack word: a warp-flag launch before this one may have acknowledged word by word)
+  if (SEND && c.tid >= 32 && c.tid < 32 + MSCCL_FLAG_WORDS && sent + 1 > (uint64_t)a.slots &&
+      !(a.direct && (in.flags & DI_SEND_DIRECT)))
+    ok = ok && waitGE(tb.sendAck + (c.tid - 32), sent + 1 - (uint64_t)a.slots, sys, c);
   if (!ok) *sAbort = 1;
   if (RECV || SEND) {
     __syncthreads();
@@ -756,27 +909,14 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
 #if MSCCL_TRACE
   if (c.tid == 0) tr4 = globaltimer();
 #endif
+  // block-level protocols post every flag word (a later warp-flag launch waits on its own word)
   if (c.tid == 0 && ll && RECV) {  // LL/LL128: data carried its own flags; the ack frees the slot
-    if (sys) stRelaxedSys(tb.recvAck, recvd + 1);
-    else stRelaxedGpu(tb.recvAck, recvd + 1);
+    postWords(tb.recvAck, recvd + 1, sys);
   } else if (c.tid == 0 && (RECV || SEND) && !ll) {
-    if (sys) {
-      fenceSys();
-      if (SEND) stRelaxedSys(tb.sendHead, sent + 1);
-      if (RECV) stRelaxedSys(tb.recvAck, recvd + 1);
-    } else {
-#if MSCCL_FENCE_MODE == 1
-      if (SEND && !ll) asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(tb.sendHead), "l"(sent + 1) : "memory");
-      if (RECV) asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(tb.recvAck), "l"(recvd + 1) : "memory");
-#elif MSCCL_FENCE_MODE == 2
-      if (SEND && !ll) stRelaxedGpu(tb.sendHead, sent + 1);
-      if (RECV) stRelaxedGpu(tb.recvAck, recvd + 1);
-#else
-      fenceGpu();
-      if (SEND && !ll) stRelaxedGpu(tb.sendHead, sent + 1);
-      if (RECV) stRelaxedGpu(tb.recvAck, recvd + 1);
-#endif
-    }
+    if (sys) fenceSys();
+    else fenceGpu();
+    if (SEND) postWords(tb.sendHead, sent + 1, sys);
+    if (RECV) postWords(tb.recvAck, recvd + 1, sys);
   }
 #if MSCCL_TRACE
   if (c.tid == 0 && a.trace) {
@@ -859,8 +999,10 @@ __device__ __noinline__ void chainExec(const Ctx& c, const DevInstr* mem, int L,
         int64_t Lk = sl < dl ? sl : dl;
         int64_t mk = (a0 + a.T < Lk ? a0 + a.T : Lk) - a0;
         if (mk > 0) {
-          if (mem[k].op == K_COPY) pieceSimple<DT, OP, false, false, true, true, false>(mk, nullptr, srcs[k], dst, nullptr, c);
-          else pieceSimple<DT, OP, false, false, true, true, true>(mk, nullptr, srcs[k], dst, nullptr, c);
+          if (mem[k].op == K_COPY)
+            pieceSimple<DT, OP, false, false, true, true, false>(mk, nullptr, srcs[k], dst, nullptr, c.tid, c.nt);
+          else
+            pieceSimple<DT, OP, false, false, true, true, true>(mk, nullptr, srcs[k], dst, nullptr, c.tid, c.nt);
         }
         __syncthreads();
       }
@@ -900,7 +1042,7 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
   const int tbi = (int)blockIdx.x - ra.ctaStart;
   if (tbi >= ra.nTB) return;
   const DevTB& tb = ra.tbs[tbi];
-  Ctx c{&a, &ra, (int)threadIdx.x, (int)blockDim.x, nullptr};
+  Ctx c{&a, &ra, (int)threadIdx.x, (int)blockDim.x, nullptr, 0};
 #if MSCCL_ENABLE_TMA
   if (a.useTma && PROTO == 0) {
     c.tma = &sTma;
@@ -921,8 +1063,14 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
 #endif
   if (threadIdx.x == 0) sAbort = 0;
   uint64_t sent = tb.sendFifo ? *(volatile uint64_t*)tb.sendCnt : 0;
+  c.sent0 = sent;
   uint64_t recvd = tb.recvFifo ? *(volatile uint64_t*)tb.recvCnt : 0;
   const uint64_t gen = *(volatile uint64_t*)&ra.gen[tbi];
+  // warp flags (R18): a warp whose wait failed (watchdog / abort) keeps walking the program
+  // without doing anything, so the block-wide barriers below still match; at the next one
+  // every thread sees sAbort and returns.
+  const bool warpMode = PROTO == 0 && a.warpFlags;
+  bool dead = false;
   __syncthreads();
   for (int t = 0; t < a.I; t++) {
     for (int s = 0; s < tb.nSteps; s++) {
@@ -965,7 +1113,23 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
         __syncthreads();
         if (sAbort) return;
       }
-      if (!dispatch<DT, OP, PROTO>(c, tb, in, t, sent, recvd, &sAbort)) return;
+      if constexpr (PROTO == 0) {
+        if (warpMode) {
+          if (!dead && *(volatile int*)&sAbort) dead = true;
+          if (!dead && !dispatchWarp<DT, OP>(c, tb, in, t, sent, recvd)) {
+            dead = true;
+            sAbort = 1;
+          }
+          if (in.hasDep) {  // every warp's part of the step is done before the semaphore moves
+            __syncthreads();
+            if (sAbort) return;
+          }
+        } else if (!dispatch<DT, OP, PROTO>(c, tb, in, t, sent, recvd, &sAbort)) {
+          return;
+        }
+      } else {
+        if (!dispatch<DT, OP, PROTO>(c, tb, in, t, sent, recvd, &sAbort)) return;
+      }
       if (in.hasDep) {  // Fig. 5 lines 25-27: the step is complete before the semaphore moves
         if (c.tid == 0) {
           fenceGpu();
@@ -974,9 +1138,21 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
       }
     }
   }
+  if (warpMode) {
+    __syncthreads();
+    if (sAbort) return;
+  }
   if (threadIdx.x == 0) {
     if (tb.sendFifo) *(volatile uint64_t*)tb.sendCnt = sent;
-    if (tb.recvFifo) *(volatile uint64_t*)tb.recvCnt = recvd;
+    if (tb.recvFifo) {
+      *(volatile uint64_t*)tb.recvCnt = recvd;
+      // words no warp of this launch owned: everything received is consumed (a later launch
+      // with more warps waits on them)
+      for (int k = blockDim.x >> 5; k < MSCCL_FLAG_WORDS; k++) {
+        if (a.sysScope) stRelaxedSys(tb.recvAck + k, recvd);
+        else stRelaxedGpu(tb.recvAck + k, recvd);
+      }
+    }
     *(volatile uint64_t*)&ra.gen[tbi] = gen + 1;
   }
 }

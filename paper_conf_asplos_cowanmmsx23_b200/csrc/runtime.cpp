@@ -26,7 +26,8 @@ using namespace msccl;
 namespace {
 
 struct Params {
-  int64_t slots = 4, slotBytes = 262144, maxChannels = 32, threads = 512, timeoutS = 20, tma = 0, direct = 1;
+  int64_t slots = 4, slotBytes = 262144, maxChannels = 32, threads = 512, timeoutS = 20, tma = 0, direct = 1,
+          warp = 0, l2PersistMiB = 0, prefetch = 0, directTile = 1;
 };
 
 std::mutex gMu;
@@ -43,6 +44,10 @@ int64_t* paramRef(Params& p, const std::string& k) {
   if (k == "MSCCL_TIMEOUT_S") return &p.timeoutS;
   if (k == "MSCCL_TMA") return &p.tma;
   if (k == "MSCCL_DIRECT") return &p.direct;
+  if (k == "MSCCL_WARP_FLAGS") return &p.warp;
+  if (k == "MSCCL_L2_PERSIST_MIB") return &p.l2PersistMiB;
+  if (k == "MSCCL_PREFETCH") return &p.prefetch;
+  if (k == "MSCCL_DIRECT_TILE") return &p.directTile;
   return nullptr;
 }
 
@@ -51,7 +56,8 @@ Params currentParams() {
   if (!gEnvRead) {
     gEnvRead = true;
     for (const char* k : {"MSCCL_SLOTS", "MSCCL_SLOT_BYTES", "MSCCL_MAX_CHANNELS", "MSCCL_THREADS", "MSCCL_TIMEOUT_S",
-                          "MSCCL_TMA", "MSCCL_DIRECT"}) {
+                          "MSCCL_TMA", "MSCCL_DIRECT", "MSCCL_WARP_FLAGS",
+                          "MSCCL_L2_PERSIST_MIB", "MSCCL_PREFETCH", "MSCCL_DIRECT_TILE"}) {
       const char* v = getenv(k);
       if (v && *v) *paramRef(gParams, k) = atoll(v);
     }
@@ -99,8 +105,9 @@ struct mscclComm {
   size_t fifoOff(int src, int ch) const {
     return ((size_t)src * prm.maxChannels + ch) * prm.slots * prm.slotBytes;
   }
-  size_t flagOff(int kind, int peer, int ch) const {  // kind: 0 head, 1 ack, 2 sendCnt, 3 recvCnt
-    return flagsOff + (((size_t)kind * nranks + peer) * prm.maxChannels + ch) * sizeof(uint64_t);
+  // kind: 0 head, 1 ack, 2 sendCnt, 3 recvCnt; MSCCL_FLAG_WORDS words (one 128-byte line) each
+  size_t flagOff(int kind, int peer, int ch) const {
+    return flagsOff + (((size_t)kind * nranks + peer) * prm.maxChannels + ch) * MSCCL_FLAG_WORDS * sizeof(uint64_t);
   }
   size_t abortOff() const { return flagOff(4, 0, 0); }
 };
@@ -119,6 +126,7 @@ struct mscclProgram {
   size_t scratchBytes = 0;
   int maxCnt = 1;
   bool hasReduce = false;
+  bool allDirect = true;  // every message of this rank's program is a direct placement (R15)
 };
 
 namespace {
@@ -163,6 +171,10 @@ mscclResult_t allocRegion(mscclComm* c) {
   c->regionBytes = c->abortOff() + 256;
   CUDACHECK(c, cudaMalloc(&c->region, c->regionBytes));
   CUDACHECK(c, cudaMemset(c->region, 0, c->regionBytes));
+  // optional L2 set-aside for evict_last (persisting) lines: the FIFO slot stores carry
+  // L2::evict_last, which only has a reserved home when the set-aside is non-zero
+  if (c->prm.l2PersistMiB > 0)
+    CUDACHECK(c, cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)c->prm.l2PersistMiB << 20));
   CUDACHECK(c, cudaHostAlloc(&c->hostAbort, sizeof(uint32_t), cudaHostAllocMapped | cudaHostAllocPortable));
   *c->hostAbort = 0;
   CUDACHECK(c, cudaHostGetDevicePointer((void**)&c->hostAbortDev, c->hostAbort, 0));
@@ -242,7 +254,9 @@ struct Geometry {
   int I, cb;
 };
 
-mscclResult_t geometry(mscclComm* c, const mscclProgram* p, int dtype, int64_t n, Geometry& g) {
+// noFifo: every message of the launch is a direct placement (R15), so no FIFO slot bounds
+// the tile: T = E (one message per chunk; results do not depend on T, reading R3).
+mscclResult_t geometry(mscclComm* c, const mscclProgram* p, int dtype, int64_t n, Geometry& g, bool noFifo = false) {
   const int w = elemBytes(dtype);
   const int V = 16 / w;
   const int R = p->algo.ngpus;
@@ -256,6 +270,7 @@ mscclResult_t geometry(mscclComm* c, const mscclProgram* p, int dtype, int64_t n
   else
     t = (p->algo.proto == PROTO_LL ? c->prm.slotBytes / 2 : c->prm.slotBytes) / ((int64_t)p->maxCnt * w) / V * V;
   if (t < V) return setErr(c, mscclInvalidUsage, "FIFO slot too small for the program's largest count");
+  if (noFifo) t = g.E;
   g.T = std::min<int64_t>(t, g.E);
   g.I = (int)((g.E + g.T - 1) / g.T);
   return mscclSuccess;
@@ -297,8 +312,14 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
         return setErr(cl->comm, mscclInvalidUsage, "ranks in a group disagree on program/count/datatype/op");
     }
     mscclProgram* p0 = v[0]->prog;
+    // direct placement needs every rank's buffers in this launch (rank r at slot r) and the
+    // Simple protocol; one launch covering all ranks also orders it against earlier launches
+    const bool useTma = p0->algo.proto == PROTO_SIMPLE && c0->prm.tma && tmaSmemBytes() > 0;
+    const bool direct = p0->algo.proto == PROTO_SIMPLE && c0->prm.direct && (int)v.size() == p0->algo.ngpus && !useTma;
+    bool noFifo = direct && c0->prm.directTile;
+    for (auto* cl : v) noFifo = noFifo && cl->prog->allDirect;
     Geometry g{};
-    mscclResult_t r = geometry(c0, p0, v[0]->dtype, v[0]->n, g);
+    mscclResult_t r = geometry(c0, p0, v[0]->dtype, v[0]->n, g, noFifo);
     if (r != mscclSuccess) return r;
     KernelArgs ka;
     memset(&ka, 0, sizeof(ka));
@@ -339,10 +360,10 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
     if (cta == 0) continue;
     const void* fn = p0->hasReduce ? interpreterKernel(v[0]->dtype, v[0]->op, ka.proto)
                                    : copyKernel(elemBytes(v[0]->dtype), ka.proto);
-    ka.useTma = (ka.proto == 0 && c0->prm.tma && tmaSmemBytes() > 0) ? 1 : 0;
-    // direct placement needs every rank's buffers in this launch (rank r at slot r) and the
-    // Simple protocol; one launch covering all ranks also orders it against earlier launches
-    ka.direct = (ka.proto == 0 && c0->prm.direct && ka.nLocal == p0->algo.ngpus && !ka.useTma) ? 1 : 0;
+    ka.useTma = useTma ? 1 : 0;
+    ka.direct = direct ? 1 : 0;
+    ka.warpFlags = (ka.proto == 0 && c0->prm.warp && !ka.useTma) ? 1 : 0;
+    ka.prefetch = (ka.proto == 0 && c0->prm.prefetch) ? 1 : 0;
     const int smem = ka.useTma ? tmaSmemBytes() : 0;
     int maxCta = 0;
     r = coResident(c0, fn, (int)c0->prm.threads, smem, maxCta);
@@ -554,9 +575,10 @@ mscclResult_t mscclCommExportHandle(mscclComm_t c, void* handle, size_t* bytes) 
   DeviceGuard g(c->dev);
   cudaIpcMemHandle_t h;
   CUDACHECK(c, cudaIpcGetMemHandle(&h, c->region));
-  static_assert(sizeof(h) + 16 <= MSCCL_HANDLE_BYTES, "handle size");
+  static_assert(sizeof(h) + 32 <= MSCCL_HANDLE_BYTES, "handle size");
   memcpy(handle, &h, sizeof(h));
-  int64_t meta[2] = {(int64_t)c->regionBytes, (int64_t)c->dev};
+  // parameters that both ends of a connection must agree on (region layout, warp partition)
+  int64_t meta[4] = {(int64_t)c->regionBytes, (int64_t)c->dev, c->prm.threads, c->prm.warp};
   memcpy((char*)handle + sizeof(h), meta, sizeof(meta));
   if (bytes) *bytes = MSCCL_HANDLE_BYTES;
   return mscclSuccess;
@@ -571,9 +593,11 @@ mscclResult_t mscclCommConnect(mscclComm_t c, const void* allHandles) {
     const char* h = (const char*)allHandles + (size_t)p * MSCCL_HANDLE_BYTES;
     cudaIpcMemHandle_t ih;
     memcpy(&ih, h, sizeof(ih));
-    int64_t meta[2];
+    int64_t meta[4];
     memcpy(meta, h + sizeof(ih), sizeof(meta));
     if ((size_t)meta[0] != c->regionBytes) return setErr(c, mscclInvalidUsage, "peer region size differs (ranks use different MSCCL_* parameters)");
+    if (meta[2] != c->prm.threads || meta[3] != c->prm.warp)
+      return setErr(c, mscclInvalidUsage, "peer uses different MSCCL_THREADS / MSCCL_WARP_FLAGS (the warp partition must match)");
     void* ptr = nullptr;
     CUDACHECK(c, cudaIpcOpenMemHandle(&ptr, ih, cudaIpcMemLazyEnablePeerAccess));
     c->peerBase[p] = (char*)ptr;
@@ -703,6 +727,8 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
       di.depStart = (uint32_t)deps.size();
       for (auto& dp : in.deps) deps.push_back(((uint32_t)dp.first << 16) | (uint32_t)dp.second);
       if (dinfo.recvDirect[t][si]) di.flags |= DI_RECV_DIRECT;
+      const bool sends = in.op == OP_SEND || in.op == OP_RRS || in.op == OP_RRCS || in.op == OP_RCS;
+      if (sends && !dinfo.sendDirect[t][si]) p->allDirect = false;
       if (dinfo.sendDirect[t][si]) {
         di.flags |= DI_SEND_DIRECT;
         di.rdstBuf = (uint8_t)dinfo.rdstBuf[t][si];

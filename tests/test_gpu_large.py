@@ -12,16 +12,21 @@ from paper_conf_asplos_cowanmmsx23_b200 import programs as P
 pytestmark = pytest.mark.gpu
 
 
-@pytest.fixture(scope="module", autouse=True, params=[1, 0], ids=["direct", "fifo"])
+@pytest.fixture(scope="module", autouse=True, params=[(1, 0), (0, 0), (1, 1), (0, 1)],
+                ids=["direct", "fifo", "warp-direct", "warp-fifo"])
 def production_params(request):
     """Production launch parameters; every test runs with direct placement (reading R15)
-    and with it disabled (all messages through the receiver-side FIFO)."""
+    and with it disabled (all messages through the receiver-side FIFO), each with block-level
+    and with per-warp (reading R18) flags of the Simple protocol."""
     from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    direct, warp = request.param
     for k, v in (("MSCCL_SLOT_BYTES", 262144), ("MSCCL_SLOTS", 4), ("MSCCL_THREADS", 256),
-                 ("MSCCL_MAX_CHANNELS", 32), ("MSCCL_TIMEOUT_S", 10), ("MSCCL_DIRECT", request.param)):
+                 ("MSCCL_MAX_CHANNELS", 32), ("MSCCL_TIMEOUT_S", 10), ("MSCCL_DIRECT", direct),
+                 ("MSCCL_WARP_FLAGS", warp)):
         runtime.set_param(k, v)
     yield
     runtime.set_param("MSCCL_DIRECT", 1)
+    runtime.set_param("MSCCL_WARP_FLAGS", 0)
 
 
 @pytest.mark.parametrize("r,extra", [(4, 12345), (3, 7), (2, 131072 * 2 + 999)])
@@ -47,6 +52,23 @@ def test_alltoall_and_allgather_default_slots():
     xs = synth.inputs(R, n, "int32", "pattern")
     got = gpu_util.run_program(P.ring_allgather(R, 1, 4).to_xml(), xs, n, "int32", out_elems=R * n)
     assert all(np.array_equal(g, e) for g, e in zip(got, mpi_ref.allgather(xs)))
+
+
+def test_protocols_share_connections():
+    """Simple, LL128 and LL programs (and two tile sizes) alternate on the same connections
+    of one communicator set: the monotone counters and every ack word stay consistent
+    across launches whatever protocol or warp partition the previous launch used."""
+    import gpu_util
+    R = 8
+    seq = [("Simple", 300001), ("LL128", 40000), ("Simple", 70001), ("LL", 9000), ("Simple", 300001),
+           ("Simple", 5000), ("LL128", 300001), ("Simple", 131072 * 3 + 17)]
+    for proto, n in seq:
+        ir = P.ring_allreduce(R, instances=2, protocol=proto).to_xml()
+        xs = synth.inputs(R, n, "float32", "uniform")
+        want = sim.simulate(irparse.parse(ir), xs, n, "float32", "sum")
+        got = gpu_util.run_program(ir, xs, n, "float32", "sum")
+        for g, w in zip(got, want):
+            assert np.array_equal(g.view(np.uint32), w.view(np.uint32)), (proto, n)
 
 
 @pytest.mark.parametrize("instances", [16, 32])

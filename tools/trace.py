@@ -27,6 +27,10 @@ def run(**kw):
     a[:] = 0
     np.ctypeslib.as_array(p, shape=(4096, 8))[:] = 0
 
-run()
-run(slot_kib=128)
-run(slot_kib=512, instances=16, threads=512)
+if __name__ == "__main__":
+    if len(sys.argv) > 1 and sys.argv[1] == "alltoall":
+        for kib in (256, 1024):
+            run(program="alltoall", instances=2, slot_kib=kib)
+    else:
+        for kib in (64, 128, 256, 512):
+            run(slot_kib=kib)
