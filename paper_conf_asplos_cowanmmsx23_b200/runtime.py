@@ -60,6 +60,7 @@ for _name, (_res, _args) in SIGNATURES.items():
     _f = getattr(lib, _name)
     _f.restype = _res
     _f.argtypes = _args
+_run_program = lib.mscclRunProgram
 
 
 class MscclError(RuntimeError):
@@ -95,21 +96,29 @@ def validate(ir_text, nranks, slots=0, max_tbs=0):
     return r == 0, err.value.decode()
 
 
+_TORCH_DT = None
+
+
 def _dtype_name(t):
-    import torch
-    m = {torch.int8: "int8", torch.uint8: "uint8", torch.int32: "int32", torch.int64: "int64",
-         torch.float16: "float16", torch.float32: "float32", torch.float64: "float64", torch.bfloat16: "bfloat16"}
-    for k in ("uint32", "uint64"):
-        if hasattr(torch, k):
-            m[getattr(torch, k)] = k
-    return m[t.dtype]
+    global _TORCH_DT
+    if _TORCH_DT is None:  # built once: this sits on the per-call path
+        import torch
+        m = {torch.int8: "int8", torch.uint8: "uint8", torch.int32: "int32", torch.int64: "int64",
+             torch.float16: "float16", torch.float32: "float32", torch.float64: "float64",
+             torch.bfloat16: "bfloat16"}
+        for k in ("uint32", "uint64"):
+            if hasattr(torch, k):
+                m[getattr(torch, k)] = k
+        _TORCH_DT = m
+    return _TORCH_DT[t.dtype]
 
 
 def _stream(stream):
-    import torch
     if stream is None:
+        import torch
         stream = torch.cuda.current_stream()
-    return _vp(stream.cuda_stream if hasattr(stream, "cuda_stream") else int(stream))
+    s = getattr(stream, "cuda_stream", None)
+    return s if s is not None else int(stream)
 
 
 @contextlib.contextmanager
@@ -239,5 +248,7 @@ class Comm:
 
     def run(self, prog, send, recv, count, op="sum", stream=None, dtype=None):
         dt = DTYPES[dtype or _dtype_name(send)]
-        _check(lib.mscclRunProgram(prog.handle, _vp(send.data_ptr()), _vp(recv.data_ptr()), count, dt, OPS[op],
-                                   self.handle, _stream(stream)), self.handle)
+        r = _run_program(prog.handle, send.data_ptr(), recv.data_ptr(), count, dt, OPS[op], self.handle,
+                         _stream(stream))
+        if r:
+            _check(r, self.handle)
