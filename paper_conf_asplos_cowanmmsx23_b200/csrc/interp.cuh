@@ -504,95 +504,137 @@ __device__ __forceinline__ bool pieceLL(int64_t m, int64_t sendUnits, const char
 // no separate head counter are needed. Lines per piece message: ceil(min(T, E - t*T)*w/120)
 // (the sender pads, reading R2).
 #ifndef MSCCL_LL128_UNROLL
-#define MSCCL_LL128_UNROLL 4
+#define MSCCL_LL128_UNROLL 4  // lines in flight per 8-lane group of a warp
 #endif
+// One batch of 4*U lines of a warp (8 lanes per line, U lines per lane group). FULL: every
+// line of the batch carries 120 payload bytes and the user pointers are 8-byte aligned, so
+// the payload moves as plain 8-byte words (no ragged-edge logic).
+template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool FULL>
+__device__ __forceinline__ bool ll128Batch(int64_t base, int64_t bytes, int64_t lines, int64_t total, const char* rslot,
+                                           const char* src, char* dst, char* sslot, uint64_t rflag, uint64_t sflag,
+                                           int g, int sub, const Ctx& c) {
+  constexpr int U = MSCCL_LL128_UNROLL;
+  const int64_t lb = g == 7 ? 8 : 16;  // payload bytes of this lane in a line
+  // 1. the local operand of every line this lane owns, loaded before the flag poll so its
+  //    latency overlaps the wait for the incoming line
+  uint64_t b0[U], b1[U];
+#pragma unroll
+  for (int u = 0; u < U; u++) {
+    b0[u] = b1[u] = 0;
+    if constexpr (SRC) {
+      const int64_t po = (base + u * 4 + sub) * 120 + g * 16;
+      if (FULL) {
+        b0[u] = *(const uint64_t*)(src + po);
+        if (g != 7) b1[u] = *(const uint64_t*)(src + po + 8);
+      } else {
+        int64_t nb = bytes - po;
+        nb = nb < 0 ? 0 : (nb > lb ? lb : nb);
+        if (nb > 0) {
+          const int64_t nb0 = nb > 8 ? 8 : nb;
+          b0[u] = loadUnitPlain(src + po, nb0);
+          if (nb > 8) b1[u] = loadUnitPlain(src + po + 8, nb - 8);
+        }
+      }
+    }
+  }
+  // 2. the incoming lines: poll until every line of the batch carries this message's flag
+  uint64_t x0[U], x1[U];
+  if constexpr (RECV) {
+    uint4 l[U];
+    uint64_t t0 = 0;
+    for (uint32_t it = 0;; it++) {
+      bool mine = true;
+#pragma unroll
+      for (int u = 0; u < U; u++) {
+        const int64_t L = base + u * 4 + sub;
+        if (FULL || L < lines) {
+          l[u] = ldvol(rslot + L * 128 + g * 16);
+          if (g == 7 && ((uint64_t)l[u].z | ((uint64_t)l[u].w << 32)) != rflag) mine = false;
+        }
+      }
+      if (__all_sync(0xffffffffu, mine)) break;
+      if (it >= 8) __nanosleep(64);  // back off after a few empty polls (L2 traffic)
+      if ((it & 255u) == 255u) {
+        uint64_t now = globaltimer();
+        if (t0 == 0) t0 = now;
+        if (*(volatile uint32_t*)c.ra->abortFlag) return false;
+        if (now - t0 > c.a->timeoutNs) {
+          raiseAbort(*c.a);
+          return false;
+        }
+      }
+    }
+#pragma unroll
+    for (int u = 0; u < U; u++) {
+      x0[u] = (uint64_t)l[u].x | ((uint64_t)l[u].y << 32);
+      x1[u] = (uint64_t)l[u].z | ((uint64_t)l[u].w << 32);
+    }
+  }
+  // 3. combine; store to dst and/or the outgoing lines
+#pragma unroll
+  for (int u = 0; u < U; u++) {
+    const int64_t L = base + u * 4 + sub;
+    if (!FULL && L >= total) continue;
+    const int64_t po = L * 120 + g * 16;
+    int64_t nb = lb;
+    if (!FULL) {
+      nb = bytes - po;
+      nb = nb < 0 ? 0 : (nb > lb ? lb : nb);
+    }
+    uint64_t v0 = 0, v1 = 0;
+    if constexpr (RECV && SRC) {  // op(received, local), as in every protocol
+      v0 = unitOp<DT, OP>(x0[u], b0[u]);
+      v1 = unitOp<DT, OP>(x1[u], b1[u]);
+    } else if constexpr (RECV) {
+      v0 = x0[u];
+      v1 = x1[u];
+    } else {
+      v0 = b0[u];
+      v1 = b1[u];
+    }
+    if constexpr (DST) {
+      if (FULL) {
+        *(uint64_t*)(dst + po) = v0;
+        if (g != 7) *(uint64_t*)(dst + po + 8) = v1;
+      } else if (nb > 0) {
+        const int64_t nb0 = nb > 8 ? 8 : nb;
+        storeUnitPlain(dst + po, v0, nb0);
+        if (nb > 8) storeUnitPlain(dst + po + 8, v1, nb - 8);
+      }
+    }
+    if constexpr (SEND) {
+      if (nb == 0) v0 = 0;  // padding line (R2): deterministic zeros
+      if (nb <= 8) v1 = 0;
+      if (g == 7) v1 = sflag;
+      stvol(sslot + L * 128 + g * 16, make_uint4((uint32_t)v0, (uint32_t)(v0 >> 32), (uint32_t)v1, (uint32_t)(v1 >> 32)));
+    }
+  }
+  return true;
+}
+
 template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
 __device__ __forceinline__ bool pieceLL128(int64_t m, int64_t sendLines, const char* rslot, const char* src, char* dst,
                                            char* sslot, uint64_t rflag, uint64_t sflag, const Ctx& c) {
   typedef typename DType<DT>::T T;
+  static_assert(!REDDST, "local reduces take the Simple path");
   constexpr int U = MSCCL_LL128_UNROLL;
   const int64_t bytes = m > 0 ? m * (int64_t)sizeof(T) : 0;
   const int64_t lines = (bytes + 119) / 120;
   const int64_t total = SEND ? (lines > sendLines ? lines : sendLines) : lines;
   const int lane = c.tid & 31, warp = c.tid >> 5, nw = c.nt >> 5;
   const int g = lane & 7, sub = lane >> 3;
-  bool ok = true;
+  const bool aligned = ((((uintptr_t)src) | ((uintptr_t)dst)) & 7) == 0;
   for (int64_t base = (int64_t)warp * 4 * U; base < total; base += (int64_t)nw * 4 * U) {
-    uint64_t x0[U], x1[U];
-    if constexpr (RECV) {
-      uint4 l[U];
-      uint64_t t0 = 0;
-      for (uint32_t it = 0;; it++) {
-        bool mine = true;
-#pragma unroll
-        for (int u = 0; u < U; u++) {
-          const int64_t L = base + u * 4 + sub;
-          if (L < lines) {
-            l[u] = ldvol(rslot + L * 128 + g * 16);
-            if (g == 7 && ((uint64_t)l[u].z | ((uint64_t)l[u].w << 32)) != rflag) mine = false;
-          }
-        }
-        if (__all_sync(0xffffffffu, mine)) break;
-        if ((it & 1023u) == 1023u) {
-          uint64_t now = globaltimer();
-          if (t0 == 0) t0 = now;
-          if (*(volatile uint32_t*)c.ra->abortFlag) { ok = false; break; }
-          if (now - t0 > c.a->timeoutNs) { raiseAbort(*c.a); ok = false; break; }
-        }
-      }
-      if (!ok) break;
-#pragma unroll
-      for (int u = 0; u < U; u++) {
-        x0[u] = (uint64_t)l[u].x | ((uint64_t)l[u].y << 32);
-        x1[u] = (uint64_t)l[u].z | ((uint64_t)l[u].w << 32);
-      }
-    }
-#pragma unroll
-    for (int u = 0; u < U; u++) {
-      const int64_t L = base + u * 4 + sub;
-      if (L >= total) continue;
-      const int64_t po = L * 120 + g * 16;                 // payload offset of this lane
-      const int64_t lb = g == 7 ? 8 : 16;                  // payload bytes of this lane
-      int64_t nb = bytes - po;
-      nb = nb < 0 ? 0 : (nb > lb ? lb : nb);
-      const int64_t nb0 = nb > 8 ? 8 : nb, nb1 = nb - nb0;
-      uint64_t v0 = 0, v1 = 0;
-      if (nb > 0) {
-        uint64_t a0 = 0, a1 = 0, b0 = 0, b1 = 0;
-        if constexpr (RECV) {
-          a0 = x0[u];
-          a1 = x1[u];
-        }
-        if constexpr (REDDST) {
-          a0 = loadUnitPlain(dst + po, nb0);
-          if (nb1) a1 = loadUnitPlain(dst + po + 8, nb1);
-        }
-        if constexpr (SRC) {
-          b0 = loadUnitPlain(src + po, nb0);
-          if (nb1) b1 = loadUnitPlain(src + po + 8, nb1);
-        }
-        if constexpr ((RECV && SRC) || REDDST) {
-          v0 = unitOp<DT, OP>(a0, b0);
-          v1 = nb1 ? unitOp<DT, OP>(a1, b1) : 0;
-        } else if constexpr (RECV) {
-          v0 = a0;
-          v1 = a1;
-        } else {
-          v0 = b0;
-          v1 = b1;
-        }
-        if constexpr (DST) {
-          storeUnitPlain(dst + po, v0, nb0);
-          if (nb1) storeUnitPlain(dst + po + 8, v1, nb1);
-        }
-      }
-      if constexpr (SEND) {
-        if (g == 7) v1 = sflag;
-        stvol(sslot + L * 128 + g * 16, make_uint4((uint32_t)v0, (uint32_t)(v0 >> 32), (uint32_t)v1, (uint32_t)(v1 >> 32)));
-      }
-    }
+    bool ok;
+    if (aligned && (base + 4 * U) * 120 <= bytes)
+      ok = ll128Batch<DT, OP, RECV, SEND, SRC, DST, true>(base, bytes, lines, total, rslot, src, dst, sslot, rflag, sflag,
+                                                          g, sub, c);
+    else
+      ok = ll128Batch<DT, OP, RECV, SEND, SRC, DST, false>(base, bytes, lines, total, rslot, src, dst, sslot, rflag,
+                                                           sflag, g, sub, c);
+    if (!ok) return false;
   }
-  return ok;
+  return true;
 }
 
 // ------------------------------------------------------------------ per-protocol piece loops

@@ -36,6 +36,14 @@ if SET == "mid":
         ("ring_ch1_i8_Simple", P.ring_allreduce(R, instances=8), 64 << 20),
         ("oneshot_Simple", P.oneshot_allreduce(R, protocol="Simple"), 4 << 20),
     ]
+if SET == "ll128":
+    cands = [
+        ("ring_ch8_LL128", P.ring_allreduce(R, channels=8, protocol="LL128"), 64 << 20),
+        ("ring_ch1_i16_LL128", P.ring_allreduce(R, instances=16, protocol="LL128"), 256 << 20),
+        ("ring_ch1_i32_LL128", P.ring_allreduce(R, instances=32, protocol="LL128"), 256 << 20),
+        ("ring_ch1_i8_Simple", P.ring_allreduce(R, instances=8), 256 << 20),
+        ("ring_ch1_i32_Simple", P.ring_allreduce(R, instances=32), 256 << 20),
+    ]
 sizes = [1 << k for k in range(10, 31, 2)]
 rows = {}
 for name, algo, maxb in cands:
