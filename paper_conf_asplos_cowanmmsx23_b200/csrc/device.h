@@ -10,6 +10,7 @@ namespace msccl {
 
 #define MSCCL_MAX_LOCAL 16  // ranks that one kernel launch may cover (virtual ranks)
 #define MSCCL_FLAG_WORDS 16 // u64 flag words per connection counter: one per warp (<= 512 threads)
+#define MSCCL_CTA_MAP 512   // largest grid whose CTA -> (rank, thread block) order the host sets
 
 enum { DI_SEND_DIRECT = 1, DI_RECV_DIRECT = 2, DI_CHAIN_HEAD = 4 };
 
@@ -80,6 +81,12 @@ struct KernelArgs {
   int32_t pad3;
   uint64_t timeoutNs;
   uint64_t* trace;            // MSCCL_TRACE builds: per-CTA phase times (ns), else null
+  // CTA c runs thread block ctaMap[c] & 4095 of local rank ctaMap[c] >> 12 (work-balanced
+  // placement: the thread blocks that move the most bytes get the lowest block indices, which
+  // the hardware spreads over distinct SMs first); ctaMapN == 0: rank by prefix sums
+  int32_t ctaMapN;
+  uint16_t ctaMap[MSCCL_CTA_MAP];
 };
+static_assert(sizeof(KernelArgs) <= 4096, "kernel parameter space");
 
 }  // namespace msccl

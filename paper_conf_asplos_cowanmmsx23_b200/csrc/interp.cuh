@@ -1077,11 +1077,17 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
   __shared__ TmaState sTma;
   extern __shared__ __align__(128) uint8_t dynSmem[];
 #endif
-  int ls = 0;
-  for (int r = 1; r < a.nLocal; r++)
-    if ((int)blockIdx.x >= a.rank[r].ctaStart) ls = r;
+  int ls = 0, tbi;
+  if (a.ctaMapN) {  // work-balanced placement chosen by the host
+    const uint32_t e = a.ctaMap[blockIdx.x];
+    ls = (int)(e >> 12);
+    tbi = (int)(e & 4095u);
+  } else {
+    for (int r = 1; r < a.nLocal; r++)
+      if ((int)blockIdx.x >= a.rank[r].ctaStart) ls = r;
+    tbi = (int)blockIdx.x - a.rank[ls].ctaStart;
+  }
   const RankArgs& ra = a.rank[ls];
-  const int tbi = (int)blockIdx.x - ra.ctaStart;
   if (tbi >= ra.nTB) return;
   const DevTB& tb = ra.tbs[tbi];
   Ctx c{&a, &ra, (int)threadIdx.x, (int)blockDim.x, nullptr, 0};

@@ -27,7 +27,7 @@ namespace {
 
 struct Params {
   int64_t slots = 4, slotBytes = 262144, maxChannels = 32, threads = 512, timeoutS = 20, tma = 0, direct = 1,
-          warp = 0, l2PersistMiB = 0, prefetch = 0, directTile = 1;
+          warp = 0, l2PersistMiB = 0, prefetch = 0, directTile = 1, balance = 0;
 };
 
 std::mutex gMu;
@@ -48,6 +48,7 @@ int64_t* paramRef(Params& p, const std::string& k) {
   if (k == "MSCCL_L2_PERSIST_MIB") return &p.l2PersistMiB;
   if (k == "MSCCL_PREFETCH") return &p.prefetch;
   if (k == "MSCCL_DIRECT_TILE") return &p.directTile;
+  if (k == "MSCCL_BALANCE") return &p.balance;
   return nullptr;
 }
 
@@ -57,7 +58,8 @@ Params currentParams() {
     gEnvRead = true;
     for (const char* k : {"MSCCL_SLOTS", "MSCCL_SLOT_BYTES", "MSCCL_MAX_CHANNELS", "MSCCL_THREADS", "MSCCL_TIMEOUT_S",
                           "MSCCL_TMA", "MSCCL_DIRECT", "MSCCL_WARP_FLAGS",
-                          "MSCCL_L2_PERSIST_MIB", "MSCCL_PREFETCH", "MSCCL_DIRECT_TILE"}) {
+                          "MSCCL_L2_PERSIST_MIB", "MSCCL_PREFETCH", "MSCCL_DIRECT_TILE",
+                          "MSCCL_BALANCE"}) {
       const char* v = getenv(k);
       if (v && *v) *paramRef(gParams, k) = atoll(v);
     }
@@ -127,6 +129,8 @@ struct mscclProgram {
   int maxCnt = 1;
   bool hasReduce = false;
   bool allDirect = true;  // every message of this rank's program is a direct placement (R15)
+  std::vector<int64_t> tbWork;        // chunk-sized operand touches per thread block (FIFO protocol)
+  std::vector<int64_t> tbWorkDirect;  // ... with direct placement (R15)
 };
 
 namespace {
@@ -358,6 +362,21 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
       if (cl->comm->sysScope) ka.sysScope = 1;
     }
     if (cta == 0) continue;
+    // work-balanced placement: thread blocks ordered by the bytes they move (heaviest first,
+    // ties by rank then id, so the order is deterministic); block indices are handed to SMs
+    // in increasing order, so the heavy blocks land on distinct SMs before any SM gets two
+    if (c0->prm.balance && cta <= MSCCL_CTA_MAP && (int)v.size() <= 16) {
+      std::vector<std::tuple<int64_t, int, int>> order;
+      for (int i = 0; i < (int)v.size(); i++) {
+        const mscclProgram* p = v[i]->prog;
+        const auto& wk = direct ? p->tbWorkDirect : p->tbWork;
+        for (int t = 0; t < p->nTB; t++) order.emplace_back(-wk[t], i, t);
+      }
+      std::stable_sort(order.begin(), order.end());
+      for (size_t k = 0; k < order.size(); k++)
+        ka.ctaMap[k] = (uint16_t)((std::get<1>(order[k]) << 12) | std::get<2>(order[k]));
+      ka.ctaMapN = (int32_t)order.size();
+    }
     const void* fn = p0->hasReduce ? interpreterKernel(v[0]->dtype, v[0]->op, ka.proto)
                                    : copyKernel(elemBytes(v[0]->dtype), ka.proto);
     ka.useTma = useTma ? 1 : 0;
@@ -689,6 +708,8 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
   p->nTB = (int)g.tbs.size();
   const DirectInfo dinfo = directPlacement(p->algo, c->rank);
   std::vector<DevTB> tbs(p->nTB);
+  p->tbWork.assign(p->nTB, 0);
+  p->tbWorkDirect.assign(p->nTB, 0);
   std::vector<DevInstr> ins;
   std::vector<uint32_t> deps;
   for (int t = 0; t < p->nTB; t++) {
@@ -727,6 +748,13 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
       di.depStart = (uint32_t)deps.size();
       for (auto& dp : in.deps) deps.push_back(((uint32_t)dp.first << 16) | (uint32_t)dp.second);
       if (dinfo.recvDirect[t][si]) di.flags |= DI_RECV_DIRECT;
+      {  // operand touches of this instruction (mscclProgramTouches costs)
+        static const int cost[OP_COUNT] = {0, 2, 2, 2, 3, 3, 3, 4, 3};
+        int cd = cost[in.op];
+        if (dinfo.recvDirect[t][si]) cd = in.op == OP_RCS ? 2 : 0;
+        p->tbWork[t] += (int64_t)cost[in.op] * in.cnt;
+        p->tbWorkDirect[t] += (int64_t)cd * in.cnt;
+      }
       const bool sends = in.op == OP_SEND || in.op == OP_RRS || in.op == OP_RRCS || in.op == OP_RCS;
       if (sends && !dinfo.sendDirect[t][si]) p->allDirect = false;
       if (dinfo.sendDirect[t][si]) {
