@@ -12,7 +12,9 @@ namespace msccl {
 #define MSCCL_FLAG_WORDS 16 // u64 flag words per connection counter: one per warp (<= 512 threads)
 #define MSCCL_CTA_MAP 512   // largest grid whose CTA -> (rank, thread block) order the host sets
 
-enum { DI_SEND_DIRECT = 1, DI_RECV_DIRECT = 2, DI_CHAIN_HEAD = 4 };
+// DI_SEND_TERMINAL: a direct send whose receiving instruction is a plain recv (the data is
+// not forwarded by the receiver's thread block: a cache hint only)
+enum { DI_SEND_DIRECT = 1, DI_RECV_DIRECT = 2, DI_CHAIN_HEAD = 4, DI_SEND_TERMINAL = 8 };
 
 struct DevInstr {     // 32 bytes
   uint8_t op, srcBuf, dstBuf, nDeps;
@@ -51,7 +53,7 @@ struct DevTB {
 struct RankArgs {
   const DevTB* tbs;
   const DevInstr* instrs;
-  const uint32_t* deps;       // (tb << 16) | step
+  const uint64_t* deps;       // (tb << 48) | (step << 32) | nSteps of tb (DevTB::depWord)
   uint64_t* sem;              // per-TB semaphores (monotone, reading R4)
   uint64_t* gen;              // per-TB launch generation
   char* buf[3];               // in, out, scratch base pointers for this call
@@ -78,7 +80,8 @@ struct KernelArgs {
   int32_t direct;             // honour DI_*_DIRECT flags (all ranks in this launch, rank == slot)
   int32_t warpFlags;          // Simple protocol: per-warp head/ack flags, no block barrier per message (R18)
   int32_t prefetch;           // Simple protocol: bulk L2 prefetch of the local operand before a receive wait
-  int32_t pad3;
+  int32_t directHints;        // bit 0: terminal direct sends store L2 evict_first; bit 1: a direct
+                              // forward demotes the lines it read to evict_normal (cache hints)
   uint64_t timeoutNs;
   uint64_t* trace;            // MSCCL_TRACE builds: per-CTA phase times (ns), else null
   // CTA c runs thread block ctaMap[c] & 4095 of local rank ctaMap[c] >> 12 (work-balanced

@@ -21,6 +21,7 @@
 #pragma once
 #include <cuda_bf16.h>
 #include <cuda_fp16.h>
+#include <stddef.h>
 #include <stdint.h>
 #include <type_traits>
 
@@ -256,6 +257,12 @@ struct Ctx {
   int tid, nt;
   TmaState* tma;  // shared-memory pipeline state (Simple protocol with TMA), or null
   uint64_t sent0; // messages posted on the send connection before this launch
+  // credit cache of the send connection (LL / LL128): every ack word is known to be >= ackKnown
+  // (the receiver has consumed that many messages), so a send whose slot was freed by then
+  // needs no flag read; uniform over the block. sAck: the 16 words seen by the waiting threads.
+  mutable uint64_t ackKnown;
+  uint64_t* sAck;
+  uint64_t* tl;   // MSCCL_TIMELINE builds: this CTA's timeline words, else null
 };
 
 static __device__ __noinline__ void raiseAbort(const KernelArgs& a) {
@@ -265,12 +272,13 @@ static __device__ __noinline__ void raiseAbort(const KernelArgs& a) {
   }
 }
 
-// Spin until *p >= target (acquire). Returns false on watchdog timeout / abort.
-__device__ __forceinline__ bool waitGE(const uint64_t* p, uint64_t target, bool sys, const Ctx& c) {
-  if ((sys ? ldAcquireSys(p) : ldAcquireGpu(p)) >= target) return true;
+// Spin until *p >= target (acquire); `seen` = the value that satisfied the wait. Returns
+// false on watchdog timeout / abort.
+__device__ __forceinline__ bool waitGE(const uint64_t* p, uint64_t target, bool sys, const Ctx& c, uint64_t& seen) {
+  if ((seen = (sys ? ldAcquireSys(p) : ldAcquireGpu(p))) >= target) return true;
   uint64_t t0 = globaltimer();
   for (uint32_t it = 1;; it++) {
-    if ((sys ? ldAcquireSys(p) : ldAcquireGpu(p)) >= target) return true;
+    if ((seen = (sys ? ldAcquireSys(p) : ldAcquireGpu(p))) >= target) return true;
     if ((it & 1023u) == 0) {
       if (*(volatile uint32_t*)c.ra->abortFlag) return false;
       if (globaltimer() - t0 > c.a->timeoutNs) {
@@ -279,6 +287,29 @@ __device__ __forceinline__ bool waitGE(const uint64_t* p, uint64_t target, bool 
       }
     }
   }
+}
+
+__device__ __forceinline__ bool waitGE(const uint64_t* p, uint64_t target, bool sys, const Ctx& c) {
+  uint64_t seen;
+  return waitGE(p, target, sys, c, seen);
+}
+
+// Cross-thread-block dependency (Fig. 5 lines 15-16): wait until thread block dtb of this
+// rank has finished step dstep of tile t in this launch (monotone semaphore, reading R4).
+__device__ __forceinline__ bool waitDep(const RankArgs& ra, uint64_t dep, uint64_t gen, int t, const Ctx& c) {
+  const int dtb = (int)(dep >> 48), dstep = (int)((dep >> 32) & 0xffff);
+  const uint64_t dn = (uint32_t)dep;  // steps of thread block dtb
+#if MSCCL_TIMELINE
+  if (c.tl && c.tid == 0) {
+    const uint64_t target = (gen << 40) | ((uint64_t)t * dn + (uint64_t)dstep + 1);
+    const uint64_t v0 = ldAcquireGpu(&ra.sem[dtb]);
+    c.tl[27] = globaltimer();
+    c.tl[28] = v0 >= target ? 1 : 0;
+    c.tl[29] = v0;
+    c.tl[30] = target;
+  }
+#endif
+  return waitGE(&ra.sem[dtb], (gen << 40) | ((uint64_t)t * dn + (uint64_t)dstep + 1), false, c);
 }
 
 // ------------------------------------------------------------------ chunk geometry (reading R1)
@@ -300,6 +331,9 @@ __device__ __forceinline__ void chunkSpan(const KernelArgs& a, int buf, int64_t 
 #ifndef MSCCL_TRACE
 #define MSCCL_TRACE 0
 #endif
+#ifndef MSCCL_TIMELINE
+#define MSCCL_TIMELINE 0
+#endif
 #ifndef MSCCL_FENCE_MODE
 #define MSCCL_FENCE_MODE 0
 #endif
@@ -312,12 +346,17 @@ __device__ __forceinline__ void chunkSpan(const KernelArgs& a, int buf, int64_t 
 
 // Main vector loop: VB-byte vectors, U independent vectors in flight per thread.
 // Returns the number of VB-byte vectors processed.
+// store hint of one piece: a direct send whose receiver does not forward the data stores it
+// L2 evict_first (reading R15, DI_SEND_TERMINAL)
+enum { HINT_SEND_FIRST = 1 };
+
 template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST, int VB>
 __device__ __forceinline__ int64_t vecLoop(int64_t nvec, const char* rslot, const char* src, char* dst, char* sslot,
-                                           int ti, int nt) {
+                                           int ti, int nt, int hint) {
   typedef typename VecT<VB>::T Vec;
   constexpr int U = ((int)RECV + (int)SRC + (int)REDDST) >= 2 ? MSCCL_UNROLL : MSCCL_UNROLL1;
-  const uint64_t pFirst = policyEvictFirst(), pLast = policyEvictLast();
+  const uint64_t pFirst = policyEvictFirst(), pLast0 = policyEvictLast();
+  const uint64_t pLast = (hint & HINT_SEND_FIRST) ? pFirst : pLast0;
   const bool canDiscard = RECV && ((((uintptr_t)rslot) & 127) == 0);
   const int lane = ti & 31, warp = ti >> 5, nw = nt >> 5;
   // Full blocks of U x 32 vectors, one block per warp-iteration (warp-uniform trip count,
@@ -370,22 +409,22 @@ __device__ __forceinline__ int64_t vecLoop(int64_t nvec, const char* rslot, cons
 // block (nt = blockDim) or one warp (nt = 32, warp flags).
 template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
 __device__ __forceinline__ void pieceSimple(int64_t m, const char* rslot, const char* src, char* dst, char* sslot,
-                                            int ti, int nt) {
+                                            int ti, int nt, int hint = 0) {
   typedef typename DType<DT>::T T;
   const int64_t bytes = m * (int64_t)sizeof(T);
   uintptr_t al = (uintptr_t)rslot | (uintptr_t)src | (uintptr_t)dst | (uintptr_t)sslot;
   int64_t done = 0;  // bytes handled by the vector paths
   if ((al & 31) == 0) {
-    done = 32 * vecLoop<DT, OP, RECV, SEND, SRC, DST, REDDST, 32>(bytes / 32, rslot, src, dst, sslot, ti, nt);
+    done = 32 * vecLoop<DT, OP, RECV, SEND, SRC, DST, REDDST, 32>(bytes / 32, rslot, src, dst, sslot, ti, nt, hint);
   } else if ((al & 15) == 0) {
-    done = 16 * vecLoop<DT, OP, RECV, SEND, SRC, DST, REDDST, 16>(bytes / 16, rslot, src, dst, sslot, ti, nt);
+    done = 16 * vecLoop<DT, OP, RECV, SEND, SRC, DST, REDDST, 16>(bytes / 16, rslot, src, dst, sslot, ti, nt, hint);
   }
   if ((al & 15) == 0 && bytes - done >= 16) {  // 16-byte remainder after the 32-byte path
     const int64_t off = done;
     const int64_t nv = (bytes - done) / 16;
     done += 16 * vecLoop<DT, OP, RECV, SEND, SRC, DST, REDDST, 16>(
                      nv, RECV ? rslot + off : nullptr, SRC ? src + off : nullptr, (DST || REDDST) ? dst + off : nullptr,
-                     SEND ? sslot + off : nullptr, ti, nt);
+                     SEND ? sslot + off : nullptr, ti, nt, hint);
   }
   // scalar tail (ragged chunk end or unaligned buffers)
   for (int64_t e = done / (int64_t)sizeof(T) + ti; e < m; e += nt) {
@@ -464,6 +503,11 @@ __device__ __forceinline__ bool pieceLL(int64_t m, int64_t sendUnits, const char
     const int64_t off = u * 8;
     const int64_t nb = has ? (bytes - off < 8 ? bytes - off : 8) : 0;
     uint64_t x = 0, y = 0, v = 0;
+    // the local operand first: its load overlaps the wait for the incoming line
+    if (has) {
+      if constexpr (REDDST) x = loadUnit(dst + off, nb);
+      if constexpr (SRC) y = loadUnit(src + off, nb);
+    }
     if constexpr (RECV) {
       if (has) {
         const char* line = rslot + u * 16;
@@ -484,8 +528,6 @@ __device__ __forceinline__ bool pieceLL(int64_t m, int64_t sendUnits, const char
       }
     }
     if (has) {
-      if constexpr (REDDST) x = loadUnit(dst + off, nb);
-      if constexpr (SRC) y = loadUnit(src + off, nb);
       if constexpr ((RECV && SRC) || REDDST) v = unitOp<DT, OP>(x, y);
       else if constexpr (RECV) v = x;
       else v = y;
@@ -694,11 +736,13 @@ __device__ __noinline__ void movePiecesSimple(const Ctx& c, const DevTB& tb, con
       if (rl - a0 < m) m = rl - a0;
     }
     if (m <= 0) continue;
+    const int hint = (sdirect && (in.flags & DI_SEND_TERMINAL)) ? (a.directHints & HINT_SEND_FIRST) : 0;
     if (rdirect) {  // the data is already in dst (the sender wrote it there)
-      if (SEND) pieceSimple<DT, OP, false, true, true, false, false>(m, nullptr, dst, nullptr, so, c.tid, c.nt);
+      if (SEND) pieceSimple<DT, OP, false, true, true, false, false>(m, nullptr, dst, nullptr, so, c.tid, c.nt, hint);
       continue;
     }
-    pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, RECV ? rslot + j * a.T * w : nullptr, src, dst, so, c.tid, c.nt);
+    pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, RECV ? rslot + j * a.T * w : nullptr, src, dst, so, c.tid, c.nt,
+                                                      hint);
   }
 }
 
@@ -919,13 +963,35 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
   // a free slot: at most `slots` messages posted and not yet consumed (§6.1)
   // (a direct message uses no slot: no credit needed, reading R15)
   // (every ack word: a warp-flag launch before this one may have acknowledged word by word)
-  if (SEND && c.tid >= 32 && c.tid < 32 + MSCCL_FLAG_WORDS && sent + 1 > (uint64_t)a.slots &&
-      !(a.direct && (in.flags & DI_SEND_DIRECT)))
-    ok = ok && waitGE(tb.sendAck + (c.tid - 32), sent + 1 - (uint64_t)a.slots, sys, c);
-  if (!ok) *sAbort = 1;
-  if (RECV || SEND) {
-    __syncthreads();
-    if (*sAbort) return false;
+  // LL / LL128: credits already seen (c.ackKnown) are not re-read, so a step that has its slot
+  // (no head to wait for: the flags travel in the lines) starts moving data without a flag
+  // round trip or barrier. Simple keeps the per-message check (it needs the barrier anyway).
+  if constexpr (!ll) {
+    if (SEND && c.tid >= 32 && c.tid < 32 + MSCCL_FLAG_WORDS && sent + 1 > (uint64_t)a.slots &&
+        !(a.direct && (in.flags & DI_SEND_DIRECT)))
+      ok = ok && waitGE(tb.sendAck + (c.tid - 32), sent + 1 - (uint64_t)a.slots, sys, c);
+    if (!ok) *sAbort = 1;
+    if (RECV || SEND) {
+      __syncthreads();
+      if (*sAbort) return false;
+    }
+  } else {
+    const uint64_t need = sent + 1 > (uint64_t)a.slots ? sent + 1 - (uint64_t)a.slots : 0;
+    const bool creditWait = SEND && need > c.ackKnown;
+    if (creditWait && c.tid >= 32 && c.tid < 32 + MSCCL_FLAG_WORDS) {
+      uint64_t seen = 0;
+      ok = ok && waitGE(tb.sendAck + (c.tid - 32), need, sys, c, seen);
+      c.sAck[c.tid - 32] = seen;
+    }
+    if (!ok) *sAbort = 1;
+    if (creditWait) {
+      __syncthreads();
+      if (*sAbort) return false;
+      uint64_t mn = c.sAck[0];
+#pragma unroll
+      for (int k = 1; k < MSCCL_FLAG_WORDS; k++) mn = c.sAck[k] < mn ? c.sAck[k] : mn;
+      c.ackKnown = mn;
+    }
   }
 #if MSCCL_TRACE
   if (c.tid == 0) tr2 = globaltimer();
@@ -1007,8 +1073,19 @@ __device__ __forceinline__ bool dispatch(const Ctx& c, const DevTB& tb, const De
 // barrier per instruction. Pieces whose members disagree on length fall back to the
 // sequential instructions.
 #define MSCCL_MAX_CHAIN 16
-template <int DT, int OP>
-__device__ __noinline__ void chainExec(const Ctx& c, const DevInstr* mem, int L, int t) {
+// Operand loads in flight per vector in a fused chain: 8 in the LL kernels (latency),
+// 2 in the Simple and LL128 kernels (a larger batch there makes ptxas spill in their data loops,
+// measured -12 % ring bandwidth).
+// Operand table of one chain piece, built in shared memory by threads 0..L-1 in parallel
+// (thread k resolves member k's source chunk) instead of by every thread in turn.
+struct ChainSmem {
+  const char* src[MSCCL_MAX_CHAIN];
+  int64_t m[MSCCL_MAX_CHAIN];
+  char* dst;
+  int64_t dl;
+};
+template <int DT, int OP, int BATCH>
+__device__ __noinline__ void chainExec(const Ctx& c, const DevInstr* mem, int L, int t, ChainSmem& cs, uint64_t* tl) {
   typedef typename DType<DT>::T T;
   const KernelArgs& a = *c.a;
   const RankArgs& ra = *c.ra;
@@ -1016,70 +1093,115 @@ __device__ __noinline__ void chainExec(const Ctx& c, const DevInstr* mem, int L,
   const int64_t a0 = (int64_t)t * a.T;
   const bool headCopy = mem[0].op == K_COPY;
   for (int j = 0; j < mem[0].cnt; j++) {
-    int64_t ds, dl;
-    chunkSpan(a, mem[0].dstBuf, (int64_t)mem[0].dstOff + j, ds, dl);
-    const char* srcs[MSCCL_MAX_CHAIN];
-    int64_t m = -1;
-    bool same = true;
-    uintptr_t al = 0;
-    for (int k = 0; k < L; k++) {
-      int64_t ss, sl;
+    if (c.tid < L) {
+      const int k = c.tid;
+      int64_t ds, dl, ss, sl;
+      chunkSpan(a, mem[0].dstBuf, (int64_t)mem[0].dstOff + j, ds, dl);
       chunkSpan(a, mem[k].srcBuf, (int64_t)mem[k].srcOff + j, ss, sl);
-      int64_t Lk = sl < dl ? sl : dl;
-      int64_t mk = (a0 + a.T < Lk ? a0 + a.T : Lk) - a0;
-      if (m < 0) m = mk;
-      else if (mk != m) same = false;
-      srcs[k] = ra.buf[mem[k].srcBuf] + (ss + a0) * w;
-      al |= (uintptr_t)srcs[k];
+      const int64_t Lk = sl < dl ? sl : dl;
+      cs.m[k] = (a0 + a.T < Lk ? a0 + a.T : Lk) - a0;
+      cs.src[k] = ra.buf[mem[k].srcBuf] + (ss + a0) * w;
+      if (k == 0) {
+        cs.dst = ra.buf[mem[0].dstBuf] + (ds + a0) * w;
+        cs.dl = dl;
+      }
     }
-    char* dst = ra.buf[mem[0].dstBuf] + (ds + a0) * w;
-    al |= (uintptr_t)dst;
+    __syncthreads();
+    const int64_t m = cs.m[0];
+    bool same = true;
+    uintptr_t al = (uintptr_t)cs.dst;
+    for (int k = 0; k < L; k++) {
+      same = same && cs.m[k] == m;
+      al |= (uintptr_t)cs.src[k];
+    }
+    char* dst = cs.dst;
     if (!same) {  // sequential fallback (a barrier between members: element->thread maps differ)
       for (int k = 0; k < L; k++) {
-        int64_t ss, sl;
-        chunkSpan(a, mem[k].srcBuf, (int64_t)mem[k].srcOff + j, ss, sl);
-        int64_t Lk = sl < dl ? sl : dl;
-        int64_t mk = (a0 + a.T < Lk ? a0 + a.T : Lk) - a0;
+        const int64_t mk = cs.m[k];
         if (mk > 0) {
           if (mem[k].op == K_COPY)
-            pieceSimple<DT, OP, false, false, true, true, false>(mk, nullptr, srcs[k], dst, nullptr, c.tid, c.nt);
+            pieceSimple<DT, OP, false, false, true, true, false>(mk, nullptr, cs.src[k], dst, nullptr, c.tid, c.nt);
           else
-            pieceSimple<DT, OP, false, false, true, true, true>(mk, nullptr, srcs[k], dst, nullptr, c.tid, c.nt);
+            pieceSimple<DT, OP, false, false, true, true, true>(mk, nullptr, cs.src[k], dst, nullptr, c.tid, c.nt);
         }
         __syncthreads();
       }
       continue;
     }
-    if (m <= 0) continue;
-    const int64_t bytes = m * w;
-    int64_t nvec = (al & 15) ? 0 : bytes / 16;
-    for (int64_t i = c.tid; i < nvec; i += c.nt) {
-      uint4 acc = headCopy ? ldcg(srcs[0] + i * 16) : ldcg(dst + i * 16);
-      for (int k = headCopy ? 1 : 0; k < L; k++) acc = vop<DT, OP>(acc, ldcg(srcs[k] + i * 16));
-      stg(dst + i * 16, acc);
+    if (m > 0) {
+      const int64_t bytes = m * w;
+      const int64_t nvec = (al & 15) ? 0 : bytes / 16;
+#if MSCCL_TIMELINE
+      if (tl && c.tid == 0) tl[17] = globaltimer();
+#endif
+      // operands of a vector are loaded in batches before they are folded (in program order),
+      // so a chain costs about one memory round trip per batch, not one per member
+      const char* first = headCopy ? cs.src[0] : dst;
+      const int k0 = headCopy ? 1 : 0;
+      for (int64_t i = c.tid; i < nvec; i += c.nt) {
+        uint4 acc = ldcg(first + i * 16);
+        for (int kb = k0; kb < L; kb += BATCH) {
+          uint4 v[BATCH];
+#pragma unroll
+          for (int u = 0; u < BATCH; u++)
+            if (kb + u < L) v[u] = ldcg(cs.src[kb + u] + i * 16);
+#pragma unroll
+          for (int u = 0; u < BATCH; u++)
+            if (kb + u < L) acc = vop<DT, OP>(acc, v[u]);
+        }
+        stg(dst + i * 16, acc);
+      }
+      for (int64_t e = nvec * 16 / w + c.tid; e < m; e += c.nt) {
+        T acc = headCopy ? *(const T*)(cs.src[0] + e * w) : *(const T*)(dst + e * w);
+        for (int k = headCopy ? 1 : 0; k < L; k++) acc = DType<DT>::op(OP, acc, *(const T*)(cs.src[k] + e * w));
+        *(T*)(dst + e * w) = acc;
+      }
     }
-    for (int64_t e = nvec * 16 / w + c.tid; e < m; e += c.nt) {
-      T acc = headCopy ? *(const T*)(srcs[0] + e * w) : *(const T*)(dst + e * w);
-      for (int k = headCopy ? 1 : 0; k < L; k++) acc = DType<DT>::op(OP, acc, *(const T*)(srcs[k] + e * w));
-      *(T*)(dst + e * w) = acc;
-    }
+    __syncthreads();  // the operand table is rewritten for the next piece
   }
 }
 
 #ifndef MSCCL_MAX_THREADS
 #define MSCCL_MAX_THREADS 512
 #endif
+#ifndef MSCCL_SMEM_INSTR
+#define MSCCL_SMEM_INSTR 64  // instructions per thread block staged in shared memory (LL / LL128)
+#endif
 
 template <int DT, int OP, int PROTO>
-__global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const __grid_constant__ KernelArgs a) {
+__global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const __grid_constant__ KernelArgs aParam) {
   __shared__ int sAbort;
+  // The launch arguments (all ranks' base pointers and tables, geometry) are copied from the
+  // parameter bank into shared memory by all threads at once: every later access is a shared
+  // load instead of a (serialised, on first touch) constant-cache miss. The CTA map stays in
+  // the parameter bank (one entry per CTA).
+  // (latency protocols only: kLat. The Simple kernels keep the HEAD-of-round layout -- these
+  // prologue changes measured -6 % on the Simple ring and buy nothing at bandwidth sizes.)
+  constexpr bool kLat = PROTO != 0;
+  constexpr int kArgWords = kLat ? (int)(offsetof(KernelArgs, ctaMap) / 4) : 1;
+  __shared__ __align__(16) uint32_t sArgs[kArgWords];
+  if constexpr (kLat) {
+    for (int i = threadIdx.x; i < kArgWords; i += blockDim.x) sArgs[i] = reinterpret_cast<const uint32_t*>(&aParam)[i];
+    __syncthreads();
+  }
+  const KernelArgs& a = kLat ? *reinterpret_cast<const KernelArgs*>(sArgs) : aParam;
 #if MSCCL_ENABLE_TMA
   __shared__ TmaState sTma;
   extern __shared__ __align__(128) uint8_t dynSmem[];
 #endif
+#if MSCCL_TIMELINE
+  // latency timeline (debug builds): [0] entry, [1] prologue done, [2 + s] end of step s
+  // (s < 10), [13]/[14] a fused chain's dependency waits / data pass done, [15] exit, [16]
+  // thread 0's own dependency wait done, [17] chain operand setup done, [18 + s] end of step
+  // s of the second tile; %globaltimer, thread 0, last launch wins
+  uint64_t* tl = a.trace ? a.trace + (size_t)blockIdx.x * 32 : nullptr;
+  if (tl && threadIdx.x == 0) tl[0] = globaltimer();
+#else
+  uint64_t* const tl = nullptr;
+#endif
   int ls = 0, tbi;
   if (a.ctaMapN) {  // work-balanced placement chosen by the host
-    const uint32_t e = a.ctaMap[blockIdx.x];
+    const uint32_t e = aParam.ctaMap[blockIdx.x];
     ls = (int)(e >> 12);
     tbi = (int)(e & 4095u);
   } else {
@@ -1089,8 +1211,22 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
   }
   const RankArgs& ra = a.rank[ls];
   if (tbi >= ra.nTB) return;
-  const DevTB& tb = ra.tbs[tbi];
-  Ctx c{&a, &ra, (int)threadIdx.x, (int)blockDim.x, nullptr, 0};
+  // Prologue: the thread block's descriptor and instruction list are staged in
+  // shared memory by parallel 16-byte loads, so the instruction loop never waits on a global
+  // round trip to decode a step.
+  __shared__ __align__(16) DevTB sTB;
+  __shared__ __align__(16) DevInstr sIns[kLat ? MSCCL_SMEM_INSTR : 1];
+  if (kLat && threadIdx.x < sizeof(DevTB) / 16)
+    reinterpret_cast<uint4*>(&sTB)[threadIdx.x] = reinterpret_cast<const uint4*>(&ra.tbs[tbi])[threadIdx.x];
+  if (kLat) __syncthreads();
+  const DevTB& tb = kLat ? sTB : ra.tbs[tbi];
+  const DevInstr* ins = ra.instrs + tb.instrStart;
+  if (kLat && tb.nSteps <= MSCCL_SMEM_INSTR) {
+    for (int i = threadIdx.x; i < tb.nSteps * (int)(sizeof(DevInstr) / 16); i += blockDim.x)
+      reinterpret_cast<uint4*>(sIns)[i] = reinterpret_cast<const uint4*>(ins)[i];
+    ins = sIns;
+  }
+  Ctx c{&a, &ra, (int)threadIdx.x, (int)blockDim.x, nullptr, 0, 0, nullptr, tl};
 #if MSCCL_ENABLE_TMA
   if (a.useTma && PROTO == 0) {
     c.tma = &sTma;
@@ -1110,6 +1246,10 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
   }
 #endif
   if (threadIdx.x == 0) sAbort = 0;
+  __shared__ uint64_t sAck[MSCCL_FLAG_WORDS];
+  __shared__ ChainSmem sChain;
+  c.sAck = sAck;
+  c.ackKnown = 0;
   uint64_t sent = tb.sendFifo ? *(volatile uint64_t*)tb.sendCnt : 0;
   c.sent0 = sent;
   uint64_t recvd = tb.recvFifo ? *(volatile uint64_t*)tb.recvCnt : 0;
@@ -1120,43 +1260,65 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
   const bool warpMode = PROTO == 0 && a.warpFlags;
   bool dead = false;
   __syncthreads();
+#if MSCCL_TIMELINE
+  if (tl && threadIdx.x == 0) tl[1] = globaltimer();
+#endif
   for (int t = 0; t < a.I; t++) {
     for (int s = 0; s < tb.nSteps; s++) {
-      const DevInstr in = ra.instrs[tb.instrStart + s];
+      const DevInstr in = ins[s];
       if constexpr (OP != R_COPY) {
         if (in.flags & DI_CHAIN_HEAD) {  // reading R16: fused local reduce chain
           const int L = in.chainLen;
           bool ok = true;
-          for (int k = 0; k < L && ok; k++) {  // all members' dependencies first
-            const DevInstr& mk = ra.instrs[tb.instrStart + s + k];
-            for (int d = c.tid; d < mk.nDeps && ok; d += c.nt) {
-              uint32_t dep = ra.deps[mk.depStart + d];
-              int dtb = (int)(dep >> 16), dstep = (int)(dep & 0xffff);
-              uint64_t target = (gen << 40) | ((uint64_t)t * (uint64_t)ra.tbs[dtb].nSteps + (uint64_t)dstep + 1);
-              ok = waitGE(&ra.sem[dtb], target, false, c);
+          // all members' dependencies first: flattened dependency f goes to thread f mod nt; a
+          // thread first collects its dependency words, then waits on all of them, so the waits
+          // of different members overlap (waiting inside the member loop serialises them: one
+          // member per loop trip)
+          {
+            constexpr int KD = 4;
+            uint64_t mine[KD];
+            int nm = 0;
+            for (int k = 0, base = 0; k < L; k++) {
+              const DevInstr& mk = ins[s + k];
+              for (int d = ((c.tid - base) % c.nt + c.nt) % c.nt; d < mk.nDeps; d += c.nt) {
+                const uint64_t dw = ra.deps[mk.depStart + d];
+                if (nm < KD) mine[nm++] = dw;
+                else ok = ok && waitDep(ra, dw, gen, t, c);  // more than KD per thread: in order
+              }
+              base += mk.nDeps;
             }
+#pragma unroll
+            for (int i = 0; i < KD; i++)
+              if (i < nm) ok = ok && waitDep(ra, mine[i], gen, t, c);
           }
+#if MSCCL_TIMELINE
+          if (tl && threadIdx.x == 0) tl[16] = globaltimer();
+#endif
           if (!ok) sAbort = 1;
           __syncthreads();
           if (sAbort) return;
-          chainExec<DT, OP>(c, ra.instrs + tb.instrStart + s, L, t);
+#if MSCCL_TIMELINE
+          if (tl && threadIdx.x == 0) tl[13] = globaltimer();
+#endif
+          chainExec<DT, OP, PROTO == 1 ? 8 : 2>(c, ins + s, L, t, sChain, tl);
           __syncthreads();
+#if MSCCL_TIMELINE
+          if (tl && threadIdx.x == 0) tl[14] = globaltimer();
+#endif
           s += L - 1;
-          if (ra.instrs[tb.instrStart + s].hasDep && c.tid == 0) {
+          if (ins[s].hasDep && c.tid == 0) {
             fenceGpu();
             stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)tb.nSteps + (uint64_t)s + 1));
           }
+#if MSCCL_TIMELINE
+          if (tl && threadIdx.x == 0 && s < 10 && t < 2) tl[(t ? 18 : 2) + s] = globaltimer();
+#endif
           continue;
         }
       }
       if (in.nDeps) {  // Fig. 5 lines 15-16; barrier after the waits (reading R10)
         bool ok = true;
-        for (int d = c.tid; d < in.nDeps && ok; d += c.nt) {
-          uint32_t dep = ra.deps[in.depStart + d];
-          int dtb = (int)(dep >> 16), dstep = (int)(dep & 0xffff);
-          uint64_t target = (gen << 40) | ((uint64_t)t * (uint64_t)ra.tbs[dtb].nSteps + (uint64_t)dstep + 1);
-          ok = waitGE(&ra.sem[dtb], target, false, c);
-        }
+        for (int d = c.tid; d < in.nDeps && ok; d += c.nt) ok = waitDep(ra, ra.deps[in.depStart + d], gen, t, c);
         if (!ok) sAbort = 1;
         __syncthreads();
         if (sAbort) return;
@@ -1184,6 +1346,9 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
           stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)tb.nSteps + (uint64_t)s + 1));
         }
       }
+#if MSCCL_TIMELINE
+      if (tl && threadIdx.x == 0 && s < 10 && t < 2) tl[(t ? 18 : 2) + s] = globaltimer();
+#endif
     }
   }
   if (warpMode) {
@@ -1202,6 +1367,9 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
       }
     }
     *(volatile uint64_t*)&ra.gen[tbi] = gen + 1;
+#if MSCCL_TIMELINE
+    if (tl) tl[15] = globaltimer();
+#endif
   }
 }
 

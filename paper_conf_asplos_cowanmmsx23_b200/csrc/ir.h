@@ -76,7 +76,7 @@ void validateIR(Algo& a, int nranks, int slots, int maxTbs, int maxChannels, int
 // sendDirect[tb][step] = the matching receive on the peer is direct (+ its dst buf/off).
 struct DirectInfo {
   std::vector<std::vector<char>> recvDirect, sendDirect;
-  std::vector<std::vector<int>> rdstBuf, rdstOff;
+  std::vector<std::vector<int>> rdstBuf, rdstOff, rterminal;
 };
 DirectInfo directPlacement(const Algo& a, int rank);
 

@@ -27,7 +27,7 @@ namespace {
 
 struct Params {
   int64_t slots = 4, slotBytes = 262144, maxChannels = 32, threads = 512, timeoutS = 20, tma = 0, direct = 1,
-          warp = 0, l2PersistMiB = 0, prefetch = 0, directTile = 1, balance = 0;
+          warp = 0, l2PersistMiB = 0, prefetch = 0, directTile = 1, balance = 0, directHints = 1;
 };
 
 std::mutex gMu;
@@ -49,6 +49,7 @@ int64_t* paramRef(Params& p, const std::string& k) {
   if (k == "MSCCL_PREFETCH") return &p.prefetch;
   if (k == "MSCCL_DIRECT_TILE") return &p.directTile;
   if (k == "MSCCL_BALANCE") return &p.balance;
+  if (k == "MSCCL_DIRECT_HINTS") return &p.directHints;
   return nullptr;
 }
 
@@ -59,7 +60,7 @@ Params currentParams() {
     for (const char* k : {"MSCCL_SLOTS", "MSCCL_SLOT_BYTES", "MSCCL_MAX_CHANNELS", "MSCCL_THREADS", "MSCCL_TIMEOUT_S",
                           "MSCCL_TMA", "MSCCL_DIRECT", "MSCCL_WARP_FLAGS",
                           "MSCCL_L2_PERSIST_MIB", "MSCCL_PREFETCH", "MSCCL_DIRECT_TILE",
-                          "MSCCL_BALANCE"}) {
+                          "MSCCL_BALANCE", "MSCCL_DIRECT_HINTS"}) {
       const char* v = getenv(k);
       if (v && *v) *paramRef(gParams, k) = atoll(v);
     }
@@ -122,7 +123,7 @@ struct mscclProgram {
   int nTB = 0, nInstr = 0;
   DevTB* dTBs = nullptr;
   DevInstr* dInstr = nullptr;
-  uint32_t* dDeps = nullptr;
+  uint64_t* dDeps = nullptr;
   uint64_t* dSem = nullptr;  // nTB sems followed by nTB gens
   char* dScratch = nullptr;
   size_t scratchBytes = 0;
@@ -211,8 +212,8 @@ uint64_t* traceBuffer() {
   if (!init) {
     init = true;
     const char* v = getenv("MSCCL_TRACE");
-    if (v && *v == '1' && cudaHostAlloc(&gTraceHost, 4096 * 8 * sizeof(uint64_t), cudaHostAllocMapped) == cudaSuccess) {
-      memset(gTraceHost, 0, 4096 * 8 * sizeof(uint64_t));
+    if (v && *v == '1' && cudaHostAlloc(&gTraceHost, 4096 * 32 * sizeof(uint64_t), cudaHostAllocMapped) == cudaSuccess) {
+      memset(gTraceHost, 0, 4096 * 32 * sizeof(uint64_t));
       cudaHostGetDevicePointer((void**)&gTraceDev, gTraceHost, 0);
     }
   }
@@ -383,6 +384,7 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
     ka.direct = direct ? 1 : 0;
     ka.warpFlags = (ka.proto == 0 && c0->prm.warp && !ka.useTma) ? 1 : 0;
     ka.prefetch = (ka.proto == 0 && c0->prm.prefetch) ? 1 : 0;
+    ka.directHints = (int32_t)c0->prm.directHints;
     const int smem = ka.useTma ? tmaSmemBytes() : 0;
     int maxCta = 0;
     r = coResident(c0, fn, (int)c0->prm.threads, smem, maxCta);
@@ -711,7 +713,7 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
   p->tbWork.assign(p->nTB, 0);
   p->tbWorkDirect.assign(p->nTB, 0);
   std::vector<DevInstr> ins;
-  std::vector<uint32_t> deps;
+  std::vector<uint64_t> deps;
   for (int t = 0; t < p->nTB; t++) {
     const ThreadBlock& tb = g.tbs[t];
     DevTB& d = tbs[t];
@@ -746,7 +748,11 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
       di.srcOff = (uint32_t)std::max(in.srcOff, 0);
       di.dstOff = (uint32_t)std::max(in.dstOff, 0);
       di.depStart = (uint32_t)deps.size();
-      for (auto& dp : in.deps) deps.push_back(((uint32_t)dp.first << 16) | (uint32_t)dp.second);
+      // dependency word: the waiter computes the semaphore target without reading the
+      // other thread block's descriptor (one memory round trip instead of two)
+      for (auto& dp : in.deps)
+        deps.push_back(((uint64_t)dp.first << 48) | ((uint64_t)dp.second << 32) |
+                       (uint64_t)(uint32_t)g.tbs[dp.first].steps.size());
       if (dinfo.recvDirect[t][si]) di.flags |= DI_RECV_DIRECT;
       {  // operand touches of this instruction (mscclProgramTouches costs)
         static const int cost[OP_COUNT] = {0, 2, 2, 2, 3, 3, 3, 4, 3};
@@ -761,6 +767,7 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
         di.flags |= DI_SEND_DIRECT;
         di.rdstBuf = (uint8_t)dinfo.rdstBuf[t][si];
         di.rdstOff = (uint32_t)dinfo.rdstOff[t][si];
+        if (dinfo.rterminal[t][si]) di.flags |= DI_SEND_TERMINAL;
       }
       ins.push_back(di);
     }
@@ -808,8 +815,8 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
     CUDACHECK(c, cudaMemcpy(p->dInstr, ins.data(), ins.size() * sizeof(DevInstr), cudaMemcpyHostToDevice));
   }
   if (!deps.empty()) {
-    CUDACHECK(c, cudaMalloc(&p->dDeps, deps.size() * sizeof(uint32_t)));
-    CUDACHECK(c, cudaMemcpy(p->dDeps, deps.data(), deps.size() * sizeof(uint32_t), cudaMemcpyHostToDevice));
+    CUDACHECK(c, cudaMalloc(&p->dDeps, deps.size() * sizeof(uint64_t)));
+    CUDACHECK(c, cudaMemcpy(p->dDeps, deps.data(), deps.size() * sizeof(uint64_t), cudaMemcpyHostToDevice));
   }
   p->index = (int)c->programs.size();
   c->programs.push_back(p.get());

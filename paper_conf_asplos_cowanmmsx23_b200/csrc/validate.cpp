@@ -218,12 +218,14 @@ DirectInfo directPlacement(const Algo& a, int rank) {
   di.sendDirect.resize(g.tbs.size());
   di.rdstBuf.resize(g.tbs.size());
   di.rdstOff.resize(g.tbs.size());
+  di.rterminal.resize(g.tbs.size());
   for (size_t t = 0; t < g.tbs.size(); t++) {
     const ThreadBlock& tb = g.tbs[t];
     di.recvDirect[t].assign(tb.steps.size(), 0);
     di.sendDirect[t].assign(tb.steps.size(), 0);
     di.rdstBuf[t].assign(tb.steps.size(), 0);
     di.rdstOff[t].assign(tb.steps.size(), 0);
+    di.rterminal[t].assign(tb.steps.size(), 0);
     for (size_t s = 0; s < tb.steps.size(); s++)
       if (opRole(tb.steps[s].op).recv) di.recvDirect[t][s] = recvCanBeDirect(a, rank, (int)t, (int)s);
     if (tb.send < 0) continue;
@@ -245,6 +247,7 @@ DirectInfo directPlacement(const Algo& a, int rank) {
           di.sendDirect[t][s] = 1;
           di.rdstBuf[t][s] = rt->steps[rs].dstBuf;
           di.rdstOff[t][s] = rt->steps[rs].dstOff;
+          di.rterminal[t][s] = rt->steps[rs].op == OP_RECV ? 1 : 0;
         }
       }
       k++;
