@@ -257,8 +257,8 @@ def sampled_parity(algo, recv_list, n, ranks_to_check):
     idx = np.unique(np.concatenate([g.integers(0, n, SEED_SAMPLES), [0, n - 1, n // 2]]))
     bad = 0
     for q in ranks_to_check:
-        want = sampled.allreduce_at(al, lambda r, i: synth.hashed_numpy(r, i, "bfloat16"), n, "bfloat16", "sum",
-                                    idx, rank=q)
+        want = sampled.reduction_at(al, lambda r, i: synth.hashed_numpy(r, i, "bfloat16"), n, "bfloat16", "sum",
+                                      idx, rank=q)
         got = recv_list[q][torch.from_numpy(idx).to(recv_list[q].device)].view(torch.int16).cpu().numpy() \
             .view(np.uint16)
         bad += int(np.count_nonzero(got != want))
@@ -463,7 +463,8 @@ def virtual_extras(comms, R, stream):
         if coll == "allgather":
             ok = all(torch.equal(recv[q].view(R, -1)[p], send[p]) for q in (0, R - 1) for p in range(R))
         else:
-            ok = None
+            bad, _ = sampled_parity(algo, recv, nb, [0, R - 1])
+            ok = bad == 0
         out[name + "_bf16_256MiB"] = {"busbw_GBps": round(busbw(coll, S, t, R), 2), "ms": round(t * 1e3, 3),
                                       "instances": 32, "bit_exact": ok}
         for c, p in zip(comms, progs):

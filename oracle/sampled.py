@@ -20,12 +20,16 @@ def _eval(tree, leafval, op, dtype):
     return nm.reduce(_eval(a, leafval, op, dtype), _eval(b, leafval, op, dtype), op, dtype)
 
 
-def allreduce_at(algo, value_at, count, dtype, op, idx, rank=0):
-    """Output of `rank` at element indices `idx` (AllReduce programs).
+def reduction_at(algo, value_at, count, dtype, op, idx, rank=0):
+    """Output of `rank` at output element indices `idx` (AllReduce / ReduceScatter programs).
 
     value_at(q, indices) -> numpy array (storage dtype) of rank q's input at `indices`.
+    Output element e lies in output chunk k = e // E at position e - k*E (the output
+    buffer is one block for both collectives, reading R1); a leaf (q, kk) of that chunk's
+    tree is input chunk kk of rank q, whose span comes from the same geometry (for
+    ReduceScatter the input holds R blocks, so kk = b*C_b + j starts at b*n + j*E).
     """
-    assert algo.coll == "allreduce"
+    assert algo.coll in ("allreduce", "reducescatter")
     trees = check(algo)
     geo = Geometry(algo, count, nm.elem_bytes(dtype))
     idx = np.asarray(idx, dtype=np.int64)
@@ -36,6 +40,12 @@ def allreduce_at(algo, value_at, count, dtype, op, idx, rank=0):
         pos = idx[sel] - k * geo.E
 
         def leaf(q, kk, pos=pos):
-            return value_at(q, kk * geo.E + pos)
+            return value_at(q, geo.span("i", kk)[0] + pos)
         out[sel] = _eval(trees[rank][int(k)], leaf, op, dtype)
     return out
+
+
+def allreduce_at(algo, value_at, count, dtype, op, idx, rank=0):
+    """Output of `rank` at element indices `idx` (AllReduce programs)."""
+    assert algo.coll == "allreduce"
+    return reduction_at(algo, value_at, count, dtype, op, idx, rank)

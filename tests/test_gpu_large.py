@@ -105,3 +105,39 @@ def test_bench_size_sampled_parity(instances):
     finally:
         for c, p in zip(cs, progs):
             c.unload(p)
+
+
+def test_bench_size_reducescatter_sampled_parity():
+    """The bench's ReduceScatter extra (ring, 32 instances, 256 MiB input per rank) at full
+    size; outputs sampled on every rank and compared bit-exactly with the oracle's reduction
+    trees (oracle.sampled.reduction_at)."""
+    import torch
+    import gpu_util
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    R, n = 8, (256 << 20) // 2
+    nb = n // R
+    algo = P.ring_reducescatter(R, 1, 32)
+    ir = algo.to_xml()
+    cs = gpu_util.comms(R)
+    progs = [c.load(ir) for c in cs]
+    try:
+        dev = torch.device("cuda:0")
+        idx = torch.arange(n, device=dev, dtype=torch.int64)
+        send = [synth.hashed(q, idx, "bfloat16") for q in range(R)]
+        del idx
+        recv = [torch.empty(nb, dtype=torch.bfloat16, device=dev) for _ in range(R)]
+        with runtime.group():
+            for q in range(R):
+                cs[q].run(progs[q], send[q], recv[q], nb)
+        torch.cuda.synchronize()
+        al = irparse.parse(ir)
+        g = np.random.default_rng(6)
+        sample = np.unique(np.concatenate([g.integers(0, nb, 2048), [0, nb - 1]]))
+        for q in range(R):
+            want = sampled.reduction_at(al, lambda rr, i: synth.hashed_numpy(rr, i, "bfloat16"), nb, "bfloat16",
+                                        "sum", sample, rank=q)
+            got = recv[q][torch.from_numpy(sample).to(dev)].view(torch.int16).cpu().numpy().view(np.uint16)
+            assert np.array_equal(got, want), "rank %d" % q
+    finally:
+        for c, p in zip(cs, progs):
+            c.unload(p)
