@@ -1161,6 +1161,124 @@ __device__ __noinline__ void chainExec(const Ctx& c, const DevInstr* mem, int L,
   }
 }
 
+// Simple-protocol kernels: the chain pass of reading R16 with its operand table in registers
+// and one operand load per member (the shared-memory table and batched loads of chainExec
+// below cut latency in the LL kernels, but their code in the Simple kernels cost 6 % of ring
+// bandwidth through register allocation of the kernel body: measured A/B).
+template <int DT, int OP>
+__device__ __noinline__ void chainExecSimple(const Ctx& c, const DevInstr* mem, int L, int t) {
+  typedef typename DType<DT>::T T;
+  const KernelArgs& a = *c.a;
+  const RankArgs& ra = *c.ra;
+  const int64_t w = sizeof(T);
+  const int64_t a0 = (int64_t)t * a.T;
+  const bool headCopy = mem[0].op == K_COPY;
+  for (int j = 0; j < mem[0].cnt; j++) {
+    int64_t ds, dl;
+    chunkSpan(a, mem[0].dstBuf, (int64_t)mem[0].dstOff + j, ds, dl);
+    const char* srcs[MSCCL_MAX_CHAIN];
+    int64_t m = -1;
+    bool same = true;
+    uintptr_t al = 0;
+    for (int k = 0; k < L; k++) {
+      int64_t ss, sl;
+      chunkSpan(a, mem[k].srcBuf, (int64_t)mem[k].srcOff + j, ss, sl);
+      int64_t Lk = sl < dl ? sl : dl;
+      int64_t mk = (a0 + a.T < Lk ? a0 + a.T : Lk) - a0;
+      if (m < 0) m = mk;
+      else if (mk != m) same = false;
+      srcs[k] = ra.buf[mem[k].srcBuf] + (ss + a0) * w;
+      al |= (uintptr_t)srcs[k];
+    }
+    char* dst = ra.buf[mem[0].dstBuf] + (ds + a0) * w;
+    al |= (uintptr_t)dst;
+    if (!same) {  // sequential fallback (a barrier between members: element->thread maps differ)
+      for (int k = 0; k < L; k++) {
+        int64_t ss, sl;
+        chunkSpan(a, mem[k].srcBuf, (int64_t)mem[k].srcOff + j, ss, sl);
+        int64_t Lk = sl < dl ? sl : dl;
+        int64_t mk = (a0 + a.T < Lk ? a0 + a.T : Lk) - a0;
+        if (mk > 0) {
+          if (mem[k].op == K_COPY)
+            pieceSimple<DT, OP, false, false, true, true, false>(mk, nullptr, srcs[k], dst, nullptr, c.tid, c.nt);
+          else
+            pieceSimple<DT, OP, false, false, true, true, true>(mk, nullptr, srcs[k], dst, nullptr, c.tid, c.nt);
+        }
+        __syncthreads();
+      }
+      continue;
+    }
+    if (m <= 0) continue;
+    const int64_t bytes = m * w;
+    int64_t nvec = (al & 15) ? 0 : bytes / 16;
+    for (int64_t i = c.tid; i < nvec; i += c.nt) {
+      uint4 acc = headCopy ? ldcg(srcs[0] + i * 16) : ldcg(dst + i * 16);
+      for (int k = headCopy ? 1 : 0; k < L; k++) acc = vop<DT, OP>(acc, ldcg(srcs[k] + i * 16));
+      stg(dst + i * 16, acc);
+    }
+    for (int64_t e = nvec * 16 / w + c.tid; e < m; e += c.nt) {
+      T acc = headCopy ? *(const T*)(srcs[0] + e * w) : *(const T*)(dst + e * w);
+      for (int k = headCopy ? 1 : 0; k < L; k++) acc = DType<DT>::op(OP, acc, *(const T*)(srcs[k] + e * w));
+      *(T*)(dst + e * w) = acc;
+    }
+  }
+}
+
+// Reading R16: one fused local reduce chain starting at step s (dependency waits of all its
+// members, the one-pass fold, the semaphore post of its last member). Returns the chain's last
+// step, or -1 on watchdog / abort. Not inlined: its dependency-collection loop in the kernel
+// body raised the Simple kernel's register pressure and cost 6 % on the ring (measured).
+template <int DT, int OP, int PROTO>
+__device__ __noinline__ int runChain(const Ctx& c, const RankArgs& ra, const DevInstr* ins, int s, int t, uint64_t gen,
+                                     int tbi, int nSteps, ChainSmem& sChain, volatile int* sAbort, uint64_t* tl) {
+  const int L = ins[s].chainLen;
+  bool ok = true;
+  // all members' dependencies first: flattened dependency f goes to thread f mod nt; a
+  // thread first collects its dependency words, then waits on all of them, so the waits
+  // of different members overlap (waiting inside the member loop serialises them: one
+  // member per loop trip)
+  {
+    constexpr int KD = 4;
+    uint64_t mine[KD];
+    int nm = 0;
+    for (int k = 0, base = 0; k < L; k++) {
+      const DevInstr& mk = ins[s + k];
+      for (int d = ((c.tid - base) % c.nt + c.nt) % c.nt; d < mk.nDeps; d += c.nt) {
+        const uint64_t dw = ra.deps[mk.depStart + d];
+        if (nm < KD) mine[nm++] = dw;
+        else ok = ok && waitDep(ra, dw, gen, t, c);  // more than KD per thread: in order
+      }
+      base += mk.nDeps;
+    }
+#pragma unroll
+    for (int i = 0; i < KD; i++)
+      if (i < nm) ok = ok && waitDep(ra, mine[i], gen, t, c);
+  }
+#if MSCCL_TIMELINE
+  if (tl && c.tid == 0) tl[16] = globaltimer();
+#endif
+  if (!ok) *sAbort = 1;
+  __syncthreads();
+  if (*sAbort) return -1;
+#if MSCCL_TIMELINE
+  if (tl && c.tid == 0) tl[13] = globaltimer();
+#endif
+  chainExec<DT, OP, PROTO == 1 ? 8 : 2>(c, ins + s, L, t, sChain, tl);
+  __syncthreads();
+#if MSCCL_TIMELINE
+  if (tl && c.tid == 0) tl[14] = globaltimer();
+#endif
+  s += L - 1;
+  if (ins[s].hasDep && c.tid == 0) {
+    fenceGpu();
+    stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)nSteps + (uint64_t)s + 1));
+  }
+#if MSCCL_TIMELINE
+  if (tl && c.tid == 0 && s < 10 && t < 2) tl[(t ? 18 : 2) + s] = globaltimer();
+#endif
+  return s;
+}
+
 #ifndef MSCCL_MAX_THREADS
 #define MSCCL_MAX_THREADS 512
 #endif
@@ -1268,51 +1386,27 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
       const DevInstr in = ins[s];
       if constexpr (OP != R_COPY) {
         if (in.flags & DI_CHAIN_HEAD) {  // reading R16: fused local reduce chain
-          const int L = in.chainLen;
-          bool ok = true;
-          // all members' dependencies first: flattened dependency f goes to thread f mod nt; a
-          // thread first collects its dependency words, then waits on all of them, so the waits
-          // of different members overlap (waiting inside the member loop serialises them: one
-          // member per loop trip)
-          {
-            constexpr int KD = 4;
-            uint64_t mine[KD];
-            int nm = 0;
-            for (int k = 0, base = 0; k < L; k++) {
+          if constexpr (PROTO == 0) {
+            const int L = in.chainLen;
+            bool ok = true;
+            for (int k = 0; k < L && ok; k++) {  // all members' dependencies first
               const DevInstr& mk = ins[s + k];
-              for (int d = ((c.tid - base) % c.nt + c.nt) % c.nt; d < mk.nDeps; d += c.nt) {
-                const uint64_t dw = ra.deps[mk.depStart + d];
-                if (nm < KD) mine[nm++] = dw;
-                else ok = ok && waitDep(ra, dw, gen, t, c);  // more than KD per thread: in order
-              }
-              base += mk.nDeps;
+              for (int d = c.tid; d < mk.nDeps && ok; d += c.nt) ok = waitDep(ra, ra.deps[mk.depStart + d], gen, t, c);
             }
-#pragma unroll
-            for (int i = 0; i < KD; i++)
-              if (i < nm) ok = ok && waitDep(ra, mine[i], gen, t, c);
+            if (!ok) sAbort = 1;
+            __syncthreads();
+            if (sAbort) return;
+            chainExecSimple<DT, OP>(c, ins + s, L, t);
+            __syncthreads();
+            s += L - 1;
+            if (ins[s].hasDep && c.tid == 0) {
+              fenceGpu();
+              stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)tb.nSteps + (uint64_t)s + 1));
+            }
+          } else {
+            s = runChain<DT, OP, PROTO>(c, ra, ins, s, t, gen, tbi, tb.nSteps, sChain, &sAbort, tl);
+            if (s < 0) return;
           }
-#if MSCCL_TIMELINE
-          if (tl && threadIdx.x == 0) tl[16] = globaltimer();
-#endif
-          if (!ok) sAbort = 1;
-          __syncthreads();
-          if (sAbort) return;
-#if MSCCL_TIMELINE
-          if (tl && threadIdx.x == 0) tl[13] = globaltimer();
-#endif
-          chainExec<DT, OP, PROTO == 1 ? 8 : 2>(c, ins + s, L, t, sChain, tl);
-          __syncthreads();
-#if MSCCL_TIMELINE
-          if (tl && threadIdx.x == 0) tl[14] = globaltimer();
-#endif
-          s += L - 1;
-          if (ins[s].hasDep && c.tid == 0) {
-            fenceGpu();
-            stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)tb.nSteps + (uint64_t)s + 1));
-          }
-#if MSCCL_TIMELINE
-          if (tl && threadIdx.x == 0 && s < 10 && t < 2) tl[(t ? 18 : 2) + s] = globaltimer();
-#endif
           continue;
         }
       }
