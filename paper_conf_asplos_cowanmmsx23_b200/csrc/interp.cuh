@@ -1224,60 +1224,6 @@ __device__ __noinline__ void chainExecSimple(const Ctx& c, const DevInstr* mem, 
   }
 }
 
-// Reading R16: one fused local reduce chain starting at step s (dependency waits of all its
-// members, the one-pass fold, the semaphore post of its last member). Returns the chain's last
-// step, or -1 on watchdog / abort. Not inlined: its dependency-collection loop in the kernel
-// body raised the Simple kernel's register pressure and cost 6 % on the ring (measured).
-template <int DT, int OP, int PROTO>
-__device__ __noinline__ int runChain(const Ctx& c, const RankArgs& ra, const DevInstr* ins, int s, int t, uint64_t gen,
-                                     int tbi, int nSteps, ChainSmem& sChain, volatile int* sAbort, uint64_t* tl) {
-  const int L = ins[s].chainLen;
-  bool ok = true;
-  // all members' dependencies first: flattened dependency f goes to thread f mod nt; a
-  // thread first collects its dependency words, then waits on all of them, so the waits
-  // of different members overlap (waiting inside the member loop serialises them: one
-  // member per loop trip)
-  {
-    constexpr int KD = 4;
-    uint64_t mine[KD];
-    int nm = 0;
-    for (int k = 0, base = 0; k < L; k++) {
-      const DevInstr& mk = ins[s + k];
-      for (int d = ((c.tid - base) % c.nt + c.nt) % c.nt; d < mk.nDeps; d += c.nt) {
-        const uint64_t dw = ra.deps[mk.depStart + d];
-        if (nm < KD) mine[nm++] = dw;
-        else ok = ok && waitDep(ra, dw, gen, t, c);  // more than KD per thread: in order
-      }
-      base += mk.nDeps;
-    }
-#pragma unroll
-    for (int i = 0; i < KD; i++)
-      if (i < nm) ok = ok && waitDep(ra, mine[i], gen, t, c);
-  }
-#if MSCCL_TIMELINE
-  if (tl && c.tid == 0) tl[16] = globaltimer();
-#endif
-  if (!ok) *sAbort = 1;
-  __syncthreads();
-  if (*sAbort) return -1;
-#if MSCCL_TIMELINE
-  if (tl && c.tid == 0) tl[13] = globaltimer();
-#endif
-  chainExec<DT, OP, PROTO == 1 ? 8 : 2>(c, ins + s, L, t, sChain, tl);
-  __syncthreads();
-#if MSCCL_TIMELINE
-  if (tl && c.tid == 0) tl[14] = globaltimer();
-#endif
-  s += L - 1;
-  if (ins[s].hasDep && c.tid == 0) {
-    fenceGpu();
-    stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)nSteps + (uint64_t)s + 1));
-  }
-#if MSCCL_TIMELINE
-  if (tl && c.tid == 0 && s < 10 && t < 2) tl[(t ? 18 : 2) + s] = globaltimer();
-#endif
-  return s;
-}
 
 #ifndef MSCCL_MAX_THREADS
 #define MSCCL_MAX_THREADS 512
@@ -1404,8 +1350,51 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
               stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)tb.nSteps + (uint64_t)s + 1));
             }
           } else {
-            s = runChain<DT, OP, PROTO>(c, ra, ins, s, t, gen, tbi, tb.nSteps, sChain, &sAbort, tl);
-            if (s < 0) return;
+            const int L = in.chainLen;
+            bool ok = true;
+            // all members' dependencies first: flattened dependency f goes to thread f mod nt; a
+            // thread first collects its dependency words, then waits on all of them, so the waits
+            // of different members overlap (waiting inside the member loop serialises them: one
+            // member per loop trip)
+            {
+              constexpr int KD = 4;
+              uint64_t mine[KD];
+              int nm = 0;
+              for (int k = 0, base = 0; k < L; k++) {
+                const DevInstr& mk = ins[s + k];
+                for (int d = ((c.tid - base) % c.nt + c.nt) % c.nt; d < mk.nDeps; d += c.nt) {
+                  const uint64_t dw = ra.deps[mk.depStart + d];
+                  if (nm < KD) mine[nm++] = dw;
+                  else ok = ok && waitDep(ra, dw, gen, t, c);  // more than KD per thread: in order
+                }
+                base += mk.nDeps;
+              }
+#pragma unroll
+              for (int i = 0; i < KD; i++)
+                if (i < nm) ok = ok && waitDep(ra, mine[i], gen, t, c);
+            }
+#if MSCCL_TIMELINE
+            if (tl && c.tid == 0) tl[16] = globaltimer();
+#endif
+            if (!ok) sAbort = 1;
+            __syncthreads();
+            if (sAbort) return;
+#if MSCCL_TIMELINE
+            if (tl && c.tid == 0) tl[13] = globaltimer();
+#endif
+            chainExec<DT, OP, PROTO == 1 ? 8 : 2>(c, ins + s, L, t, sChain, tl);
+            __syncthreads();
+#if MSCCL_TIMELINE
+            if (tl && c.tid == 0) tl[14] = globaltimer();
+#endif
+            s += L - 1;
+            if (ins[s].hasDep && c.tid == 0) {
+              fenceGpu();
+              stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)tb.nSteps + (uint64_t)s + 1));
+            }
+#if MSCCL_TIMELINE
+            if (tl && c.tid == 0 && s < 10 && t < 2) tl[(t ? 18 : 2) + s] = globaltimer();
+#endif
           }
           continue;
         }
