@@ -337,6 +337,9 @@ __device__ __forceinline__ void chunkSpan(const KernelArgs& a, int buf, int64_t 
 #ifndef MSCCL_FENCE_MODE
 #define MSCCL_FENCE_MODE 0
 #endif
+#ifndef MSCCL_POST_LAST_WARP
+#define MSCCL_POST_LAST_WARP 1
+#endif
 #ifndef MSCCL_UNROLL
 #define MSCCL_UNROLL 4   // vectors in flight per lane and input stream (two input streams)
 #endif
@@ -1020,7 +1023,9 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
   // block-level protocols post every flag word (a later warp-flag launch waits on its own word)
   if (c.tid == 0 && ll && RECV) {  // LL/LL128: data carried its own flags; the ack frees the slot
     postWords(tb.recvAck, recvd + 1, sys);
-  } else if (c.tid == 0 && (RECV || SEND) && !ll) {
+  } else if (c.tid == (MSCCL_POST_LAST_WARP ? c.nt - 32 : 0) && (RECV || SEND) && !ll) {
+    // Simple: lane 0 of the last warp posts, so thread 0 (the head poller) goes straight to the
+    // next step's wait and the fence latency overlaps it (option MSCCL_POST_LAST_WARP)
     if (sys) fenceSys();
     else fenceGpu();
     if (SEND) postWords(tb.sendHead, sent + 1, sys);
