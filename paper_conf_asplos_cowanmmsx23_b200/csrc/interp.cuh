@@ -1327,6 +1327,9 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
   // without doing anything, so the block-wide barriers below still match; at the next one
   // every thread sees sAbort and returns.
   const bool warpMode = PROTO == 0 && a.warpFlags;
+  // semaphore posts (fence + store) by lane 0 of the last warp: thread 0 polls the next step's
+  // head / dependencies meanwhile; every post follows a block barrier (option MSCCL_POST_LAST_WARP)
+  const int kPoster = MSCCL_POST_LAST_WARP ? (int)blockDim.x - 32 : 0;
   bool dead = false;
   __syncthreads();
 #if MSCCL_TIMELINE
@@ -1350,7 +1353,7 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
             chainExecSimple<DT, OP>(c, ins + s, L, t);
             __syncthreads();
             s += L - 1;
-            if (ins[s].hasDep && c.tid == 0) {
+            if (ins[s].hasDep && c.tid == kPoster) {
               fenceGpu();
               stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)tb.nSteps + (uint64_t)s + 1));
             }
@@ -1393,7 +1396,7 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
             if (tl && c.tid == 0) tl[14] = globaltimer();
 #endif
             s += L - 1;
-            if (ins[s].hasDep && c.tid == 0) {
+            if (ins[s].hasDep && c.tid == kPoster) {
               fenceGpu();
               stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)tb.nSteps + (uint64_t)s + 1));
             }
@@ -1429,7 +1432,7 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
         if (!dispatch<DT, OP, PROTO>(c, tb, in, t, sent, recvd, &sAbort)) return;
       }
       if (in.hasDep) {  // Fig. 5 lines 25-27: the step is complete before the semaphore moves
-        if (c.tid == 0) {
+        if (c.tid == kPoster) {
           fenceGpu();
           stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)tb.nSteps + (uint64_t)s + 1));
         }
