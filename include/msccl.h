@@ -15,8 +15,12 @@
  *    valid until the stream reaches the operation; `count`s are ELEMENTS of `datatype`;
  *  - a communicator is not thread-safe (NCCL rule); all ranks must load the same programs
  *    in the same order and issue the same collectives with the same count/dtype/op;
- *  - calls are asynchronous on `stream` and contain no host synchronisation or
- *    allocation, so they can be captured in a CUDA graph;
+ *  - calls are asynchronous on `stream` and contain no host synchronisation. A call
+ *    allocates only when a program loaded WITHOUT maxBytes needs more scratch than any
+ *    earlier call (it then grows; the old buffer lives until unload). Programs loaded with
+ *    maxBytes pre-size their scratch, so every call in their size range can be captured in
+ *    a CUDA graph, the first one included; a call that would have to grow scratch while the
+ *    stream is capturing returns mscclInvalidUsage instead;
  *  - mscclGetLastError(comm) returns a human-readable reason for the last failure
  *    (for program errors: rank/thread block/step and the violated rule V1..V9).
  */
@@ -92,8 +96,33 @@ mscclResult_t mscclCommUserRank(const mscclComm_t comm, int* rank);
 mscclResult_t mscclCommCuDevice(const mscclComm_t comm, int* device);
 
 /* Sticky asynchronous error: mscclRemoteError after a device watchdog timeout (a spin
- * wait exceeded MSCCL_TIMEOUT_S, default 20 s) or an abort raised by a peer. */
+ * wait exceeded MSCCL_TIMEOUT_S, default 60 s; <= 0 disables the watchdog) or an abort
+ * raised by a peer. */
 mscclResult_t mscclCommGetAsyncError(mscclComm_t comm, mscclResult_t* asyncError);
+
+/* ---------------------------------------------------------------- buffer registration
+ * Direct placement (readings R15 / R15b; the paper's future work, §7.5
+ * P:L2615-2624): a sender stores a message straight into the receiver's destination chunk
+ * instead of the receiver-side FIFO. Within one process (mscclCommInitAll, any devices)
+ * every buffer is reachable and nothing needs registering. For one process per GPU (CUDA
+ * IPC), a receiver's buffer is reachable only if it lies inside a REGISTERED range:
+ *   mscclCommRegister(comm, buff, size, &reg)   every rank, same order (collective)
+ *   mscclRegExport(reg, desc)                   MSCCL_REG_DESC_BYTES bytes
+ *   (exchange the descriptors, e.g. torch.distributed all_gather)
+ *   mscclRegConnect(reg, allDescs)              nranks * MSCCL_REG_DESC_BYTES, rank order;
+ *                                               maps every peer's range; all ranks must
+ *                                               return from it before any uses the buffer
+ * A call whose recvbuff (or sendbuff, for in-place programs) is not inside a connected
+ * registration simply uses the FIFO for messages to this rank. Registration allocates and
+ * synchronises (not capturable). mscclCommDeregister unmaps (collective, after the stream
+ * work that used the buffer has completed). Errors: InvalidArgument (null, size 0, range
+ * not inside one device allocation, more than MSCCL_MAX_REGISTRATIONS), UnhandledCudaError. */
+typedef struct mscclReg* mscclReg_t;
+#define MSCCL_REG_DESC_BYTES 128
+mscclResult_t mscclCommRegister(mscclComm_t comm, void* buff, size_t size, mscclReg_t* reg);
+mscclResult_t mscclRegExport(mscclReg_t reg, void* desc);
+mscclResult_t mscclRegConnect(mscclReg_t reg, const void* allDescs);
+mscclResult_t mscclCommDeregister(mscclComm_t comm, mscclReg_t reg);
 
 /* ---------------------------------------------------------------- programs */
 
@@ -116,6 +145,17 @@ mscclResult_t mscclProgramInfo(mscclProgram_t program, int* nThreadBlocks, int* 
  * and with direct placement (directPlacement != 0, reading R15) a direct recv costs 0 and
  * a direct rcs 2 (the data arrived in dst). */
 mscclResult_t mscclProgramTouches(mscclProgram_t program, int directPlacement, int64_t* touches);
+
+/* Direct-placement marking the loader computes for rank `rank` of an IR program (reading
+ * R15; needs no GPU). For every instruction in (thread block, step) order of that rank,
+ * flags[k] = bit 0 DIRECT_SEND (the message is stored into the receiver's destination),
+ * bit 1 DIRECT_RECV (the data is already in dst when the head arrives); for a direct send
+ * rdst[2k], rdst[2k+1] = the receiver's destination buffer (0 i, 1 o, 2 s) and chunk.
+ * maxInstr = capacity of flags (rdst: 2*maxInstr); *nInstr = instructions of the rank.
+ * Exported so the CPU oracle's race detector (oracle/races.py) can check the marking
+ * independently. Returns mscclInvalidProgram if the IR does not parse or validate. */
+mscclResult_t mscclDebugDirectPlacement(const char* ir, size_t irBytes, int rank, int32_t* flags,
+                                        int32_t* rdst, int maxInstr, int* nInstr);
 
 /* Comm-free structural validation (rules V1..V9 of DESIGN.md) — needs no GPU.
  * slots = FIFO slots per connection used by the deadlock check (0 = library default),
@@ -161,10 +201,15 @@ const char* mscclGetErrorString(mscclResult_t result);
 const char* mscclGetLastError(mscclComm_t comm); /* comm may be NULL: last global error */
 
 /* Tuning knobs (process-wide, read when a communicator is created; env vars of the same
- * name override at first use): "MSCCL_SLOTS" FIFO slots per connection (1..16, default 4),
- * "MSCCL_SLOT_BYTES" Simple-protocol slot size (default 262144), "MSCCL_MAX_CHANNELS"
- * (default 32), "MSCCL_THREADS" threads per CTA (default 512), "MSCCL_TIMEOUT_S"
- * watchdog (default 20). Returns mscclInvalidArgument for an unknown key. */
+ * name override at first use). Defaults are the tuned configuration of DESIGN.md §7:
+ * "MSCCL_SLOTS" FIFO slots per connection (1..16, default 4); "MSCCL_SLOT_BYTES" Simple
+ * slot (default 262144), "MSCCL_LL_SLOT_BYTES" (65536), "MSCCL_LL128_SLOT_BYTES" (262144)
+ * -- each protocol has its own slots; "MSCCL_MAX_CHANNELS" (32); "MSCCL_THREADS" threads
+ * per CTA (64..256, default 256 = 2 CTAs per SM); "MSCCL_TIMEOUT_S" watchdog (default 60,
+ * <= 0 disables); "MSCCL_DIRECT" direct placement (1); "MSCCL_DIRECT_TILE" one tile per
+ * chunk when every message is direct (1); "MSCCL_MAX_REGISTRATIONS" (64). All ranks must
+ * use the same values (mscclCommConnect checks). Returns mscclInvalidArgument for an
+ * unknown key. */
 mscclResult_t mscclSetParam(const char* key, int64_t value);
 mscclResult_t mscclGetParam(const char* key, int64_t* value);
 

@@ -8,9 +8,12 @@
 
 namespace msccl {
 
-#define MSCCL_MAX_LOCAL 16  // ranks that one kernel launch may cover (virtual ranks)
-#define MSCCL_FLAG_WORDS 16 // u64 flag words per connection counter: one per warp (<= 512 threads)
-#define MSCCL_CTA_MAP 512   // largest grid whose CTA -> (rank, thread block) order the host sets
+#define MSCCL_MAX_LOCAL 16   // ranks that one kernel launch may cover (virtual ranks)
+#define MSCCL_FLAG_STRIDE 16 // u64 words between connection counters (one 128-byte line each)
+#define MSCCL_REF_REG (1ull << 63)  // destination reference: registered-buffer (index, offset) form
+#ifndef MSCCL_MAX_THREADS
+#define MSCCL_MAX_THREADS 256  // threads per CTA (MSCCL_THREADS <= this); 2 CTAs per SM at 256
+#endif
 
 // DI_SEND_TERMINAL: a direct send whose receiving instruction is a plain recv (the data is
 // not forwarded by the receiver's thread block: a cache hint only)
@@ -35,20 +38,21 @@ struct DevTB {
   uint32_t instrStart;
   int32_t tbId;
   int32_t sendPeer;           // rank of the send peer (-1 if none)
-  // send connection (peer = receiver): FIFO and head counter live in the PEER's region.
-  // head/ack are arrays of MSCCL_FLAG_WORDS words: with warp flags (Simple protocol) warp w
-  // of the sender and warp w of the receiver own word w (reading R18); block-level protocols
-  // wait on word 0 and post every word.
+  // send connection (peer = receiver): FIFO and head counter live in the PEER's region; the
+  // FIFO is the region of this program's protocol (each protocol has its own slots).
   char* sendFifo;             // peer FIFO base for (me -> peer, chan); nullptr if no send peer
   uint64_t* sendHead;         // peer: messages posted by me
   uint64_t* sendAck;          // mine: messages the peer consumed (written by the peer)
-  uint64_t* sendCnt;          // mine: persistent count of messages I posted
+  uint64_t* sendCnt;          // mine: [0] messages I posted, [1] launches on this connection
+  uint64_t* sendReady;        // mine: [0] receiver's launch ordinal, [1..3] its in/out/sc refs
   // receive connection (peer = sender)
   char* recvFifo;             // my FIFO base for (peer -> me, chan)
   uint64_t* recvHead;         // mine: messages the peer posted (written by the peer)
   uint64_t* recvAck;          // peer: messages I consumed
-  uint64_t* recvCnt;          // mine: persistent count of messages I consumed
+  uint64_t* recvCnt;          // mine: [0] messages I consumed, [1] launches on this connection
+  uint64_t* recvReady;        // peer: the sender's ready line for this connection (I write it)
 };
+static_assert(sizeof(DevTB) % 16 == 0, "DevTB is staged with 16-byte loads");
 
 struct RankArgs {
   const DevTB* tbs;
@@ -61,6 +65,14 @@ struct RankArgs {
   int32_t ctaStart;           // first CTA of this rank in the grid
   uint32_t* abortFlag;        // this rank's abort word (device memory of its region)
   uint32_t* hostAbort;        // this rank's host-mapped pinned word (watchdog report)
+  // cross-launch direct placement (reading R15b): how a sender reaches this rank's in/out/sc
+  // in this call (raw pointer, MSCCL_REF_REG|idx<<40|offset, or 0 = not reachable), the mask of
+  // buffers whose direct receives are honoured, and this rank's table of peers' registered
+  // buffers mapped into this process: regMap[peer * regMax + idx]
+  uint64_t bufRef[3];
+  char* const* regMap;
+  int32_t regMax;
+  int32_t directMask;
 };
 
 struct KernelArgs {
@@ -76,20 +88,15 @@ struct KernelArgs {
   int32_t proto;              // 0 Simple, 1 LL
   int64_t slotBytes;
   int32_t sysScope;           // 1 when any peer is another GPU
-  int32_t useTma;             // Simple protocol: bulk-copy (TMA) pipeline through shared memory
-  int32_t direct;             // honour DI_*_DIRECT flags (all ranks in this launch, rank == slot)
-  int32_t warpFlags;          // Simple protocol: per-warp head/ack flags, no block barrier per message (R18)
-  int32_t prefetch;           // Simple protocol: bulk L2 prefetch of the local operand before a receive wait
-  int32_t directHints;        // bit 0: terminal direct sends store L2 evict_first; bit 1: a direct
-                              // forward demotes the lines it read to evict_normal (cache hints)
-  uint64_t timeoutNs;
+  // direct placement (reading R15): 0 off; 1 every rank is in this launch (rank == slot);
+  // 2 cross-launch (ranks in other launches / processes, ready handshake per connection)
+  int32_t direct;
+  int32_t directHints;        // bit 0: terminal direct sends store L2 evict_first (cache hint)
+  int32_t pad0;
+  uint64_t timeoutNs;         // device watchdog; 0 = disabled
   uint64_t* trace;            // MSCCL_TRACE builds: per-CTA phase times (ns), else null
-  // CTA c runs thread block ctaMap[c] & 4095 of local rank ctaMap[c] >> 12 (work-balanced
-  // placement: the thread blocks that move the most bytes get the lowest block indices, which
-  // the hardware spreads over distinct SMs first); ctaMapN == 0: rank by prefix sums
-  int32_t ctaMapN;
-  uint16_t ctaMap[MSCCL_CTA_MAP];
 };
 static_assert(sizeof(KernelArgs) <= 4096, "kernel parameter space");
+static_assert(sizeof(KernelArgs) % 4 == 0, "KernelArgs is staged as 32-bit words");
 
 }  // namespace msccl

@@ -235,13 +235,10 @@ __device__ __forceinline__ void stRelaxedGpu(uint64_t* p, uint64_t v) {
 }
 __device__ __forceinline__ void fenceSys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
 __device__ __forceinline__ void fenceGpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
-// store v to every flag word of a connection counter (block-level protocols, DevTB comment)
-__device__ __forceinline__ void postWords(uint64_t* p, uint64_t v, bool sys) {
-#pragma unroll
-  for (int k = 0; k < MSCCL_FLAG_WORDS; k++) {
-    if (sys) stRelaxedSys(p + k, v);
-    else stRelaxedGpu(p + k, v);
-  }
+// post a connection counter (one u64 word in its own 128-byte line)
+__device__ __forceinline__ void postFlag(uint64_t* p, uint64_t v, bool sys) {
+  if (sys) stRelaxedSys(p, v);
+  else stRelaxedGpu(p, v);
 }
 __device__ __forceinline__ uint64_t globaltimer() {
   uint64_t t;
@@ -250,19 +247,21 @@ __device__ __forceinline__ uint64_t globaltimer() {
 }
 
 // ------------------------------------------------------------------ watchdog + waits
-struct TmaState;  // tma_pipe.cuh (MSCCL_ENABLE_TMA builds)
 struct Ctx {
   const KernelArgs* a;
   const RankArgs* ra;
   int tid, nt;
-  TmaState* tma;  // shared-memory pipeline state (Simple protocol with TMA), or null
-  uint64_t sent0; // messages posted on the send connection before this launch
-  // credit cache of the send connection (LL / LL128): every ack word is known to be >= ackKnown
+  // credit cache of the send connection (LL / LL128): the ack word is known to be >= ackKnown
   // (the receiver has consumed that many messages), so a send whose slot was freed by then
-  // needs no flag read; uniform over the block. sAck: the 16 words seen by the waiting threads.
+  // needs no flag read; uniform over the block. sAck: the ack value seen by the waiting thread.
   mutable uint64_t ackKnown;
   uint64_t* sAck;
-  uint64_t* tl;   // MSCCL_TIMELINE builds: this CTA's timeline words, else null
+  // direct placement (reading R15): the send peer's in/out/scratch base pointers in this
+  // address space (shared memory; null = not reachable in this launch), and whether this
+  // launch's ready handshake has been done (cross-launch mode; uniform over the block)
+  char** peerDst;
+  mutable bool readyDone;
+  uint64_t sendL;  // thread 32: this launch's ordinal on the send connection
 };
 
 static __device__ __noinline__ void raiseAbort(const KernelArgs& a) {
@@ -281,7 +280,7 @@ __device__ __forceinline__ bool waitGE(const uint64_t* p, uint64_t target, bool 
     if ((seen = (sys ? ldAcquireSys(p) : ldAcquireGpu(p))) >= target) return true;
     if ((it & 1023u) == 0) {
       if (*(volatile uint32_t*)c.ra->abortFlag) return false;
-      if (globaltimer() - t0 > c.a->timeoutNs) {
+      if (c.a->timeoutNs && globaltimer() - t0 > c.a->timeoutNs) {
         raiseAbort(*c.a);
         return false;
       }
@@ -299,16 +298,6 @@ __device__ __forceinline__ bool waitGE(const uint64_t* p, uint64_t target, bool 
 __device__ __forceinline__ bool waitDep(const RankArgs& ra, uint64_t dep, uint64_t gen, int t, const Ctx& c) {
   const int dtb = (int)(dep >> 48), dstep = (int)((dep >> 32) & 0xffff);
   const uint64_t dn = (uint32_t)dep;  // steps of thread block dtb
-#if MSCCL_TIMELINE
-  if (c.tl && c.tid == 0) {
-    const uint64_t target = (gen << 40) | ((uint64_t)t * dn + (uint64_t)dstep + 1);
-    const uint64_t v0 = ldAcquireGpu(&ra.sem[dtb]);
-    c.tl[27] = globaltimer();
-    c.tl[28] = v0 >= target ? 1 : 0;
-    c.tl[29] = v0;
-    c.tl[30] = target;
-  }
-#endif
   return waitGE(&ra.sem[dtb], (gen << 40) | ((uint64_t)t * dn + (uint64_t)dstep + 1), false, c);
 }
 
@@ -330,12 +319,6 @@ __device__ __forceinline__ void chunkSpan(const KernelArgs& a, int buf, int64_t 
 // written to dst (DST) and/or the outgoing slot (SEND).
 #ifndef MSCCL_TRACE
 #define MSCCL_TRACE 0
-#endif
-#ifndef MSCCL_TIMELINE
-#define MSCCL_TIMELINE 0
-#endif
-#ifndef MSCCL_FENCE_MODE
-#define MSCCL_FENCE_MODE 0
 #endif
 #ifndef MSCCL_POST_LAST_WARP
 #define MSCCL_POST_LAST_WARP 1
@@ -443,13 +426,6 @@ __device__ __forceinline__ void pieceSimple(int64_t m, const char* rslot, const 
   }
 }
 
-#ifndef MSCCL_ENABLE_TMA
-#define MSCCL_ENABLE_TMA 0
-#endif
-#if MSCCL_ENABLE_TMA
-#include "tma_pipe.cuh"
-#endif
-
 // ------------------------------------------------------------------ LL-protocol piece
 // Payload travels in 8-byte units inside 16-byte lines {lo32, flag, hi32, flag}.
 // user-buffer units for LL128 (not concurrently written by peers): plain cached accesses
@@ -522,7 +498,7 @@ __device__ __forceinline__ bool pieceLL(int64_t m, int64_t sendUnits, const char
             if (l.y == rflag && l.w == rflag) break;
             if ((it & 1023u) == 0) {
               if (*(volatile uint32_t*)c.ra->abortFlag) { ok = false; break; }
-              if (globaltimer() - t0 > c.a->timeoutNs) { raiseAbort(*c.a); ok = false; break; }
+              if (c.a->timeoutNs && globaltimer() - t0 > c.a->timeoutNs) { raiseAbort(*c.a); ok = false; break; }
             }
           }
           if (!ok) break;
@@ -603,7 +579,7 @@ __device__ __forceinline__ bool ll128Batch(int64_t base, int64_t bytes, int64_t 
         uint64_t now = globaltimer();
         if (t0 == 0) t0 = now;
         if (*(volatile uint32_t*)c.ra->abortFlag) return false;
-        if (now - t0 > c.a->timeoutNs) {
+        if (c.a->timeoutNs && now - t0 > c.a->timeoutNs) {
           raiseAbort(*c.a);
           return false;
         }
@@ -703,30 +679,48 @@ __device__ __forceinline__ int64_t pieceGeom(const Ctx& c, const DevInstr& in, i
   return hi - a0;
 }
 
-// Bulk L2 prefetch (the TMA engine, no registers) of the local operand of an instruction that
-// is about to wait for its incoming message: the HBM reads of the source tile overlap the
-// wait instead of following it. Issued by one thread; purely a cache hint.
-template <int DT, bool SRC, bool DST, bool REDDST>
-__device__ __noinline__ void prefetchLocal(const Ctx& c, const DevInstr& in, int t) {
-  MSCCL_PIECE_GEOM
-  (void)a0;
-  for (int j = 0; j < in.cnt; j++) {
-    const char* src;
-    char* dst;
-    const int64_t m = pieceGeom<DT, SRC, DST, REDDST>(c, in, t, j, src, dst);
-    const char* p = SRC ? src : dst;
-    if (m * w < 16 || (((uintptr_t)p) & 15)) continue;
-    const uint32_t bytes = (uint32_t)((m * w) & ~(int64_t)15);
-    asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;" ::"l"(p), "r"(bytes) : "memory");
+// Cross-launch direct placement (a.direct == 2, reading R15b): before its first direct store of
+// a launch, the sender's thread 32 waits until the receiving thread block of THIS launch has
+// published its destination references on the connection's ready line (so the receiver's
+// stream has finished every earlier use of that buffer), then resolves them into pointers of
+// this process (raw pointer for single-process communicators, registered-buffer table entry
+// for CUDA IPC peers). A zero reference means "not reachable": the connection falls back to
+// the FIFO for this launch, and the receiver (which published the zero) does the same.
+__device__ __forceinline__ char* resolveRef(const RankArgs& ra, int peer, uint64_t ref) {
+  if (ref == 0) return nullptr;
+  if (!(ref & MSCCL_REF_REG)) return (char*)ref;  // raw pointer (one address space)
+  const uint32_t idx = (uint32_t)((ref >> 40) & 0x7fffffu);
+  const uint64_t off = ref & ((1ull << 40) - 1);
+  if (idx >= (uint32_t)ra.regMax) return nullptr;
+  char* base = ra.regMap[(size_t)peer * ra.regMax + idx];
+  return base ? base + off : nullptr;
+}
+
+__device__ __forceinline__ bool waitReady(const Ctx& c, const DevTB& tb) {
+  uint64_t seen;
+  if (!waitGE(tb.sendReady, c.sendL, c.a->sysScope != 0, c, seen)) return false;
+#pragma unroll
+  for (int b = 0; b < 3; b++) {
+    const uint64_t ref = *(volatile const uint64_t*)(tb.sendReady + 1 + b);
+    c.peerDst[b] = resolveRef(*c.ra, tb.sendPeer, ref);
   }
+  return true;
+}
+
+// is this send / receive a direct placement in this launch (reading R15)?
+__device__ __forceinline__ bool sendIsDirect(const Ctx& c, const DevInstr& in) {
+  return (in.flags & DI_SEND_DIRECT) && c.a->direct && (c.a->direct == 1 || c.peerDst[in.rdstBuf] != nullptr);
+}
+__device__ __forceinline__ bool recvIsDirect(const Ctx& c, const DevInstr& in) {
+  return (in.flags & DI_RECV_DIRECT) && c.a->direct && ((c.ra->directMask >> in.dstBuf) & 1);
 }
 
 template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
 __device__ __noinline__ void movePiecesSimple(const Ctx& c, const DevTB& tb, const DevInstr& in, int t,
                                               const char* rslot, char* sslot) {
   MSCCL_PIECE_GEOM
-  const bool sdirect = SEND && a.direct && (in.flags & DI_SEND_DIRECT);
-  const bool rdirect = RECV && a.direct && (in.flags & DI_RECV_DIRECT);
+  const bool sdirect = SEND && sendIsDirect(c, in);
+  const bool rdirect = RECV && recvIsDirect(c, in);
   for (int j = 0; j < in.cnt; j++) {
     const char* src;
     char* dst;
@@ -735,7 +729,7 @@ __device__ __noinline__ void movePiecesSimple(const Ctx& c, const DevTB& tb, con
     if (sdirect) {  // reading R15: write straight into the receiver's destination chunk
       int64_t rs, rl;
       chunkSpan(a, in.rdstBuf, (int64_t)in.rdstOff + j, rs, rl);
-      so = a.rank[tb.sendPeer].buf[in.rdstBuf] + (rs + a0) * w;
+      so = c.peerDst[in.rdstBuf] + (rs + a0) * w;
       if (rl - a0 < m) m = rl - a0;
     }
     if (m <= 0) continue;
@@ -784,195 +778,34 @@ __device__ __noinline__ bool movePiecesLL128(const Ctx& c, const DevInstr& in, i
   return ok;
 }
 
-#if MSCCL_ENABLE_TMA
-// TMA path; returns false (nothing moved) when a piece is not 16-byte aligned
-template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
-__device__ __noinline__ bool movePiecesTma(const Ctx& c, const DevInstr& in, int t, const char* rslot, char* sslot) {
-  MSCCL_PIECE_GEOM
-  (void)a0;
-  constexpr int MAXP = 8;
-  if (in.cnt > MAXP) return false;
-  TmaPiece ps[MAXP];
-  int64_t ms[MAXP];
-  bool aligned = true;
-  for (int j = 0; j < in.cnt; j++) {
-    const char* src;
-    char* dst;
-    int64_t m = pieceGeom<DT, SRC, DST, REDDST>(c, in, t, j, src, dst);
-    m = m > 0 ? m : 0;
-    ms[j] = m;
-    TmaPiece& p = ps[j];
-    p.inA = RECV ? rslot + j * a.T * w : (REDDST ? dst : src);
-    p.inB = (RECV && SRC) || REDDST ? src : nullptr;
-    p.out0 = DST ? dst : nullptr;
-    p.out1 = SEND ? sslot + j * a.T * w : nullptr;
-    p.bytes = (m * w) & ~(int64_t)15;
-    uintptr_t al = (uintptr_t)p.inA | (uintptr_t)p.inB | (uintptr_t)p.out0 | (uintptr_t)p.out1;
-    if (m > 0 && (al & 15)) aligned = false;
-  }
-  if (!aligned) return false;
-  tmaMessage<DT, OP, (RECV && SRC) || REDDST, MAXP>(*c.tma, ps, in.cnt, RECV, c.tid, c.nt);
-  for (int j = 0; j < in.cnt; j++) {  // < 16-byte tails of ragged pieces
-    const int64_t e0 = ps[j].bytes / w;
-    if (e0 >= ms[j]) continue;
-    const int64_t k = e0 * w;
-    const char* srcp = (RECV && SRC) || REDDST ? ps[j].inB : ps[j].inA;
-    pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(
-        ms[j] - e0, RECV ? ps[j].inA + k : nullptr, SRC ? srcp + k : nullptr,
-        (DST || REDDST) ? (REDDST ? (char*)ps[j].inA : ps[j].out0) + k : nullptr, SEND ? ps[j].out1 + k : nullptr, c.tid,
-        c.nt);
-  }
-  return true;
-}
-
-#endif  // MSCCL_ENABLE_TMA
-
-// ------------------------------------------------------------------ warp flags (reading R18)
-// Simple protocol without a block barrier per message. A piece of a tile (T elements) is cut
-// into nw contiguous byte ranges of P = ceil(T*w/nw) rounded up to 1 KiB (32 lanes x 32
-// bytes); warp w of every thread block moves range w of every piece, and head/ack word w of a
-// connection carries only warp w's progress. Sender warp w and receiver warp w therefore
-// form their own pipeline: a warp starts on its part of a message as soon as the upstream
-// warp with the same index has posted it, and the other warps on the SM keep the memory
-// system busy while it waits. The partition depends only on (T, nw), fixed for a launch:
-// every message that passes through a slot during a launch is cut the same way (so word w's
-// ack frees exactly the bytes sender warp w overwrites), and the program-order hazards of one
-// thread block (an instruction reading what an earlier one wrote, same chunk and tile) stay
-// inside one warp. A slot whose previous message belongs to an earlier launch (possibly cut
-// differently) is reused only when every word has acknowledged it.
-template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
-__device__ __noinline__ void movePiecesWarp(const Ctx& c, const DevTB& tb, const DevInstr& in, int t,
-                                            const char* rslot, char* sslot) {
-  MSCCL_PIECE_GEOM
-  const int lane = c.tid & 31, warp = c.tid >> 5, nw = c.nt >> 5;
-  const int64_t P = ((a.T * w + nw - 1) / nw + 1023) / 1024 * 1024;
-  const int64_t lo = (int64_t)warp * P;
-  if (lo >= (a.E - a0 < a.T ? a.E - a0 : a.T) * w) return;  // beyond tile t of a full chunk
-  const int64_t hiw = lo + P;
-  const bool sdirect = SEND && a.direct && (in.flags & DI_SEND_DIRECT);
-  const bool rdirect = RECV && a.direct && (in.flags & DI_RECV_DIRECT);
-  for (int j = 0; j < in.cnt; j++) {
-    const char* src;
-    char* dst;
-    int64_t m = pieceGeom<DT, SRC, DST, REDDST>(c, in, t, j, src, dst);
-    char* so = SEND ? sslot + j * a.T * w : nullptr;
-    if (sdirect) {  // reading R15: write straight into the receiver's destination chunk
-      int64_t rs, rl;
-      chunkSpan(a, in.rdstBuf, (int64_t)in.rdstOff + j, rs, rl);
-      so = a.rank[tb.sendPeer].buf[in.rdstBuf] + (rs + a0) * w;
-      if (rl - a0 < m) m = rl - a0;
-    }
-    const int64_t hi = hiw < m * w ? hiw : m * w;
-    if (hi <= lo) continue;
-    const int64_t mw = (hi - lo) / w;
-    if (rdirect) {  // the data is already in dst (the sender wrote it there)
-      if (SEND) pieceSimple<DT, OP, false, true, true, false, false>(mw, nullptr, dst + lo, nullptr, so + lo, lane, 32);
-      continue;
-    }
-    pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(mw, RECV ? rslot + j * a.T * w + lo : nullptr,
-                                                      SRC ? src + lo : nullptr, (DST || REDDST) ? dst + lo : nullptr,
-                                                      SEND ? so + lo : nullptr, lane, 32);
-  }
-}
-
-template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
-__device__ __noinline__ bool runOpWarp(const Ctx& c, const DevTB& tb, const DevInstr& in, int t, uint64_t& sent,
-                                       uint64_t& recvd) {
-  const KernelArgs& a = *c.a;
-  const int lane = c.tid & 31, warp = c.tid >> 5;
-  const bool sys = a.sysScope != 0;
-  bool ok = true;
-  if constexpr (RECV && (SRC || REDDST)) {
-    if (a.prefetch && c.tid == 32) prefetchLocal<DT, SRC, DST, REDDST>(c, in, t);
-  }
-  if (RECV && lane == 0) ok = waitGE(tb.recvHead + warp, recvd + 1, sys, c);
-  // a free slot for this warp's part (a direct message uses none, reading R15): the slot's
-  // previous message must be consumed -- by receiver warp w if this launch posted it, by every
-  // receiver warp if an earlier launch did (lanes 0..15 wait on one word each)
-  if (SEND && sent + 1 > (uint64_t)a.slots && !(a.direct && (in.flags & DI_SEND_DIRECT))) {
-    const uint64_t target = sent + 1 - (uint64_t)a.slots;
-    if (target > c.sent0) {
-      if (lane == 0) ok = ok && waitGE(tb.sendAck + warp, target, sys, c);
-    } else if (lane < MSCCL_FLAG_WORDS) {
-      ok = ok && waitGE(tb.sendAck + lane, target, sys, c);
-    }
-  }
-  if (!__all_sync(0xffffffffu, ok)) return false;
-  __syncwarp();  // lane 0's acquire orders the other lanes' reads (bar.warp.sync is a memory barrier among the warp)
-  const char* rslot = RECV ? tb.recvFifo + (int64_t)(recvd % (uint64_t)a.slots) * a.slotBytes : nullptr;
-  char* sslot = SEND ? tb.sendFifo + (int64_t)(sent % (uint64_t)a.slots) * a.slotBytes : nullptr;
-  movePiecesWarp<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, tb, in, t, rslot, sslot);
-  if (RECV || SEND) {
-    __syncwarp();
-    if (lane == 0) {  // release: this warp's stores (and consumed reads) before its flag words
-      if (sys) fenceSys();
-      else fenceGpu();
-      if (SEND) {
-        if (sys) stRelaxedSys(tb.sendHead + warp, sent + 1);
-        else stRelaxedGpu(tb.sendHead + warp, sent + 1);
-      }
-      if (RECV) {
-        if (sys) stRelaxedSys(tb.recvAck + warp, recvd + 1);
-        else stRelaxedGpu(tb.recvAck + warp, recvd + 1);
-      }
-    }
-  }
-  if (SEND) sent++;
-  if (RECV) recvd++;
-  return true;
-}
-
-template <int DT, int OP>
-__device__ __forceinline__ bool dispatchWarp(const Ctx& c, const DevTB& tb, const DevInstr& in, int t, uint64_t& sent,
-                                             uint64_t& recvd) {
-  switch (in.op) {
-    case K_SEND: return runOpWarp<DT, OP, false, true, true, false, false>(c, tb, in, t, sent, recvd);
-    case K_RECV: return runOpWarp<DT, OP, true, false, false, true, false>(c, tb, in, t, sent, recvd);
-    case K_COPY: return runOpWarp<DT, OP, false, false, true, true, false>(c, tb, in, t, sent, recvd);
-    case K_RCS: return runOpWarp<DT, OP, true, true, false, true, false>(c, tb, in, t, sent, recvd);
-    default: break;
-  }
-  if (OP != R_COPY) {
-    switch (in.op) {
-      case K_REDUCE: return runOpWarp<DT, OP, false, false, true, true, true>(c, tb, in, t, sent, recvd);
-      case K_RRC: return runOpWarp<DT, OP, true, false, true, true, false>(c, tb, in, t, sent, recvd);
-      case K_RRS: return runOpWarp<DT, OP, true, true, true, false, false>(c, tb, in, t, sent, recvd);
-      case K_RRCS: return runOpWarp<DT, OP, true, true, true, true, false>(c, tb, in, t, sent, recvd);
-      default: break;
-    }
-  }
-  return true;  // nop
-}
-
 // ------------------------------------------------------------------ one instruction, one tile
 template <int DT, int OP, int PROTO, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
 __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr& in, int t, uint64_t& sent,
                                    uint64_t& recvd, volatile int* sAbort) {
   const KernelArgs& a = *c.a;
-  const RankArgs& ra = *c.ra;
   constexpr bool ll = PROTO != 0;  // LL / LL128: the flags travel inside the data lines
   bool ok = true;
   const bool sys = a.sysScope != 0;  // virtual ranks on one GPU only need gpu-scope ordering
 #if MSCCL_TRACE
   uint64_t tr0 = c.tid == 0 ? globaltimer() : 0, tr1 = 0, tr2 = 0, tr3 = 0, tr4 = 0;
 #endif
-  if constexpr (!ll && RECV && (SRC || REDDST)) {
-    if (a.prefetch && c.tid == 64) prefetchLocal<DT, SRC, DST, REDDST>(c, in, t);
-  }
   if (RECV && !ll && c.tid == 0) ok = waitGE(tb.recvHead, recvd + 1, sys, c);
 #if MSCCL_TRACE
   if (c.tid == 0) tr1 = globaltimer();
 #endif
   // a free slot: at most `slots` messages posted and not yet consumed (§6.1)
   // (a direct message uses no slot: no credit needed, reading R15)
-  // (every ack word: a warp-flag launch before this one may have acknowledged word by word)
   // LL / LL128: credits already seen (c.ackKnown) are not re-read, so a step that has its slot
   // (no head to wait for: the flags travel in the lines) starts moving data without a flag
   // round trip or barrier. Simple keeps the per-message check (it needs the barrier anyway).
   if constexpr (!ll) {
-    if (SEND && c.tid >= 32 && c.tid < 32 + MSCCL_FLAG_WORDS && sent + 1 > (uint64_t)a.slots &&
-        !(a.direct && (in.flags & DI_SEND_DIRECT)))
-      ok = ok && waitGE(tb.sendAck + (c.tid - 32), sent + 1 - (uint64_t)a.slots, sys, c);
+    if (SEND && a.direct == 2 && (in.flags & DI_SEND_DIRECT) && !c.readyDone) {
+      if (c.tid == 32) ok = waitReady(c, tb);  // first direct store of this launch on this connection
+      __syncthreads();                         // c.peerDst visible to every thread
+      c.readyDone = true;
+    }
+    if (SEND && c.tid == 32 && sent + 1 > (uint64_t)a.slots && !sendIsDirect(c, in))
+      ok = ok && waitGE(tb.sendAck, sent + 1 - (uint64_t)a.slots, sys, c);
     if (!ok) *sAbort = 1;
     if (RECV || SEND) {
       __syncthreads();
@@ -981,19 +814,16 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
   } else {
     const uint64_t need = sent + 1 > (uint64_t)a.slots ? sent + 1 - (uint64_t)a.slots : 0;
     const bool creditWait = SEND && need > c.ackKnown;
-    if (creditWait && c.tid >= 32 && c.tid < 32 + MSCCL_FLAG_WORDS) {
+    if (creditWait && c.tid == 32) {
       uint64_t seen = 0;
-      ok = ok && waitGE(tb.sendAck + (c.tid - 32), need, sys, c, seen);
-      c.sAck[c.tid - 32] = seen;
+      ok = ok && waitGE(tb.sendAck, need, sys, c, seen);
+      *c.sAck = seen;
     }
     if (!ok) *sAbort = 1;
     if (creditWait) {
       __syncthreads();
       if (*sAbort) return false;
-      uint64_t mn = c.sAck[0];
-#pragma unroll
-      for (int k = 1; k < MSCCL_FLAG_WORDS; k++) mn = c.sAck[k] < mn ? c.sAck[k] : mn;
-      c.ackKnown = mn;
+      c.ackKnown = *c.sAck;
     }
   }
 #if MSCCL_TRACE
@@ -1003,10 +833,7 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
   char* sslot = SEND ? tb.sendFifo + (int64_t)(sent % (uint64_t)a.slots) * a.slotBytes : nullptr;
   // each protocol's data path is its own non-inlined function (separate register allocation)
   if constexpr (!ll || (!RECV && !SEND)) {
-#if MSCCL_ENABLE_TMA
-    if (c.tma == nullptr || !movePiecesTma<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, in, t, rslot, sslot))
-#endif
-      movePiecesSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, tb, in, t, rslot, sslot);
+    movePiecesSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, tb, in, t, rslot, sslot);
   } else if constexpr (PROTO == 2) {
     if (!movePiecesLL128<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, in, t, rslot, sslot, recvd + 1, sent + 1)) *sAbort = 1;
   } else {
@@ -1020,16 +847,15 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
 #if MSCCL_TRACE
   if (c.tid == 0) tr4 = globaltimer();
 #endif
-  // block-level protocols post every flag word (a later warp-flag launch waits on its own word)
   if (c.tid == 0 && ll && RECV) {  // LL/LL128: data carried its own flags; the ack frees the slot
-    postWords(tb.recvAck, recvd + 1, sys);
+    postFlag(tb.recvAck, recvd + 1, sys);
   } else if (c.tid == (MSCCL_POST_LAST_WARP ? c.nt - 32 : 0) && (RECV || SEND) && !ll) {
     // Simple: lane 0 of the last warp posts, so thread 0 (the head poller) goes straight to the
     // next step's wait and the fence latency overlaps it (option MSCCL_POST_LAST_WARP)
     if (sys) fenceSys();
     else fenceGpu();
-    if (SEND) postWords(tb.sendHead, sent + 1, sys);
-    if (RECV) postWords(tb.recvAck, recvd + 1, sys);
+    if (SEND) postFlag(tb.sendHead, sent + 1, sys);
+    if (RECV) postFlag(tb.recvAck, recvd + 1, sys);
   }
 #if MSCCL_TRACE
   if (c.tid == 0 && a.trace) {
@@ -1090,7 +916,7 @@ struct ChainSmem {
   int64_t dl;
 };
 template <int DT, int OP, int BATCH>
-__device__ __noinline__ void chainExec(const Ctx& c, const DevInstr* mem, int L, int t, ChainSmem& cs, uint64_t* tl) {
+__device__ __noinline__ void chainExec(const Ctx& c, const DevInstr* mem, int L, int t, ChainSmem& cs) {
   typedef typename DType<DT>::T T;
   const KernelArgs& a = *c.a;
   const RankArgs& ra = *c.ra;
@@ -1136,9 +962,6 @@ __device__ __noinline__ void chainExec(const Ctx& c, const DevInstr* mem, int L,
     if (m > 0) {
       const int64_t bytes = m * w;
       const int64_t nvec = (al & 15) ? 0 : bytes / 16;
-#if MSCCL_TIMELINE
-      if (tl && c.tid == 0) tl[17] = globaltimer();
-#endif
       // operands of a vector are loaded in batches before they are folded (in program order),
       // so a chain costs about one memory round trip per batch, not one per member
       const char* first = headCopy ? cs.src[0] : dst;
@@ -1230,54 +1053,33 @@ __device__ __noinline__ void chainExecSimple(const Ctx& c, const DevInstr* mem, 
 }
 
 
-#ifndef MSCCL_MAX_THREADS
-#define MSCCL_MAX_THREADS 512
+#ifndef MSCCL_MIN_BLOCKS
+#define MSCCL_MIN_BLOCKS (512 / MSCCL_MAX_THREADS)
 #endif
 #ifndef MSCCL_SMEM_INSTR
 #define MSCCL_SMEM_INSTR 64  // instructions per thread block staged in shared memory (LL / LL128)
 #endif
 
 template <int DT, int OP, int PROTO>
-__global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const __grid_constant__ KernelArgs aParam) {
+__global__ void __launch_bounds__(MSCCL_MAX_THREADS, MSCCL_MIN_BLOCKS) mscclInterpreter(const __grid_constant__ KernelArgs aParam) {
   __shared__ int sAbort;
   // The launch arguments (all ranks' base pointers and tables, geometry) are copied from the
   // parameter bank into shared memory by all threads at once: every later access is a shared
-  // load instead of a (serialised, on first touch) constant-cache miss. The CTA map stays in
-  // the parameter bank (one entry per CTA).
-  // (latency protocols only: kLat. The Simple kernels keep the HEAD-of-round layout -- these
-  // prologue changes measured -6 % on the Simple ring and buy nothing at bandwidth sizes.)
+  // load instead of a (serialised, on first touch) constant-cache miss.
+  // (latency protocols only: kLat. The Simple kernels keep the arguments in the parameter
+  // bank -- this prologue measured -6 % on the Simple ring and buys nothing at bandwidth sizes.)
   constexpr bool kLat = PROTO != 0;
-  constexpr int kArgWords = kLat ? (int)(offsetof(KernelArgs, ctaMap) / 4) : 1;
+  constexpr int kArgWords = kLat ? (int)(sizeof(KernelArgs) / 4) : 1;
   __shared__ __align__(16) uint32_t sArgs[kArgWords];
   if constexpr (kLat) {
     for (int i = threadIdx.x; i < kArgWords; i += blockDim.x) sArgs[i] = reinterpret_cast<const uint32_t*>(&aParam)[i];
     __syncthreads();
   }
   const KernelArgs& a = kLat ? *reinterpret_cast<const KernelArgs*>(sArgs) : aParam;
-#if MSCCL_ENABLE_TMA
-  __shared__ TmaState sTma;
-  extern __shared__ __align__(128) uint8_t dynSmem[];
-#endif
-#if MSCCL_TIMELINE
-  // latency timeline (debug builds): [0] entry, [1] prologue done, [2 + s] end of step s
-  // (s < 10), [13]/[14] a fused chain's dependency waits / data pass done, [15] exit, [16]
-  // thread 0's own dependency wait done, [17] chain operand setup done, [18 + s] end of step
-  // s of the second tile; %globaltimer, thread 0, last launch wins
-  uint64_t* tl = a.trace ? a.trace + (size_t)blockIdx.x * 32 : nullptr;
-  if (tl && threadIdx.x == 0) tl[0] = globaltimer();
-#else
-  uint64_t* const tl = nullptr;
-#endif
-  int ls = 0, tbi;
-  if (a.ctaMapN) {  // work-balanced placement chosen by the host
-    const uint32_t e = aParam.ctaMap[blockIdx.x];
-    ls = (int)(e >> 12);
-    tbi = (int)(e & 4095u);
-  } else {
-    for (int r = 1; r < a.nLocal; r++)
-      if ((int)blockIdx.x >= a.rank[r].ctaStart) ls = r;
-    tbi = (int)blockIdx.x - a.rank[ls].ctaStart;
-  }
+  int ls = 0;
+  for (int r = 1; r < a.nLocal; r++)
+    if ((int)blockIdx.x >= a.rank[r].ctaStart) ls = r;
+  const int tbi = (int)blockIdx.x - a.rank[ls].ctaStart;
   const RankArgs& ra = a.rank[ls];
   if (tbi >= ra.nTB) return;
   // Prologue: the thread block's descriptor and instruction list are staged in
@@ -1295,114 +1097,82 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
       reinterpret_cast<uint4*>(sIns)[i] = reinterpret_cast<const uint4*>(ins)[i];
     ins = sIns;
   }
-  Ctx c{&a, &ra, (int)threadIdx.x, (int)blockDim.x, nullptr, 0, 0, nullptr, tl};
-#if MSCCL_ENABLE_TMA
-  if (a.useTma && PROTO == 0) {
-    c.tma = &sTma;
-    if (threadIdx.x == 0) {
-      sTma.A = dynSmem;
-      sTma.B = dynSmem + TMA_NST * TMA_CB;
-      sTma.full = reinterpret_cast<uint64_t*>(dynSmem + 2 * TMA_NST * TMA_CB);
-      sTma.comp = sTma.full + TMA_NST;
-      sTma.gc = 0;
-      for (int i = 0; i < TMA_NST; i++) {
-        mbarInit(&sTma.full[i], 1);
-        mbarInit(&sTma.comp[i], blockDim.x / 32 - 1);
-      }
-      // make the initialised barriers visible to the async proxy (TMA complete_tx)
-      asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-  }
-#endif
-  if (threadIdx.x == 0) sAbort = 0;
-  __shared__ uint64_t sAck[MSCCL_FLAG_WORDS];
+  __shared__ uint64_t sAck;
+  __shared__ char* sPeerDst[3];
   __shared__ ChainSmem sChain;
-  c.sAck = sAck;
-  c.ackKnown = 0;
+  Ctx c{&a, &ra, (int)threadIdx.x, (int)blockDim.x, 0, &sAck, sPeerDst, false, 0};
+  if (threadIdx.x == 0) {
+    sAbort = 0;
+    // one-launch direct placement: the send peer is local rank tb.sendPeer of this launch
+    for (int b = 0; b < 3; b++)
+      sPeerDst[b] = (a.direct == 1 && tb.sendPeer >= 0) ? a.rank[tb.sendPeer].buf[b] : nullptr;
+  }
   uint64_t sent = tb.sendFifo ? *(volatile uint64_t*)tb.sendCnt : 0;
-  c.sent0 = sent;
   uint64_t recvd = tb.recvFifo ? *(volatile uint64_t*)tb.recvCnt : 0;
   const uint64_t gen = *(volatile uint64_t*)&ra.gen[tbi];
-  // warp flags (R18): a warp whose wait failed (watchdog / abort) keeps walking the program
-  // without doing anything, so the block-wide barriers below still match; at the next one
-  // every thread sees sAbort and returns.
-  const bool warpMode = PROTO == 0 && a.warpFlags;
+  // Launch ordinals per connection (word 1 of the persistent counter lines) stay in lock-step
+  // on both ends in every launch; in cross-launch direct mode the receiving thread block also
+  // publishes where its destinations are (reading R15b), released by one fence.
+  if (threadIdx.x == 32 && tb.sendFifo) {
+    c.sendL = *(volatile uint64_t*)(tb.sendCnt + 1) + 1;
+    *(volatile uint64_t*)(tb.sendCnt + 1) = c.sendL;
+  }
+  if (threadIdx.x == 0 && tb.recvFifo) {
+    const uint64_t L = *(volatile uint64_t*)(tb.recvCnt + 1) + 1;
+    *(volatile uint64_t*)(tb.recvCnt + 1) = L;
+    if (a.direct == 2) {
+      for (int b = 0; b < 3; b++) postFlag(tb.recvReady + 1 + b, ra.bufRef[b], a.sysScope != 0);
+      if (a.sysScope) fenceSys();
+      else fenceGpu();
+      postFlag(tb.recvReady, L, a.sysScope != 0);
+    }
+  }
   // semaphore posts (fence + store) by lane 0 of the last warp: thread 0 polls the next step's
   // head / dependencies meanwhile; every post follows a block barrier (option MSCCL_POST_LAST_WARP)
   const int kPoster = MSCCL_POST_LAST_WARP ? (int)blockDim.x - 32 : 0;
-  bool dead = false;
   __syncthreads();
-#if MSCCL_TIMELINE
-  if (tl && threadIdx.x == 0) tl[1] = globaltimer();
-#endif
   for (int t = 0; t < a.I; t++) {
     for (int s = 0; s < tb.nSteps; s++) {
       const DevInstr in = ins[s];
       if constexpr (OP != R_COPY) {
         if (in.flags & DI_CHAIN_HEAD) {  // reading R16: fused local reduce chain
+          const int L = in.chainLen;
+          bool ok = true;
           if constexpr (PROTO == 0) {
-            const int L = in.chainLen;
-            bool ok = true;
             for (int k = 0; k < L && ok; k++) {  // all members' dependencies first
               const DevInstr& mk = ins[s + k];
               for (int d = c.tid; d < mk.nDeps && ok; d += c.nt) ok = waitDep(ra, ra.deps[mk.depStart + d], gen, t, c);
             }
-            if (!ok) sAbort = 1;
-            __syncthreads();
-            if (sAbort) return;
-            chainExecSimple<DT, OP>(c, ins + s, L, t);
-            __syncthreads();
-            s += L - 1;
-            if (ins[s].hasDep && c.tid == kPoster) {
-              fenceGpu();
-              stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)tb.nSteps + (uint64_t)s + 1));
-            }
           } else {
-            const int L = in.chainLen;
-            bool ok = true;
-            // all members' dependencies first: flattened dependency f goes to thread f mod nt; a
-            // thread first collects its dependency words, then waits on all of them, so the waits
-            // of different members overlap (waiting inside the member loop serialises them: one
-            // member per loop trip)
-            {
-              constexpr int KD = 4;
-              uint64_t mine[KD];
-              int nm = 0;
-              for (int k = 0, base = 0; k < L; k++) {
-                const DevInstr& mk = ins[s + k];
-                for (int d = ((c.tid - base) % c.nt + c.nt) % c.nt; d < mk.nDeps; d += c.nt) {
-                  const uint64_t dw = ra.deps[mk.depStart + d];
-                  if (nm < KD) mine[nm++] = dw;
-                  else ok = ok && waitDep(ra, dw, gen, t, c);  // more than KD per thread: in order
-                }
-                base += mk.nDeps;
+            // flattened dependency f goes to thread f mod nt; a thread first collects its
+            // dependency words, then waits on all of them, so the waits of different members
+            // overlap (waiting inside the member loop serialises them: one member per loop trip)
+            constexpr int KD = 4;
+            uint64_t mine[KD];
+            int nm = 0;
+            for (int k = 0, base = 0; k < L; k++) {
+              const DevInstr& mk = ins[s + k];
+              for (int d = ((c.tid - base) % c.nt + c.nt) % c.nt; d < mk.nDeps; d += c.nt) {
+                const uint64_t dw = ra.deps[mk.depStart + d];
+                if (nm < KD) mine[nm++] = dw;
+                else ok = ok && waitDep(ra, dw, gen, t, c);  // more than KD per thread: in order
               }
+              base += mk.nDeps;
+            }
 #pragma unroll
-              for (int i = 0; i < KD; i++)
-                if (i < nm) ok = ok && waitDep(ra, mine[i], gen, t, c);
-            }
-#if MSCCL_TIMELINE
-            if (tl && c.tid == 0) tl[16] = globaltimer();
-#endif
-            if (!ok) sAbort = 1;
-            __syncthreads();
-            if (sAbort) return;
-#if MSCCL_TIMELINE
-            if (tl && c.tid == 0) tl[13] = globaltimer();
-#endif
-            chainExec<DT, OP, PROTO == 1 ? 8 : 2>(c, ins + s, L, t, sChain, tl);
-            __syncthreads();
-#if MSCCL_TIMELINE
-            if (tl && c.tid == 0) tl[14] = globaltimer();
-#endif
-            s += L - 1;
-            if (ins[s].hasDep && c.tid == kPoster) {
-              fenceGpu();
-              stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)tb.nSteps + (uint64_t)s + 1));
-            }
-#if MSCCL_TIMELINE
-            if (tl && c.tid == 0 && s < 10 && t < 2) tl[(t ? 18 : 2) + s] = globaltimer();
-#endif
+            for (int i = 0; i < KD; i++)
+              if (i < nm) ok = ok && waitDep(ra, mine[i], gen, t, c);
+          }
+          if (!ok) sAbort = 1;
+          __syncthreads();
+          if (sAbort) return;
+          if constexpr (PROTO == 0) chainExecSimple<DT, OP>(c, ins + s, L, t);
+          else chainExec<DT, OP, PROTO == 1 ? 8 : 2>(c, ins + s, L, t, sChain);
+          __syncthreads();
+          s += L - 1;
+          if (ins[s].hasDep && c.tid == kPoster) {
+            fenceGpu();
+            stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)tb.nSteps + (uint64_t)s + 1));
           }
           continue;
         }
@@ -1414,53 +1184,19 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, 1) mscclInterpreter(const _
         __syncthreads();
         if (sAbort) return;
       }
-      if constexpr (PROTO == 0) {
-        if (warpMode) {
-          if (!dead && *(volatile int*)&sAbort) dead = true;
-          if (!dead && !dispatchWarp<DT, OP>(c, tb, in, t, sent, recvd)) {
-            dead = true;
-            sAbort = 1;
-          }
-          if (in.hasDep) {  // every warp's part of the step is done before the semaphore moves
-            __syncthreads();
-            if (sAbort) return;
-          }
-        } else if (!dispatch<DT, OP, PROTO>(c, tb, in, t, sent, recvd, &sAbort)) {
-          return;
-        }
-      } else {
-        if (!dispatch<DT, OP, PROTO>(c, tb, in, t, sent, recvd, &sAbort)) return;
-      }
+      if (!dispatch<DT, OP, PROTO>(c, tb, in, t, sent, recvd, &sAbort)) return;
       if (in.hasDep) {  // Fig. 5 lines 25-27: the step is complete before the semaphore moves
         if (c.tid == kPoster) {
           fenceGpu();
           stRelaxedGpu(&ra.sem[tbi], (gen << 40) | ((uint64_t)t * (uint64_t)tb.nSteps + (uint64_t)s + 1));
         }
       }
-#if MSCCL_TIMELINE
-      if (tl && threadIdx.x == 0 && s < 10 && t < 2) tl[(t ? 18 : 2) + s] = globaltimer();
-#endif
     }
   }
-  if (warpMode) {
-    __syncthreads();
-    if (sAbort) return;
-  }
-  if (threadIdx.x == 0) {
+  if (threadIdx.x == 0) {  // epilogue: persist the connection counters and the generation
     if (tb.sendFifo) *(volatile uint64_t*)tb.sendCnt = sent;
-    if (tb.recvFifo) {
-      *(volatile uint64_t*)tb.recvCnt = recvd;
-      // words no warp of this launch owned: everything received is consumed (a later launch
-      // with more warps waits on them)
-      for (int k = blockDim.x >> 5; k < MSCCL_FLAG_WORDS; k++) {
-        if (a.sysScope) stRelaxedSys(tb.recvAck + k, recvd);
-        else stRelaxedGpu(tb.recvAck + k, recvd);
-      }
-    }
+    if (tb.recvFifo) *(volatile uint64_t*)tb.recvCnt = recvd;
     *(volatile uint64_t*)&ra.gen[tbi] = gen + 1;
-#if MSCCL_TIMELINE
-    if (tl) tl[15] = globaltimer();
-#endif
   }
 }
 

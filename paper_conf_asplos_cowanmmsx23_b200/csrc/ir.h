@@ -69,6 +69,8 @@ Algo parseIR(const char* text, size_t len);  // throws IRError (rule V1)
 
 // Throws IRError("Vn: ...") on the first violated rule (V1..V9).
 void validateIR(Algo& a, int nranks, int slots, int maxTbs, int maxChannels, int iters = 2);
+// V9 alone at a given pipeline depth (the launch's real I); throws IRError("V9: ...").
+void deadlockCheckIR(const Algo& a, int slots, int iters);
 
 // Direct placement analysis (reading R15). For rank `rank`: recvDirect[tb][step] = the
 // receive may find its data already in its destination (op r / rcs whose destination

@@ -4,5 +4,4 @@
 namespace msccl {
 const void* interpreterKernel(int dtype, int op, int proto);  // op 0..3 sum/prod/max/min; proto 0 Simple 1 LL 2 LL128
 const void* copyKernel(int elemBytes, int proto);             // programs with no reduction
-int tmaSmemBytes();  // dynamic shared memory of the TMA pipeline (0 when not compiled in)
 }  // namespace msccl

@@ -1,5 +1,6 @@
 // Host runtime behind include/msccl.h: communicators, shared regions, program loading,
 // program selection by size range (MSCCLang §6), geometry, launch.
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -10,6 +11,7 @@
 #include <map>
 #include <memory>
 #include <mutex>
+#include <set>
 #include <sstream>
 #include <string>
 #include <tuple>
@@ -25,9 +27,11 @@ using namespace msccl;
 // ------------------------------------------------------------------ parameters
 namespace {
 
+// Library defaults = the tuned configuration: 4 x 256 KiB Simple slots, 256
+// threads per CTA (2 CTAs per SM), direct placement on. LL / LL128 have their own FIFO slots.
 struct Params {
-  int64_t slots = 4, slotBytes = 262144, maxChannels = 32, threads = 512, timeoutS = 20, tma = 0, direct = 1,
-          warp = 0, l2PersistMiB = 0, prefetch = 0, directTile = 1, balance = 0, directHints = 1;
+  int64_t slots = 4, slotBytes = 262144, llSlotBytes = 65536, ll128SlotBytes = 262144, maxChannels = 32,
+          threads = 256, timeoutS = 60, direct = 1, directTile = 1, directHints = 1, regMax = 64;
 };
 
 std::mutex gMu;
@@ -39,16 +43,14 @@ std::atomic<uint64_t> gLaunches{0};
 int64_t* paramRef(Params& p, const std::string& k) {
   if (k == "MSCCL_SLOTS") return &p.slots;
   if (k == "MSCCL_SLOT_BYTES") return &p.slotBytes;
+  if (k == "MSCCL_LL_SLOT_BYTES") return &p.llSlotBytes;
+  if (k == "MSCCL_LL128_SLOT_BYTES") return &p.ll128SlotBytes;
+  if (k == "MSCCL_MAX_REGISTRATIONS") return &p.regMax;
   if (k == "MSCCL_MAX_CHANNELS") return &p.maxChannels;
   if (k == "MSCCL_THREADS") return &p.threads;
   if (k == "MSCCL_TIMEOUT_S") return &p.timeoutS;
-  if (k == "MSCCL_TMA") return &p.tma;
   if (k == "MSCCL_DIRECT") return &p.direct;
-  if (k == "MSCCL_WARP_FLAGS") return &p.warp;
-  if (k == "MSCCL_L2_PERSIST_MIB") return &p.l2PersistMiB;
-  if (k == "MSCCL_PREFETCH") return &p.prefetch;
   if (k == "MSCCL_DIRECT_TILE") return &p.directTile;
-  if (k == "MSCCL_BALANCE") return &p.balance;
   if (k == "MSCCL_DIRECT_HINTS") return &p.directHints;
   return nullptr;
 }
@@ -57,10 +59,9 @@ Params currentParams() {
   std::lock_guard<std::mutex> g(gMu);
   if (!gEnvRead) {
     gEnvRead = true;
-    for (const char* k : {"MSCCL_SLOTS", "MSCCL_SLOT_BYTES", "MSCCL_MAX_CHANNELS", "MSCCL_THREADS", "MSCCL_TIMEOUT_S",
-                          "MSCCL_TMA", "MSCCL_DIRECT", "MSCCL_WARP_FLAGS",
-                          "MSCCL_L2_PERSIST_MIB", "MSCCL_PREFETCH", "MSCCL_DIRECT_TILE",
-                          "MSCCL_BALANCE", "MSCCL_DIRECT_HINTS"}) {
+    for (const char* k : {"MSCCL_SLOTS", "MSCCL_SLOT_BYTES", "MSCCL_LL_SLOT_BYTES", "MSCCL_LL128_SLOT_BYTES",
+                          "MSCCL_MAX_CHANNELS", "MSCCL_THREADS", "MSCCL_TIMEOUT_S", "MSCCL_DIRECT",
+                          "MSCCL_DIRECT_TILE", "MSCCL_DIRECT_HINTS", "MSCCL_MAX_REGISTRATIONS"}) {
       const char* v = getenv(k);
       if (v && *v) *paramRef(gParams, k) = atoll(v);
     }
@@ -87,6 +88,20 @@ struct Clique {  // ranks created together by mscclCommInitAll
 
 struct mscclProgram;
 
+// A registered user buffer (reading R15b): peers of a CUDA-IPC communicator can place messages
+// straight into it. Registration index = position in the comm's table (same on every rank when
+// every rank registers in the same order, but each rank publishes its own index anyway).
+struct mscclReg {
+  mscclComm* comm = nullptr;
+  int idx = -1;
+  char* base = nullptr;      // registered range [base, base + size) in this process
+  size_t size = 0;
+  bool connected = false;    // mscclRegConnect done: every peer's matching buffer is mapped
+  char* allocBase = nullptr;  // the device allocation holding the range (what CUDA IPC exports)
+  std::vector<char*> peerMapped;  // IPC mappings this rank uses for peers' buffer `idx` (allocation bases)
+  std::vector<std::pair<int, std::string>> peerKeys;  // their ipcCache entries
+};
+
 struct mscclComm {
   int nranks = 0, rank = 0, dev = 0;
   Params prm;
@@ -103,16 +118,31 @@ struct mscclComm {
   std::vector<mscclProgram*> programs;
   std::string lastError;
   int maxCoResident = 0;
+  std::vector<mscclReg*> regs;         // by index (nullptr = free)
+  char** dRegMap = nullptr;            // device [nranks][regMax]: peers' registered buffers, mapped here
+  std::vector<char*> hRegMap;
+  // opened peer allocations (CUDA IPC handles can be opened once per process): refcounted
+  std::map<std::pair<int, std::string>, std::pair<char*, int>> ipcCache;
 
-  // region layout
-  size_t fifoOff(int src, int ch) const {
-    return ((size_t)src * prm.maxChannels + ch) * prm.slots * prm.slotBytes;
+  // region layout: one receiver-side FIFO per protocol (Simple, LL, LL128), each
+  // [src rank][channel][slot] x that protocol's slot bytes, then the flag lines
+  int64_t protoSlotBytes(int proto) const {
+    return proto == PROTO_LL ? prm.llSlotBytes : proto == PROTO_LL128 ? prm.ll128SlotBytes : prm.slotBytes;
   }
-  // kind: 0 head, 1 ack, 2 sendCnt, 3 recvCnt; MSCCL_FLAG_WORDS words (one 128-byte line) each
+  size_t fifoBase(int proto) const {
+    size_t off = 0;
+    for (int p = 0; p < proto; p++) off += (size_t)nranks * prm.maxChannels * prm.slots * protoSlotBytes(p);
+    return off;
+  }
+  size_t fifoOff(int proto, int src, int ch) const {
+    return fifoBase(proto) + ((size_t)src * prm.maxChannels + ch) * prm.slots * protoSlotBytes(proto);
+  }
+  // kind: 0 head, 1 ack, 2 sendCnt, 3 recvCnt, 4 ready (line of the SENDER's region, written by
+  // the receiver); one 128-byte line each
   size_t flagOff(int kind, int peer, int ch) const {
-    return flagsOff + (((size_t)kind * nranks + peer) * prm.maxChannels + ch) * MSCCL_FLAG_WORDS * sizeof(uint64_t);
+    return flagsOff + (((size_t)kind * nranks + peer) * prm.maxChannels + ch) * MSCCL_FLAG_STRIDE * sizeof(uint64_t);
   }
-  size_t abortOff() const { return flagOff(4, 0, 0); }
+  size_t abortOff() const { return flagOff(5, 0, 0); }
 };
 
 struct mscclProgram {
@@ -127,11 +157,11 @@ struct mscclProgram {
   uint64_t* dSem = nullptr;  // nTB sems followed by nTB gens
   char* dScratch = nullptr;
   size_t scratchBytes = 0;
+  std::vector<char*> retiredScratch;  // outgrown scratch buffers: a captured graph may still use them
   int maxCnt = 1;
   bool hasReduce = false;
   bool allDirect = true;  // every message of this rank's program is a direct placement (R15)
-  std::vector<int64_t> tbWork;        // chunk-sized operand touches per thread block (FIFO protocol)
-  std::vector<int64_t> tbWorkDirect;  // ... with direct placement (R15)
+  std::set<int> v9Iters;  // pipeline depths I at which V9 (deadlock freedom) has been verified
 };
 
 namespace {
@@ -167,19 +197,25 @@ struct DeviceGuard {
 mscclResult_t allocRegion(mscclComm* c) {
   c->prm = currentParams();
   if (c->prm.slots < 1 || c->prm.slots > 16) return setErr(c, mscclInvalidArgument, "MSCCL_SLOTS must be in 1..16");
-  if (c->prm.slotBytes < 4096 || c->prm.slotBytes % 256) return setErr(c, mscclInvalidArgument, "MSCCL_SLOT_BYTES must be a multiple of 256, >= 4096");
-  if (c->prm.threads < 64 || c->prm.threads > 512 || c->prm.threads % 32) return setErr(c, mscclInvalidArgument, "MSCCL_THREADS must be a multiple of 32 in 64..512");
+  for (int64_t b : {c->prm.slotBytes, c->prm.llSlotBytes, c->prm.ll128SlotBytes})
+    if (b < 4096 || b % 256)
+      return setErr(c, mscclInvalidArgument, "MSCCL_SLOT_BYTES / MSCCL_LL_SLOT_BYTES / MSCCL_LL128_SLOT_BYTES must be multiples of 256, >= 4096");
+  if (c->prm.threads < 64 || c->prm.threads > MSCCL_MAX_THREADS || c->prm.threads % 32) {
+    std::ostringstream o;
+    o << "MSCCL_THREADS must be a multiple of 32 in 64.." << MSCCL_MAX_THREADS;
+    return setErr(c, mscclInvalidArgument, o.str());
+  }
   if (c->prm.maxChannels < 1 || c->prm.maxChannels > 1024) return setErr(c, mscclInvalidArgument, "MSCCL_MAX_CHANNELS out of range");
+  if (c->prm.regMax < 1 || c->prm.regMax > (1 << 20)) return setErr(c, mscclInvalidArgument, "MSCCL_MAX_REGISTRATIONS out of range");
   DeviceGuard g(c->dev);
-  c->fifoBytes = (size_t)c->nranks * c->prm.maxChannels * c->prm.slots * c->prm.slotBytes;
+  c->fifoBytes = c->fifoBase(3);
   c->flagsOff = c->fifoBytes;
   c->regionBytes = c->abortOff() + 256;
   CUDACHECK(c, cudaMalloc(&c->region, c->regionBytes));
   CUDACHECK(c, cudaMemset(c->region, 0, c->regionBytes));
-  // optional L2 set-aside for evict_last (persisting) lines: the FIFO slot stores carry
-  // L2::evict_last, which only has a reserved home when the set-aside is non-zero
-  if (c->prm.l2PersistMiB > 0)
-    CUDACHECK(c, cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, (size_t)c->prm.l2PersistMiB << 20));
+  c->hRegMap.assign((size_t)c->nranks * c->prm.regMax, nullptr);
+  CUDACHECK(c, cudaMalloc(&c->dRegMap, c->hRegMap.size() * sizeof(char*)));
+  CUDACHECK(c, cudaMemset(c->dRegMap, 0, c->hRegMap.size() * sizeof(char*)));
   CUDACHECK(c, cudaHostAlloc(&c->hostAbort, sizeof(uint32_t), cudaHostAllocMapped | cudaHostAllocPortable));
   *c->hostAbort = 0;
   CUDACHECK(c, cudaHostGetDevicePointer((void**)&c->hostAbortDev, c->hostAbort, 0));
@@ -201,6 +237,7 @@ void freeProgram(mscclProgram* p) {
   cudaFree(p->dDeps);
   cudaFree(p->dSem);
   cudaFree(p->dScratch);
+  for (char* x : p->retiredScratch) cudaFree(x);
   delete p;
 }
 
@@ -241,6 +278,23 @@ mscclResult_t coResident(mscclComm* c, const void* fn, int threads, int smem, in
   return mscclSuccess;
 }
 
+// drop a registration: unpublish it and close the peer mappings nobody else uses
+void releaseReg(mscclComm* c, mscclReg* r) {
+  for (auto& k : r->peerKeys) {
+    auto it = c->ipcCache.find(k);
+    if (it != c->ipcCache.end() && --it->second.second == 0) {
+      cudaIpcCloseMemHandle(it->second.first);
+      c->ipcCache.erase(it);
+    }
+  }
+  if (r->idx >= 0 && r->idx < (int)c->regs.size()) {
+    c->regs[r->idx] = nullptr;
+    for (int p = 0; p < c->nranks; p++) c->hRegMap[(size_t)p * c->prm.regMax + r->idx] = nullptr;
+    cudaMemcpy(c->dRegMap, c->hRegMap.data(), c->hRegMap.size() * sizeof(char*), cudaMemcpyHostToDevice);
+  }
+  delete r;
+}
+
 // ------------------------------------------------------------------ groups and launches
 struct Call {
   mscclComm* comm;
@@ -249,6 +303,7 @@ struct Call {
   int dtype, op;
   int64_t n;
   cudaStream_t stream;
+  bool aliased;  // in-place call of an out-of-place (aliassafe) program: no direct placement
 };
 
 thread_local int tGroupDepth = 0;
@@ -270,10 +325,11 @@ mscclResult_t geometry(mscclComm* c, const mscclProgram* p, int dtype, int64_t n
   int64_t e = (n + g.cb - 1) / g.cb;
   g.E = (e + V - 1) / V * V;
   int64_t t;
+  const int64_t sb = c->protoSlotBytes(p->algo.proto);
   if (p->algo.proto == PROTO_LL128)  // whole 128-byte lines (120 payload bytes) per piece
-    t = (c->prm.slotBytes / 128 / p->maxCnt) * 120 / w / V * V;
+    t = (sb / 128 / p->maxCnt) * 120 / w / V * V;
   else
-    t = (p->algo.proto == PROTO_LL ? c->prm.slotBytes / 2 : c->prm.slotBytes) / ((int64_t)p->maxCnt * w) / V * V;
+    t = (p->algo.proto == PROTO_LL ? sb / 2 : sb) / ((int64_t)p->maxCnt * w) / V * V;
   if (t < V) return setErr(c, mscclInvalidUsage, "FIFO slot too small for the program's largest count");
   if (noFifo) t = g.E;
   g.T = std::min<int64_t>(t, g.E);
@@ -281,17 +337,55 @@ mscclResult_t geometry(mscclComm* c, const mscclProgram* p, int dtype, int64_t n
   return mscclSuccess;
 }
 
-mscclResult_t ensureScratch(mscclComm* c, mscclProgram* p, size_t bytes) {
+// Scratch (SURVEY §8(b) Ownership): pre-sized at mscclLoadProgram for the program's maxBytes,
+// so calls inside that size range never allocate and can be captured in a CUDA graph. A
+// program loaded without a maxBytes grows its scratch on the first (uncaptured) call that needs
+// more; the outgrown buffer is kept until the program is unloaded, because kernels already
+// queued, or graphs captured earlier, still reference it. No host synchronisation either way.
+mscclResult_t ensureScratch(mscclComm* c, mscclProgram* p, size_t bytes, cudaStream_t stream) {
   if (bytes <= p->scratchBytes) return mscclSuccess;
+  cudaStreamCaptureStatus cs = cudaStreamCaptureStatusNone;
+  CUDACHECK(c, cudaStreamIsCapturing(stream, &cs));
+  if (cs != cudaStreamCaptureStatusNone) {
+    std::ostringstream o;
+    o << "program '" << p->algo.name << "' needs " << bytes << " bytes of scratch but has " << p->scratchBytes
+      << " while the stream is being captured: load it with maxBytes covering this call (scratch is then "
+         "pre-sized) or run one uncaptured call of this size first";
+    return setErr(c, mscclInvalidUsage, o.str());
+  }
   DeviceGuard dg(c->dev);
-  CUDACHECK(c, cudaDeviceSynchronize());  // growing scratch: the old one may be in use
-  cudaFree(p->dScratch);
-  p->dScratch = nullptr;
-  p->scratchBytes = 0;
   size_t sz = (bytes + 4095) / 4096 * 4096;
-  CUDACHECK(c, cudaMalloc(&p->dScratch, sz));
+  char* nb = nullptr;
+  CUDACHECK(c, cudaMalloc(&nb, sz));
+  if (p->dScratch) p->retiredScratch.push_back(p->dScratch);
+  p->dScratch = nb;
   p->scratchBytes = sz;
   return mscclSuccess;
+}
+
+// V9 at the launch's real pipeline depth: the loader checked
+// 2 iterations; the first call with a deeper pipeline re-runs the abstract machine with I
+// iterations and the program remembers the verdict per I.
+mscclResult_t checkDepth(mscclComm* c, mscclProgram* p, int I) {
+  if (I <= 2 || p->v9Iters.count(I)) return mscclSuccess;
+  try {
+    deadlockCheckIR(p->algo, (int)c->prm.slots, I);
+  } catch (const IRError& e) {
+    return setErr(c, mscclInvalidProgram, std::string(e.what()) + " (pipeline depth I=" + std::to_string(I) + ")");
+  }
+  p->v9Iters.insert(I);
+  return mscclSuccess;
+}
+
+// how a sender reaches [p, p+bytes) of rank c in this call (reading R15b): a raw pointer when
+// every rank lives in this process (peer access / virtual ranks), else a registered buffer
+uint64_t bufferRef(mscclComm* c, const char* p, size_t bytes) {
+  if (!p) return 0;
+  if (c->clique) return (uint64_t)(uintptr_t)p;
+  for (auto* r : c->regs)
+    if (r && r->connected && p >= r->base && p + bytes <= r->base + r->size)
+      return MSCCL_REF_REG | ((uint64_t)r->idx << 40) | (uint64_t)(p - r->base);
+  return 0;
 }
 
 mscclResult_t launchCalls(std::vector<Call>& calls) {
@@ -303,6 +397,12 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
     std::sort(v.begin(), v.end(), [](Call* a, Call* b) { return a->comm->rank < b->comm->rank; });
     mscclComm* c0 = v[0]->comm;
     if ((int)v.size() > MSCCL_MAX_LOCAL) return setErr(c0, mscclInvalidUsage, "too many ranks on one device");
+    // one call per communicator per launch: two calls on one comm would share its connection
+    // counters, semaphores and FIFOs inside one grid (NCCL aggregates such calls; here it is an error)
+    for (size_t i = 1; i < v.size(); i++)
+      if (v[i]->comm == v[i - 1]->comm || v[i]->comm->rank == v[i - 1]->comm->rank)
+        return setErr(v[i]->comm, mscclInvalidUsage,
+                      "two collectives on one communicator (or rank) inside one mscclGroupStart/End");
     if (c0->clique) {
       int onDev = 0;
       for (auto* cm : c0->clique->comms)
@@ -317,11 +417,19 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
         return setErr(cl->comm, mscclInvalidUsage, "ranks in a group disagree on program/count/datatype/op");
     }
     mscclProgram* p0 = v[0]->prog;
-    // direct placement needs every rank's buffers in this launch (rank r at slot r) and the
-    // Simple protocol; one launch covering all ranks also orders it against earlier launches
-    const bool useTma = p0->algo.proto == PROTO_SIMPLE && c0->prm.tma && tmaSmemBytes() > 0;
-    const bool direct = p0->algo.proto == PROTO_SIMPLE && c0->prm.direct && (int)v.size() == p0->algo.ngpus && !useTma;
-    bool noFifo = direct && c0->prm.directTile;
+    const int R = p0->algo.ngpus;
+    // Direct placement (reading R15) needs the Simple protocol. Mode 1: every rank 0..R-1 of the
+    // program is in this launch exactly once (slot r = rank r), so the sender reaches the
+    // receiver's buffers through this launch's arguments. Mode 2 (reading R15b): some ranks run
+    // in other launches or processes; each connection does a ready handshake per launch.
+    bool allHere = (int)v.size() == R;
+    for (int i = 0; allHere && i < (int)v.size(); i++) allHere = v[i]->comm->rank == i && v[i]->comm->nranks == R;
+    int direct = 0;
+    if (p0->algo.proto == PROTO_SIMPLE && c0->prm.direct) direct = allHere ? 1 : 2;
+    bool aliasedAny = false;
+    for (auto* cl : v) aliasedAny = aliasedAny || cl->aliased;
+    if (direct == 1 && aliasedAny) direct = 0;  // ADVICE: in-place call of an out-of-place program
+    bool noFifo = direct == 1 && c0->prm.directTile;
     for (auto* cl : v) noFifo = noFifo && cl->prog->allDirect;
     Geometry g{};
     mscclResult_t r = geometry(c0, p0, v[0]->dtype, v[0]->n, g, noFifo);
@@ -336,21 +444,26 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
     ka.cb = g.cb;
     ka.slots = (int)c0->prm.slots;
     ka.proto = p0->algo.proto == PROTO_LL ? 1 : (p0->algo.proto == PROTO_LL128 ? 2 : 0);
-    ka.slotBytes = c0->prm.slotBytes;
-    ka.timeoutNs = (uint64_t)c0->prm.timeoutS * 1000000000ull;
+    ka.slotBytes = c0->protoSlotBytes(p0->algo.proto);
+    ka.timeoutNs = c0->prm.timeoutS > 0 ? (uint64_t)c0->prm.timeoutS * 1000000000ull : 0;  // <= 0: no watchdog
     ka.trace = traceBuffer();
+    ka.direct = direct;
+    ka.directHints = (int32_t)c0->prm.directHints;
     int cta = 0;
     for (int i = 0; i < (int)v.size(); i++) {
       Call* cl = v[i];
       mscclProgram* p = cl->prog;
+      r = checkDepth(cl->comm, p, g.I);
+      if (r != mscclSuccess) return r;
       RankArgs& ra = ka.rank[i];
       ra.tbs = p->dTBs;
       ra.instrs = p->dInstr;
       ra.deps = p->dDeps;
       ra.sem = p->dSem;
       ra.gen = p->dSem + p->nTB;
-      size_t need = (size_t)p->algo.gpus[cl->comm->rank].sChunks * g.E * elemBytes(cl->dtype);
-      r = ensureScratch(cl->comm, p, need);
+      const int w = elemBytes(cl->dtype);
+      size_t need = (size_t)p->algo.gpus[cl->comm->rank].sChunks * g.E * w;
+      r = ensureScratch(cl->comm, p, need, cl->stream);
       if (r != mscclSuccess) return r;
       ra.buf[0] = cl->buf[0];
       ra.buf[1] = cl->buf[1];
@@ -359,49 +472,41 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
       ra.ctaStart = cta;
       ra.abortFlag = (uint32_t*)(cl->comm->region + cl->comm->abortOff());
       ra.hostAbort = cl->comm->hostAbortDev;
+      ra.regMap = cl->comm->dRegMap;
+      ra.regMax = (int32_t)cl->comm->prm.regMax;
+      if (direct == 1) {
+        ra.directMask = 7;
+      } else if (direct == 2 && !cl->aliased) {
+        const int Rr = cl->comm->nranks;
+        const size_t bytes[3] = {(size_t)g.n * blocksOf(p->algo.coll, BUF_IN, Rr) * w,
+                                 (size_t)g.n * blocksOf(p->algo.coll, BUF_OUT, Rr) * w, need};
+        for (int b = 0; b < 3; b++) {
+          ra.bufRef[b] = bufferRef(cl->comm, ra.buf[b], bytes[b]);
+          if (ra.bufRef[b]) ra.directMask |= 1 << b;
+        }
+      }
       cta += p->nTB;
       if (cl->comm->sysScope) ka.sysScope = 1;
     }
     if (cta == 0) continue;
-    // work-balanced placement: thread blocks ordered by the bytes they move (heaviest first,
-    // ties by rank then id, so the order is deterministic); block indices are handed to SMs
-    // in increasing order, so the heavy blocks land on distinct SMs before any SM gets two
-    if (c0->prm.balance && cta <= MSCCL_CTA_MAP && (int)v.size() <= 16) {
-      std::vector<std::tuple<int64_t, int, int>> order;
-      for (int i = 0; i < (int)v.size(); i++) {
-        const mscclProgram* p = v[i]->prog;
-        const auto& wk = direct ? p->tbWorkDirect : p->tbWork;
-        for (int t = 0; t < p->nTB; t++) order.emplace_back(-wk[t], i, t);
-      }
-      std::stable_sort(order.begin(), order.end());
-      for (size_t k = 0; k < order.size(); k++)
-        ka.ctaMap[k] = (uint16_t)((std::get<1>(order[k]) << 12) | std::get<2>(order[k]));
-      ka.ctaMapN = (int32_t)order.size();
-    }
     const void* fn = p0->hasReduce ? interpreterKernel(v[0]->dtype, v[0]->op, ka.proto)
                                    : copyKernel(elemBytes(v[0]->dtype), ka.proto);
-    ka.useTma = useTma ? 1 : 0;
-    ka.direct = direct ? 1 : 0;
-    ka.warpFlags = (ka.proto == 0 && c0->prm.warp && !ka.useTma) ? 1 : 0;
-    ka.prefetch = (ka.proto == 0 && c0->prm.prefetch) ? 1 : 0;
-    ka.directHints = (int32_t)c0->prm.directHints;
-    const int smem = ka.useTma ? tmaSmemBytes() : 0;
     int maxCta = 0;
-    r = coResident(c0, fn, (int)c0->prm.threads, smem, maxCta);
+    r = coResident(c0, fn, (int)c0->prm.threads, 0, maxCta);
     if (r != mscclSuccess) return r;
     if (cta > maxCta) {
       std::ostringstream o;
       o << "program needs " << cta << " co-resident CTAs on device " << c0->dev << " but at most " << maxCta
-        << " fit (use fewer instances/channels, or MSCCL_TMA=0 / fewer MSCCL_THREADS for more CTAs per SM)";
+        << " fit (use fewer instances/channels, or fewer MSCCL_THREADS for more CTAs per SM)";
       return setErr(c0, mscclInvalidUsage, o.str());
     }
     DeviceGuard dg(c0->dev);
     void* args[] = {&ka};
     if (debugOn())
-      fprintf(stderr, "[msccl] launch dev %d ranks %d program %s ctas %d threads %d n %lld E %lld T %lld I %d\n",
+      fprintf(stderr, "[msccl] launch dev %d ranks %d program %s ctas %d threads %d n %lld E %lld T %lld I %d direct %d\n",
               c0->dev, ka.nLocal, p0->algo.name.c_str(), cta, (int)c0->prm.threads, (long long)g.n,
-              (long long)g.E, (long long)g.T, g.I);
-    CUDACHECK(c0, cudaLaunchCooperativeKernel(fn, dim3(cta), dim3((unsigned)c0->prm.threads), args, (size_t)smem,
+              (long long)g.E, (long long)g.T, g.I, direct);
+    CUDACHECK(c0, cudaLaunchCooperativeKernel(fn, dim3(cta), dim3((unsigned)c0->prm.threads), args, 0,
                                               v[0]->stream));
     gLaunches++;
   }
@@ -467,6 +572,7 @@ mscclResult_t runColl(mscclProgram* p, int coll, const void* sendbuff, void* rec
   cl.op = op;
   cl.n = (int64_t)count;
   cl.stream = stream;
+  cl.aliased = false;
   if (p->algo.inplace) {
     if (!inplace) {  // reading R8: an in-place program called out of place gets a pre-copy
       DeviceGuard dg(c->dev);
@@ -477,6 +583,7 @@ mscclResult_t runColl(mscclProgram* p, int coll, const void* sendbuff, void* rec
   } else {
     if (inplace && !p->algo.aliassafe)
       return setErr(c, mscclInvalidUsage, "in-place call on an out-of-place program that is not marked aliassafe");
+    cl.aliased = inplace;
     cl.buf[0] = (char*)sb;
     cl.buf[1] = rb;
   }
@@ -596,10 +703,12 @@ mscclResult_t mscclCommExportHandle(mscclComm_t c, void* handle, size_t* bytes) 
   DeviceGuard g(c->dev);
   cudaIpcMemHandle_t h;
   CUDACHECK(c, cudaIpcGetMemHandle(&h, c->region));
-  static_assert(sizeof(h) + 32 <= MSCCL_HANDLE_BYTES, "handle size");
   memcpy(handle, &h, sizeof(h));
   // parameters that both ends of a connection must agree on (region layout, warp partition)
-  int64_t meta[4] = {(int64_t)c->regionBytes, (int64_t)c->dev, c->prm.threads, c->prm.warp};
+  // parameters both ends of a connection must agree on (region layout, slot geometry)
+  int64_t meta[8] = {(int64_t)c->regionBytes, (int64_t)c->dev,     c->prm.threads,        c->prm.slots,
+                     c->prm.slotBytes,         c->prm.llSlotBytes, c->prm.ll128SlotBytes, c->prm.maxChannels};
+  static_assert(sizeof(cudaIpcMemHandle_t) + sizeof(meta) <= MSCCL_HANDLE_BYTES, "handle size");
   memcpy((char*)handle + sizeof(h), meta, sizeof(meta));
   if (bytes) *bytes = MSCCL_HANDLE_BYTES;
   return mscclSuccess;
@@ -614,11 +723,19 @@ mscclResult_t mscclCommConnect(mscclComm_t c, const void* allHandles) {
     const char* h = (const char*)allHandles + (size_t)p * MSCCL_HANDLE_BYTES;
     cudaIpcMemHandle_t ih;
     memcpy(&ih, h, sizeof(ih));
-    int64_t meta[4];
+    int64_t meta[8];
     memcpy(meta, h + sizeof(ih), sizeof(meta));
-    if ((size_t)meta[0] != c->regionBytes) return setErr(c, mscclInvalidUsage, "peer region size differs (ranks use different MSCCL_* parameters)");
-    if (meta[2] != c->prm.threads || meta[3] != c->prm.warp)
-      return setErr(c, mscclInvalidUsage, "peer uses different MSCCL_THREADS / MSCCL_WARP_FLAGS (the warp partition must match)");
+    const int64_t mine[8] = {(int64_t)c->regionBytes, 0,  c->prm.threads,        c->prm.slots,
+                             c->prm.slotBytes,         c->prm.llSlotBytes, c->prm.ll128SlotBytes, c->prm.maxChannels};
+    static const char* names[8] = {"region size", "", "MSCCL_THREADS", "MSCCL_SLOTS", "MSCCL_SLOT_BYTES",
+                                   "MSCCL_LL_SLOT_BYTES", "MSCCL_LL128_SLOT_BYTES", "MSCCL_MAX_CHANNELS"};
+    for (int k = 0; k < 8; k++)
+      if (k != 1 && meta[k] != mine[k]) {
+        std::ostringstream o;
+        o << "rank " << p << " uses a different " << names[k] << " (" << meta[k] << " vs " << mine[k]
+          << "): every rank must use the same MSCCL_* parameters";
+        return setErr(c, mscclInvalidUsage, o.str());
+      }
     void* ptr = nullptr;
     CUDACHECK(c, cudaIpcOpenMemHandle(&ptr, ih, cudaIpcMemLazyEnablePeerAccess));
     c->peerBase[p] = (char*)ptr;
@@ -636,6 +753,10 @@ mscclResult_t mscclCommDestroy(mscclComm_t c) {
     cudaDeviceSynchronize();
     for (auto* p : c->programs) freeProgram(p);
     c->programs.clear();
+    for (auto* r : std::vector<mscclReg*>(c->regs))
+      if (r) releaseReg(c, r);
+    c->regs.clear();
+    cudaFree(c->dRegMap);
     for (int p = 0; p < c->nranks; p++)
       if (c->peerIpc[p]) cudaIpcCloseMemHandle(c->peerBase[p]);
     cudaFree(c->region);
@@ -646,6 +767,145 @@ mscclResult_t mscclCommDestroy(mscclComm_t c) {
     v.erase(std::remove(v.begin(), v.end(), c), v.end());
   }
   delete c;
+  return mscclSuccess;
+}
+
+// ------------------------------------------------------------------ buffer registration (R15b)
+namespace {
+struct RegDesc {  // MSCCL_REG_DESC_BYTES bytes on the wire
+  cudaIpcMemHandle_t h;
+  uint64_t offset;  // registered range start - allocation base
+  uint64_t size;
+  int32_t idx, rank, single, pad;
+};
+static_assert(sizeof(RegDesc) <= MSCCL_REG_DESC_BYTES, "registration descriptor size");
+
+typedef CUresult (*AddrRangeFn)(unsigned long long*, size_t*, unsigned long long);
+}  // namespace
+
+mscclResult_t mscclCommRegister(mscclComm_t c, void* buff, size_t size, mscclReg_t* out) {
+  if (!c || !buff || !size || !out) return setErr(c, mscclInvalidArgument, "mscclCommRegister: null argument or size 0");
+  int idx = -1;
+  for (int i = 0; i < (int)c->prm.regMax && idx < 0; i++)
+    if (i >= (int)c->regs.size() || !c->regs[i]) idx = i;
+  if (idx < 0) return setErr(c, mscclInvalidArgument, "mscclCommRegister: MSCCL_MAX_REGISTRATIONS buffers already registered");
+  // the allocation that holds [buff, buff+size) (CUDA IPC exports whole allocations)
+  static AddrRangeFn addrRange = nullptr;
+  if (!addrRange) {
+    void* fn = nullptr;
+    cudaDriverEntryPointQueryResult q;
+    CUDACHECK(c, cudaGetDriverEntryPoint("cuMemGetAddressRange", &fn, cudaEnableDefault, &q));
+    if (!fn || q != cudaDriverEntryPointSuccess) return setErr(c, mscclSystemError, "cuMemGetAddressRange unavailable");
+    addrRange = (AddrRangeFn)fn;
+  }
+  DeviceGuard g(c->dev);
+  unsigned long long base = 0;
+  size_t asize = 0;
+  if (addrRange(&base, &asize, (unsigned long long)(uintptr_t)buff) != 0 ||
+      (uintptr_t)buff + size > base + asize)
+    return setErr(c, mscclInvalidArgument, "mscclCommRegister: range is not inside one device allocation");
+  mscclReg* r = new mscclReg();
+  r->comm = c;
+  r->idx = idx;
+  r->base = (char*)buff;
+  r->size = size;
+  r->allocBase = (char*)(uintptr_t)base;
+  r->peerMapped.assign(c->nranks, nullptr);
+  if ((int)c->regs.size() <= idx) c->regs.resize(idx + 1, nullptr);
+  c->regs[idx] = r;
+  *out = r;
+  return mscclSuccess;
+}
+
+mscclResult_t mscclRegExport(mscclReg_t r, void* desc) {
+  if (!r || !desc) return setErr(r ? r->comm : nullptr, mscclInvalidArgument, "mscclRegExport: null argument");
+  mscclComm* c = r->comm;
+  RegDesc d;
+  memset(&d, 0, sizeof(d));
+  d.offset = (uint64_t)(r->base - r->allocBase);
+  d.size = r->size;
+  d.idx = r->idx;
+  d.rank = c->rank;
+  d.single = c->clique ? 1 : 0;
+  if (!c->clique) {
+    DeviceGuard g(c->dev);
+    CUDACHECK(c, cudaIpcGetMemHandle(&d.h, r->allocBase));
+  }
+  memset(desc, 0, MSCCL_REG_DESC_BYTES);
+  memcpy(desc, &d, sizeof(d));
+  return mscclSuccess;
+}
+
+mscclResult_t mscclRegConnect(mscclReg_t r, const void* all) {
+  if (!r || !all) return setErr(r ? r->comm : nullptr, mscclInvalidArgument, "mscclRegConnect: null argument");
+  mscclComm* c = r->comm;
+  if (c->clique) {  // one address space: senders use raw pointers, nothing to map
+    r->connected = true;
+    return mscclSuccess;
+  }
+  DeviceGuard g(c->dev);
+  for (int p = 0; p < c->nranks; p++) {
+    if (p == c->rank) continue;
+    RegDesc d;
+    memcpy(&d, (const char*)all + (size_t)p * MSCCL_REG_DESC_BYTES, sizeof(d));
+    if (d.rank != p || d.idx < 0 || d.idx >= c->prm.regMax || d.single)
+      return setErr(c, mscclInvalidArgument, "mscclRegConnect: descriptors are not in rank order / from another kind of communicator");
+    // one mapping per peer allocation (a handle can be opened once per process)
+    std::string key(reinterpret_cast<const char*>(&d.h), sizeof(d.h));
+    auto it = c->ipcCache.find({p, key});
+    char* m = nullptr;
+    if (it != c->ipcCache.end()) {
+      m = it->second.first;
+      it->second.second++;
+    } else {
+      void* ptr = nullptr;
+      CUDACHECK(c, cudaIpcOpenMemHandle(&ptr, d.h, cudaIpcMemLazyEnablePeerAccess));
+      m = (char*)ptr;
+      c->ipcCache[{p, key}] = {m, 1};
+    }
+    r->peerMapped[p] = m;
+    r->peerKeys.push_back({p, key});
+    c->hRegMap[(size_t)p * c->prm.regMax + d.idx] = m + d.offset;
+  }
+  CUDACHECK(c, cudaMemcpy(c->dRegMap, c->hRegMap.data(), c->hRegMap.size() * sizeof(char*), cudaMemcpyHostToDevice));
+  r->connected = true;
+  return mscclSuccess;
+}
+
+mscclResult_t mscclCommDeregister(mscclComm_t c, mscclReg_t r) {
+  if (!c || !r || r->comm != c) return setErr(c, mscclInvalidArgument, "mscclCommDeregister: bad arguments");
+  DeviceGuard g(c->dev);
+  CUDACHECK(c, cudaDeviceSynchronize());  // kernels that may still store into peers' mapped buffers
+  releaseReg(c, r);
+  return mscclSuccess;
+}
+
+// Direct-placement marking of the loader for one rank, for the oracle's race detector.
+mscclResult_t mscclDebugDirectPlacement(const char* ir, size_t irBytes, int rank, int32_t* flags, int32_t* rdst,
+                                        int maxInstr, int* nInstr) {
+  if (!ir || !nInstr) return mscclInvalidArgument;
+  try {
+    Algo a = parseIR(ir, irBytes);
+    Params prm = currentParams();
+    validateIR(a, a.ngpus, (int)prm.slots, 1 << 15, 1 << 20);
+    if (rank < 0 || rank >= a.ngpus) return mscclInvalidArgument;
+    const DirectInfo di = directPlacement(a, rank);
+    const GpuProgram& g = a.gpus[rank];
+    int k = 0;
+    for (size_t t = 0; t < g.tbs.size(); t++)
+      for (size_t s = 0; s < g.tbs[t].steps.size(); s++, k++) {
+        if (k >= maxInstr || !flags) continue;
+        flags[k] = (di.sendDirect[t][s] ? 1 : 0) | (di.recvDirect[t][s] ? 2 : 0);
+        if (rdst) {
+          rdst[2 * k] = di.sendDirect[t][s] ? di.rdstBuf[t][s] : -1;
+          rdst[2 * k + 1] = di.sendDirect[t][s] ? di.rdstOff[t][s] : -1;
+        }
+      }
+    *nInstr = k;
+  } catch (const IRError& e) {
+    setErr(nullptr, mscclInvalidProgram, e.what());
+    return mscclInvalidProgram;
+  }
   return mscclSuccess;
 }
 
@@ -710,8 +970,6 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
   p->nTB = (int)g.tbs.size();
   const DirectInfo dinfo = directPlacement(p->algo, c->rank);
   std::vector<DevTB> tbs(p->nTB);
-  p->tbWork.assign(p->nTB, 0);
-  p->tbWorkDirect.assign(p->nTB, 0);
   std::vector<DevInstr> ins;
   std::vector<uint64_t> deps;
   for (int t = 0; t < p->nTB; t++) {
@@ -722,17 +980,20 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
     d.instrStart = (uint32_t)ins.size();
     d.tbId = tb.id;
     d.sendPeer = tb.send;
+    const int pr = p->algo.proto;
     if (tb.send >= 0) {
-      d.sendFifo = c->peerBase[tb.send] + c->fifoOff(c->rank, tb.chan);
+      d.sendFifo = c->peerBase[tb.send] + c->fifoOff(pr, c->rank, tb.chan);
       d.sendHead = (uint64_t*)(c->peerBase[tb.send] + c->flagOff(0, c->rank, tb.chan));
       d.sendAck = (uint64_t*)(c->region + c->flagOff(1, tb.send, tb.chan));
       d.sendCnt = (uint64_t*)(c->region + c->flagOff(2, tb.send, tb.chan));
+      d.sendReady = (uint64_t*)(c->region + c->flagOff(4, tb.send, tb.chan));
     }
     if (tb.recv >= 0) {
-      d.recvFifo = c->region + c->fifoOff(tb.recv, tb.chan);
+      d.recvFifo = c->region + c->fifoOff(pr, tb.recv, tb.chan);
       d.recvHead = (uint64_t*)(c->region + c->flagOff(0, tb.recv, tb.chan));
       d.recvAck = (uint64_t*)(c->peerBase[tb.recv] + c->flagOff(1, c->rank, tb.chan));
       d.recvCnt = (uint64_t*)(c->region + c->flagOff(3, tb.recv, tb.chan));
+      d.recvReady = (uint64_t*)(c->peerBase[tb.recv] + c->flagOff(4, c->rank, tb.chan));
     }
     for (size_t si = 0; si < tb.steps.size(); si++) {
       const Instr& in = tb.steps[si];
@@ -754,13 +1015,6 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
         deps.push_back(((uint64_t)dp.first << 48) | ((uint64_t)dp.second << 32) |
                        (uint64_t)(uint32_t)g.tbs[dp.first].steps.size());
       if (dinfo.recvDirect[t][si]) di.flags |= DI_RECV_DIRECT;
-      {  // operand touches of this instruction (mscclProgramTouches costs)
-        static const int cost[OP_COUNT] = {0, 2, 2, 2, 3, 3, 3, 4, 3};
-        int cd = cost[in.op];
-        if (dinfo.recvDirect[t][si]) cd = in.op == OP_RCS ? 2 : 0;
-        p->tbWork[t] += (int64_t)cost[in.op] * in.cnt;
-        p->tbWorkDirect[t] += (int64_t)cd * in.cnt;
-      }
       const bool sends = in.op == OP_SEND || in.op == OP_RRS || in.op == OP_RRCS || in.op == OP_RCS;
       if (sends && !dinfo.sendDirect[t][si]) p->allDirect = false;
       if (dinfo.sendDirect[t][si]) {
@@ -817,6 +1071,14 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
   if (!deps.empty()) {
     CUDACHECK(c, cudaMalloc(&p->dDeps, deps.size() * sizeof(uint64_t)));
     CUDACHECK(c, cudaMemcpy(p->dDeps, deps.data(), deps.size() * sizeof(uint64_t), cudaMemcpyHostToDevice));
+  }
+  // scratch pre-sized for the largest call of the size range: every chunk of a
+  // call with count*w < maxBytes has E*w <= maxBytes/cb + 16 bytes (reading R1)
+  if (maxBytes > 0 && g.sChunks > 0) {
+    const int cb = std::max(1, p->algo.gpus[0].iChunks / blocksOf(p->algo.coll, BUF_IN, p->algo.ngpus));
+    const size_t perChunk = maxBytes / cb + 32;
+    p->scratchBytes = ((size_t)g.sChunks * perChunk + 4095) / 4096 * 4096;
+    CUDACHECK(c, cudaMalloc(&p->dScratch, p->scratchBytes));
   }
   p->index = (int)c->programs.size();
   c->programs.push_back(p.get());

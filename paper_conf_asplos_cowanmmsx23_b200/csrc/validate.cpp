@@ -83,6 +83,8 @@ void deadlockCheck(const Algo& a, int slots, int iters) {
 
 }  // namespace
 
+void deadlockCheckIR(const Algo& a, int slots, int iters) { deadlockCheck(a, slots, iters); }
+
 void validateIR(Algo& a, int nranks, int slots, int maxTbs, int maxChannels, int iters) {
   const int R = a.ngpus;
   if (nranks > 0 && R != nranks) {

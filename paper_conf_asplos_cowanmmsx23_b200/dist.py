@@ -32,3 +32,14 @@ def init_from_process_group(device, group=None):
     from .runtime import Comm
     rank, world = dist.get_rank(group), dist.get_world_size(group)
     return connect(Comm.init_rank(world, rank, device), group)
+
+
+def register(comm, tensor, group=None):
+    """Collective buffer registration for direct placement across processes (reading R15b):
+    mscclCommRegister + exchange of the descriptors + mscclRegConnect on every rank, then a
+    barrier so that no rank publishes the buffer before every peer has mapped it."""
+    import torch.distributed as dist
+    reg = comm.register(tensor)
+    reg.connect(exchange_handles(reg.export(), group))
+    dist.barrier(group)
+    return reg

@@ -20,6 +20,7 @@ if not os.path.exists(LIBPATH):
 lib = ctypes.CDLL(LIBPATH)
 
 HANDLE_BYTES = 128
+REG_DESC_BYTES = 128
 RESULTS = {0: "Success", 1: "UnhandledCudaError", 2: "SystemError", 3: "InternalError", 4: "InvalidArgument",
            5: "InvalidUsage", 6: "RemoteError", 7: "InProgress", 8: "InvalidProgram", 9: "NoMatchingProgram"}
 DTYPES = {"int8": 0, "uint8": 1, "int32": 2, "uint32": 3, "int64": 4, "uint64": 5, "float16": 6, "float32": 7,
@@ -55,6 +56,12 @@ SIGNATURES = {
     "mscclSetParam": (_i, [_c.c_char_p, _i64]),
     "mscclGetParam": (_i, [_c.c_char_p, _c.POINTER(_i64)]),
     "mscclLaunchCount": (_c.c_uint64, []),
+    "mscclCommRegister": (_i, [_vp, _vp, _sz, _c.POINTER(_vp)]),
+    "mscclRegExport": (_i, [_vp, _vp]),
+    "mscclRegConnect": (_i, [_vp, _vp]),
+    "mscclCommDeregister": (_i, [_vp, _vp]),
+    "mscclDebugDirectPlacement": (_i, [_c.c_char_p, _sz, _i, _c.POINTER(_c.c_int32), _c.POINTER(_c.c_int32), _i,
+                                       _c.POINTER(_i)]),
 }
 for _name, (_res, _args) in SIGNATURES.items():
     _f = getattr(lib, _name)
@@ -94,6 +101,19 @@ def validate(ir_text, nranks, slots=0, max_tbs=0):
     err = _c.create_string_buffer(1024)
     r = lib.mscclValidateProgram(b, len(b), nranks, slots, max_tbs, err, 1024)
     return r == 0, err.value.decode()
+
+
+def direct_placement(ir_text, rank):
+    """The loader's direct-placement marking for `rank` (mscclDebugDirectPlacement, no GPU):
+    a list, in (thread block, step) order, of (flags, rdst_buf, rdst_chunk) with flags bit 0 =
+    direct send, bit 1 = direct receive (reading R15)."""
+    b = ir_text.encode() if isinstance(ir_text, str) else ir_text
+    n = _i()
+    _check(lib.mscclDebugDirectPlacement(b, len(b), rank, None, None, 0, _c.byref(n)))
+    flags = (_c.c_int32 * max(1, n.value))()
+    rdst = (_c.c_int32 * max(2, 2 * n.value))()
+    _check(lib.mscclDebugDirectPlacement(b, len(b), rank, flags, rdst, n.value, _c.byref(n)))
+    return [(flags[k], rdst[2 * k], rdst[2 * k + 1]) for k in range(n.value)]
 
 
 _TORCH_DT = None
@@ -150,6 +170,27 @@ class Program:
         v = _i64()
         _check(lib.mscclProgramTouches(self.handle, int(direct), _c.byref(v)), self.comm.handle)
         return v.value
+
+
+class Registration:
+    """A registered buffer (mscclReg_t)."""
+
+    def __init__(self, comm, handle):
+        self.comm = comm
+        self.handle = handle
+
+    def export(self):
+        buf = _c.create_string_buffer(REG_DESC_BYTES)
+        _check(lib.mscclRegExport(self.handle, buf), self.comm.handle)
+        return buf.raw
+
+    def connect(self, all_descs):
+        _check(lib.mscclRegConnect(self.handle, b"".join(all_descs)), self.comm.handle)
+
+    def deregister(self):
+        if self.handle:
+            _check(lib.mscclCommDeregister(self.comm.handle, self.handle), self.comm.handle)
+            self.handle = None
 
 
 class Comm:
@@ -213,6 +254,17 @@ class Comm:
 
     def last_error(self):
         return lib.mscclGetLastError(self.handle).decode(errors="replace")
+
+    # --- buffer registration (direct placement across processes, reading R15b)
+    def register(self, tensor_or_ptr, nbytes=None):
+        """mscclCommRegister: returns a Registration; export()/connect() complete it."""
+        if nbytes is None:
+            ptr, nbytes = tensor_or_ptr.data_ptr(), tensor_or_ptr.numel() * tensor_or_ptr.element_size()
+        else:
+            ptr = int(tensor_or_ptr)
+        h = _vp()
+        _check(lib.mscclCommRegister(self.handle, _vp(ptr), nbytes, _c.byref(h)), self.handle)
+        return Registration(self, h)
 
     # --- programs
     def load(self, ir_text, min_bytes=0, max_bytes=0):

@@ -122,7 +122,7 @@ def test_cuda_graph_capture_and_replay(env):
         want = sim.simulate(irparse.parse(algo.to_xml()), xs, n, "bfloat16")
         send = [torch.from_numpy(x.view(np.int16).copy()).cuda().view(torch.bfloat16) for x in xs]
         recv = [torch.empty_like(s) for s in send]
-        _call(runtime, comms, lambda q, c: c.allreduce(send[q], recv[q]))  # warm-up (scratch etc.)
+        _call(runtime, comms, lambda q, c: c.allreduce(send[q], recv[q]))  # warm-up
         torch.cuda.synchronize()
         g = torch.cuda.CUDAGraph()
         with torch.cuda.graph(g):
@@ -134,6 +134,115 @@ def test_cuda_graph_capture_and_replay(env):
             torch.cuda.synchronize()
             for q in range(R):
                 assert np.array_equal(recv[q].view(torch.int16).cpu().numpy().view(np.uint16), want[q])
+    finally:
+        for c, p in zip(comms, ps):
+            c.unload(p)
+
+
+@pytest.mark.parametrize("make", ["allpairs", "oneshot"])
+def test_first_call_of_fresh_program_captured_in_graph(env, make):
+    """SURVEY §8(b) Ownership: a program loaded with maxBytes has its scratch pre-sized, so
+    the FIRST call after mscclLoadProgram can be captured in a CUDA graph (no allocation, no
+    host sync) and the replays are bit-exact with the oracle."""
+    torch, runtime, comms = env
+    algo = P.allpairs_allreduce(R, protocol="Simple") if make == "allpairs" else P.oneshot_allreduce(R, protocol="LL")
+    n = 12289
+    ps = [c.load(algo.to_xml(), 0, 1 << 20) for c in comms]
+    try:
+        xs = synth.inputs(R, n, "float16", "uniform")
+        want = sim.simulate(irparse.parse(algo.to_xml()), xs, n, "float16")
+        send = [torch.from_numpy(x.view(np.int16).copy()).cuda().view(torch.float16) for x in xs]
+        recv = [torch.empty_like(s) for s in send]
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            _call(runtime, comms, lambda q, c: c.allreduce(send[q], recv[q]))
+        for _ in range(2):
+            for r in recv:
+                r.zero_()
+            g.replay()
+            torch.cuda.synchronize()
+            for q in range(R):
+                assert np.array_equal(recv[q].view(torch.int16).cpu().numpy().view(np.uint16), want[q].view(np.uint16))
+    finally:
+        for c, p in zip(comms, ps):
+            c.unload(p)
+
+
+def test_scratch_growth_during_capture_is_refused(env):
+    """A program loaded without maxBytes grows scratch on demand; if that would happen while
+    the stream is being captured the call returns InvalidUsage (nothing is captured), and
+    after one uncaptured call of that size capture works."""
+    torch, runtime, comms = env
+    algo = P.allpairs_allreduce(R, protocol="Simple")
+    ps = [c.load(algo.to_xml()) for c in comms]
+    try:
+        n = 50001
+        xs = synth.inputs(R, n, "float32", "uniform")
+        want = sim.simulate(irparse.parse(algo.to_xml()), xs, n, "float32")
+        send = [torch.from_numpy(x).cuda() for x in xs]
+        recv = [torch.empty_like(s) for s in send]
+        torch.cuda.synchronize()
+        s = torch.cuda.Stream()
+        g = torch.cuda.CUDAGraph()
+        with pytest.raises(runtime.MscclError) as ei:
+            with torch.cuda.graph(g, stream=s):
+                _call(runtime, comms, lambda q, c: c.allreduce(send[q], recv[q]))
+        assert ei.value.code == 5
+        torch.cuda.synchronize()
+        _call(runtime, comms, lambda q, c: c.allreduce(send[q], recv[q]))   # grows scratch
+        torch.cuda.synchronize()
+        g = torch.cuda.CUDAGraph()
+        with torch.cuda.graph(g):
+            _call(runtime, comms, lambda q, c: c.allreduce(send[q], recv[q]))
+        for r in recv:
+            r.zero_()
+        g.replay()
+        torch.cuda.synchronize()
+        for q in range(R):
+            assert np.array_equal(recv[q].cpu().numpy().view(np.uint32), want[q].view(np.uint32))
+    finally:
+        for c, p in zip(comms, ps):
+            c.unload(p)
+
+
+def test_two_calls_on_one_comm_in_one_group_rejected(env):
+    """two collectives on the same communicator inside one group would share its
+    connection counters and semaphores in one grid; the launch is refused."""
+    torch, runtime, comms = env
+    algo = P.ring_allreduce(R)
+    ps = [c.load(algo.to_xml()) for c in comms]
+    try:
+        x = torch.zeros(4096, device="cuda")
+        ys = [torch.zeros(4096, device="cuda") for _ in range(R + 1)]
+        with pytest.raises(runtime.MscclError) as ei:
+            with runtime.group():
+                for q, c in enumerate(comms):
+                    c.allreduce(x, ys[q])
+                comms[0].allreduce(x, ys[R])
+        assert ei.value.code == 5
+    finally:
+        torch.cuda.synchronize()
+        for c, p in zip(comms, ps):
+            c.unload(p)
+
+
+def test_aliassafe_inplace_call_disables_direct_placement(env):
+    """an out-of-place program marked aliassafe may be called in place; the
+    launch then runs without direct placement (its analysis assumes distinct in/out) and the
+    result equals the out-of-place result bit for bit."""
+    torch, runtime, comms = env
+    ir = P.ring_allreduce(R, instances=2).to_xml().replace("<algo ", '<algo aliassafe="1" ', 1)
+    ps = [c.load(ir) for c in comms]
+    try:
+        n = 40000
+        xs = synth.inputs(R, n, "float32", "uniform")
+        want = sim.simulate(irparse.parse(ir), xs, n, "float32")
+        bufs = [torch.from_numpy(x).cuda() for x in xs]
+        _call(runtime, comms, lambda q, c: c.allreduce(bufs[q], bufs[q]))
+        torch.cuda.synchronize()
+        for q in range(R):
+            assert np.array_equal(bufs[q].cpu().numpy().view(np.uint32), want[q].view(np.uint32))
     finally:
         for c, p in zip(comms, ps):
             c.unload(p)

@@ -1,4 +1,4 @@
-"""GPU parity at production launch parameters (256 KiB slots, 512 threads, unrolled 256-bit
+"""GPU parity at production launch parameters (256 KiB slots, 256 threads, unrolled 256-bit
 vector loops, L2 discard of consumed FIFO lines) with partial last tiles and ragged
 chunks, plus sampled parity at the bench's full size (256 MiB per rank, 8 virtual ranks,
 1 channel x 16 instances) against the oracle's reduction trees (oracle/sampled.py)."""
@@ -12,21 +12,17 @@ from paper_conf_asplos_cowanmmsx23_b200 import programs as P
 pytestmark = pytest.mark.gpu
 
 
-@pytest.fixture(scope="module", autouse=True, params=[(1, 0), (0, 0), (1, 1), (0, 1)],
-                ids=["direct", "fifo", "warp-direct", "warp-fifo"])
+@pytest.fixture(scope="module", autouse=True, params=[1, 0], ids=["direct", "fifo"])
 def production_params(request):
     """Production launch parameters; every test runs with direct placement (reading R15)
-    and with it disabled (all messages through the receiver-side FIFO), each with block-level
-    and with per-warp (reading R18) flags of the Simple protocol."""
+    and with it disabled (all messages through the receiver-side FIFO)."""
     from paper_conf_asplos_cowanmmsx23_b200 import runtime
-    direct, warp = request.param
-    for k, v in (("MSCCL_SLOT_BYTES", 262144), ("MSCCL_SLOTS", 4), ("MSCCL_THREADS", 256),
-                 ("MSCCL_MAX_CHANNELS", 32), ("MSCCL_TIMEOUT_S", 10), ("MSCCL_DIRECT", direct),
-                 ("MSCCL_WARP_FLAGS", warp)):
+    for k, v in (("MSCCL_SLOT_BYTES", 262144), ("MSCCL_LL_SLOT_BYTES", 65536), ("MSCCL_LL128_SLOT_BYTES", 262144),
+                 ("MSCCL_SLOTS", 4), ("MSCCL_THREADS", 256), ("MSCCL_MAX_CHANNELS", 32), ("MSCCL_TIMEOUT_S", 10),
+                 ("MSCCL_DIRECT", request.param)):
         runtime.set_param(k, v)
     yield
     runtime.set_param("MSCCL_DIRECT", 1)
-    runtime.set_param("MSCCL_WARP_FLAGS", 0)
 
 
 @pytest.mark.parametrize("r,extra", [(4, 12345), (3, 7), (2, 131072 * 2 + 999)])
@@ -56,8 +52,8 @@ def test_alltoall_and_allgather_default_slots():
 
 def test_protocols_share_connections():
     """Simple, LL128 and LL programs (and two tile sizes) alternate on the same connections
-    of one communicator set: the monotone counters and every ack word stay consistent
-    across launches whatever protocol or warp partition the previous launch used."""
+    of one communicator set: the monotone counters stay consistent across launches
+    whatever protocol the previous launch used."""
     import gpu_util
     R = 8
     seq = [("Simple", 300001), ("LL128", 40000), ("Simple", 70001), ("LL", 9000), ("Simple", 300001),
@@ -69,6 +65,25 @@ def test_protocols_share_connections():
         got = gpu_util.run_program(ir, xs, n, "float32", "sum")
         for g, w in zip(got, want):
             assert np.array_equal(g.view(np.uint32), w.view(np.uint32)), (proto, n)
+
+
+def test_mixed_protocols_small_int_payload_matching_sequence_numbers():
+    """Simple, LL and LL128 programs alternate on one communicator set with int32
+    data whose words equal the connections' upcoming message sequence numbers (1..400). A
+    receiver that accepted stale bytes of another protocol as a valid LL / LL128 line (the
+    flag check of an LL line is equality with the sequence number) would read old data. Each
+    protocol has its own FIFO slots, so every result is bit-exact with the oracle."""
+    import gpu_util
+    R = 8
+    seq = [("Simple", 60001), ("LL", 3001), ("Simple", 90001), ("LL128", 20001), ("LL", 5001), ("Simple", 40001),
+           ("LL128", 7001), ("LL", 60001), ("Simple", 8001), ("LL", 12001)]
+    for k, (proto, n) in enumerate(seq):
+        ir = P.ring_allreduce(R, instances=2, protocol=proto).to_xml()
+        xs = [((np.arange(n, dtype=np.int64) * (q + 3) + k) % 400 + 1).astype(np.int32) for q in range(R)]
+        want = sim.simulate(irparse.parse(ir), xs, n, "int32", "max")
+        got = gpu_util.run_program(ir, xs, n, "int32", "max")
+        for g, w in zip(got, want):
+            assert np.array_equal(g, w), (proto, n)
 
 
 @pytest.mark.parametrize("instances", [16, 32])

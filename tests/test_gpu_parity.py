@@ -26,6 +26,8 @@ SLOT = 16384
 def small_slots():
     from paper_conf_asplos_cowanmmsx23_b200 import runtime
     runtime.set_param("MSCCL_SLOT_BYTES", SLOT)
+    runtime.set_param("MSCCL_LL_SLOT_BYTES", SLOT)
+    runtime.set_param("MSCCL_LL128_SLOT_BYTES", SLOT)
     runtime.set_param("MSCCL_SLOTS", 4)
     runtime.set_param("MSCCL_TIMEOUT_S", 5)
     yield
