@@ -20,7 +20,11 @@ sim       : executes an IR over per-rank host buffers with bounded FIFOs and
             cross-thread-block semaphores.
 symbolic  : multiset and ordered-tree chunk labels; collective postconditions
             (P:L761-821).
-validate  : structural rules V1-V9 of DESIGN.md, incl. abstract-machine deadlock check.
+validate  : structural rules V1-V9 of DESIGN.md, incl. abstract-machine deadlock check,
+            and V10 (races=True): no happens-before race (``races``).
+races     : happens-before race detection between instructions (program order, deps,
+            k-th send -> k-th receive) and the
+            independent check of the loader's direct-placement marking (reading R15).
 
 Parity status: every function is pinned by ``tests/test_oracle_*.py`` (see DESIGN.md
 "Oracle pins"). The reduction order the paper's own All-Pairs program used is not

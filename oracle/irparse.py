@@ -113,7 +113,10 @@ def _list(el, key):
         x = x.strip()
         if x == "":
             continue
-        out.append(int(x))
+        try:
+            out.append(int(x))
+        except ValueError:
+            raise IRError("<%s> attribute %s=%r is not an integer list" % (el.tag, key, v))
     return out
 
 
@@ -153,6 +156,9 @@ def parse(text):
                 if len(depid) != len(deps):
                     raise IRError("depid/deps length mismatch")
                 pairs = [(b, s) for b, s in zip(depid, deps) if b >= 0]
+                for k in ("srcbuf", "dstbuf"):   # V1 "known enums" (DESIGN.md validator rules)
+                    if st.get(k, "-") not in BUFS + ("-",):
+                        raise IRError("unknown buffer %r" % st.get(k))
                 tb.steps.append(Step(s=_int(st, "s"), op=op, srcbuf=st.get("srcbuf", "-"),
                                      srcoff=_int(st, "srcoff"), dstbuf=st.get("dstbuf", "-"),
                                      dstoff=_int(st, "dstoff"), cnt=_int(st, "cnt"), deps=pairs,

@@ -15,6 +15,9 @@ V8 deps name an existing (tb, step) of another thread block on the same GPU, and
    referenced step sets hasdep (Fig. 5 lines 25-27)
 V9 no deadlock in the abstract machine with the protocol's FIFO slot count, run for >= 2
    pipeline iterations (§5.2; §6.1)
+V10 (races=True) no happens-before race between instructions (oracle/races.py; §3.3
+   P:L859-867, §5.2); with `marking` (the loader's direct placement) also none
+   after the direct writes are moved to the sends
 """
 from .irparse import BUFS
 from .sim import Deadlock, Machine, NullDomain
@@ -28,7 +31,7 @@ def _fail(rule, msg):
     raise ValidationError("%s: %s" % (rule, msg))
 
 
-def validate(algo, nranks=None, slots=8, max_tbs=148, max_channels=64, iters=2):
+def validate(algo, nranks=None, slots=8, max_tbs=148, max_channels=64, iters=2, races=False, marking=None):
     R = algo.ngpus
     if nranks is not None and nranks != R:
         _fail("V2", "program is for %d ranks, communicator has %d" % (R, nranks))
@@ -121,4 +124,16 @@ def validate(algo, nranks=None, slots=8, max_tbs=148, max_channels=64, iters=2):
         Machine(algo, NullDomain(), slots=slots, iters=iters).run()
     except Deadlock as e:
         _fail("V9", "deadlock with %d FIFO slots: %s" % (slots, e))
+    if races or marking is not None:
+        from . import races as hb
+        found = hb.find_races(algo, limit=1)
+        if found:
+            _fail("V10", "%r" % found[0])
+        if marking is not None:
+            try:
+                found = hb.check_direct(algo, marking, limit=1)
+            except hb.MarkingError as e:
+                _fail("V10", "direct-placement marking: %s" % e)
+            if found:
+                _fail("V10", "with direct placement: %r" % found[0])
     return True

@@ -118,3 +118,63 @@ def recv_before_send_ir():
         g.tbs = [ir.ThreadBlock(0, 1 - q, 1 - q, 0, [ir.Step("r", dstbuf="o", dstoff=0), ir.Step("s", "i", 0)])]
         a.gpus.append(g)
     return a.to_xml()
+
+
+# ---------------------------------------------------------------- seeded random mutation
+# (the C++ loader and the oracle's validator must return the same rule on
+# random IR mutants, not only on hand-written ones.) One random edit per mutant: an attribute
+# of a step / thread block / gpu / algo set to a value from a small adversarial domain, a
+# step deleted / duplicated / swapped, a dependency redirected, or a thread block removed.
+def random_bases():
+    return [(P.ring_allreduce(4).to_xml(), 4), (P.allpairs_allreduce(4).to_xml(), 4),
+            (P.ring_allgather(4, 1, 2).to_xml(), 4), (P.ring_reducescatter(4, 1, 1).to_xml(), 4),
+            (P.alltoall_twostep(2, 2).to_xml(), 4), (P.hierarchical_allreduce(2, 2).to_xml(), 4),
+            (P.ring_allreduce(4, inplace=True).to_xml(), 4), (P.oneshot_allreduce(4).to_xml(), 4)]
+
+
+def mutate(text, rng):
+    import xml.etree.ElementTree as ET
+    root = ET.fromstring(text)
+    gpus = list(root); g = rng.choice(gpus); tbs = list(g); tb = rng.choice(tbs); steps = list(tb)
+    kind = rng.randrange(9)
+    vals = ["-2", "-1", "0", "1", "2", "3", "4", "7", "65536", "x", "-"]
+    if kind == 0 and steps:
+        st = rng.choice(steps); a = rng.choice(["type","srcbuf","srcoff","dstbuf","dstoff","cnt","depid","deps","hasdep"])
+        if a == "type": st.set(a, rng.choice(["s","r","cpy","re","rrc","rrs","rrcs","rcs","nop","zz"]))
+        elif a.endswith("buf"): st.set(a, rng.choice(["i","o","s","-","q"]))
+        else: st.set(a, rng.choice(vals))
+    elif kind == 1:
+        tb.set(rng.choice(["send","recv","chan","id"]), rng.choice(vals[:8]))
+    elif kind == 2:
+        g.set(rng.choice(["i_chunks","o_chunks","s_chunks","id"]), rng.choice(vals[:9]))
+    elif kind == 3 and steps:
+        tb.remove(rng.choice(steps))
+        for i, st in enumerate(list(tb)): st.set("s", str(i))
+    elif kind == 4 and steps:
+        st = rng.choice(steps); import copy; c = copy.deepcopy(st); tb.append(c)
+        for i, st in enumerate(list(tb)): st.set("s", str(i))
+    elif kind == 5 and len(steps) > 1:
+        i, j = rng.sample(range(len(steps)), 2)
+        for x in list(tb): tb.remove(x)
+        steps[i], steps[j] = steps[j], steps[i]
+        for k, st in enumerate(steps): st.set("s", str(k)); tb.append(st)
+    elif kind == 6 and steps:
+        st = rng.choice(steps); b = rng.randrange(len(tbs)); s = rng.randrange(4)
+        st.set("depid", str(b)); st.set("deps", str(s))
+    elif kind == 7:
+        root.set(rng.choice(["ngpus","coll","proto","inplace"]), rng.choice(["1","2","4","5","allreduce","allgather","custom","LL","Simple","bogus"]))
+    else:
+        g.remove(tb)
+    return ET.tostring(root, encoding="unicode")
+
+
+def random_mutants(seed, n):
+    """n (text, nranks) mutants from a seeded generator."""
+    import random
+    rng = random.Random(seed)
+    bases = random_bases()
+    out = []
+    for _ in range(n):
+        base, R = rng.choice(bases)
+        out.append((mutate(base, rng), R))
+    return out

@@ -92,3 +92,28 @@ def test_cpp_parser_rejects_malformed(rt):
                 'dstoff="0" cnt="1" depid="-1" deps="-1" hasdep="0"/></tb></gpu></algo>']:
         ok, msg = rt.validate(bad, 1)
         assert not ok and msg.startswith("V1"), (bad, msg)
+
+
+@pytest.mark.parametrize("seed", [0, 1, 2])
+def test_cpp_and_python_validators_agree_on_random_mutants(rt, seed):
+    """1000 seeded random IR mutants per seed: both validators accept, or both reject with
+    the same rule (V1..V9)."""
+    seen = set()
+    accepted = 0
+    for text, R in irmutate.random_mutants(seed, 1000):
+        ok, msg = rt.validate(text, R, slots=8)
+        try:
+            pyval.validate(irparse.parse(text), nranks=R, slots=8)
+            py = None
+        except irparse.IRError:
+            py = "V1"
+        except pyval.ValidationError as e:
+            py = str(e)[:2]
+        cpp = None if ok else msg[:2]
+        assert cpp == py, (cpp, msg, py, text)
+        if cpp:
+            seen.add(cpp)
+        else:
+            accepted += 1
+    assert {"V1", "V2", "V3", "V4", "V5", "V6", "V7", "V8"} <= seen, seen  # V9: deadlock fixtures above
+    assert 50 < accepted < 900
