@@ -1,21 +1,36 @@
 #!/usr/bin/env python3
 """Benchmark of the MSCCL-IR interpreter (MSCCLang, ASPLOS '23) on B200.
 
-Metric (BASELINE.json): AllReduce / AllToAll bus bandwidth (nccl-tests convention,
-busBW = S/t * 2(R-1)/R for AllReduce, S = bytes per rank) — one JSON line on stdout.
+Metric (BASELINE.json): AllReduce / AllToAll bus bandwidth vs size at 2/4/8 B200 and the
+1 KB latency. busBW follows the nccl-tests convention: algBW x 2(R-1)/R for
+AllReduce and x (R-1)/R for AllGather / ReduceScatter / AllToAll, with S = bytes per rank.
 
-Workload of the default run (N=1, one GPU): BASELINE config 1 — ring AllReduce, bf16,
-8 channels, pipelined chunks — executed by R=8 VIRTUAL ranks on one B200 (all ranks'
-buffers and FIFOs in that GPU's HBM, one cooperative interpreter launch per step), at
-S = 256 MiB per rank (inputs 2 GiB > 126 MB L2, so no L2 flush is needed). With one GPU
-the "links" are HBM: the roofline is HBM bandwidth.
+Default run (N = 1: one GPU, no flags) -- one JSON line:
+  workload = the largest single-GPU analogue of BASELINE configs[1] ("Ring AllReduce
+  8xB200, bf16, pipelined chunks"): ring AllReduce MSCCL-IR, bf16, R = 8 VIRTUAL ranks on
+  one B200 (every rank's buffers, FIFOs and peer stores in that GPU's HBM, one cooperative
+  interpreter launch per step), 256 MiB per rank, 1 channel x 32 instances (256 CTAs).
+  One GPU cannot host NVLink traffic, so this line is HBM-bound and its roofline is the
+  measured HBM copy bandwidth. Inputs: 2 GiB > 126 MB L2, no flush needed.
+  Extras measured on the same virtual ranks (each named by the BASELINE config it
+  mirrors): the 1 KiB fp16 latency (configs[2]), the launch-latency floor, the AllToAll at
+  256 MiB per rank (configs[3]), and AllGather / ReduceScatter (configs[4]).
 
-Under torchrun (N>1) each process drives one GPU as one rank over CUDA IPC peer memory
-(NVLink/NVSwitch): ring AllReduce over N ranks, S per rank fixed ("weak"), value = busBW
-from the max over ranks of the CUDA-event time.
+Under torchrun (N > 1) each process drives one GPU as one rank over CUDA IPC peer memory
+(NVLink / NVSwitch). User buffers are registered (mscclCommRegister), so messages are
+placed directly into the peer's buffer (reading R15b). value = ring AllReduce busBW at S
+per rank from the max over ranks of the CUDA-event time; roofline = NVLink per direction
+(measured peer copy, nominal 900 GB/s); NCCL 2.28.9 runs in the same loop as the
+comparison arm. MSCCL_FORCE_DEVICE=<d> puts every rank on GPU d, which exercises the
+multi-process plumbing on a one-GPU box (NCCL is then skipped: it refuses two ranks on one
+GPU).
 
-`--impl reference` times the CPU oracle (oracle/sim.py) executing the same program on a
-bounded sample of the same workload, on the host cores.
+--sweep PATH : per-size JSON lines (1 KiB..1 GiB, x2) for AllReduce and AllToAll, eager and
+  CUDA graph, the paper's protocol (20 warm-up + 50 timed ops) plus a
+  1000-iteration latency mode for <= 64 KiB; MSCCL (size-range program sets, §6
+  P:L1268-1273) and, with N > 1, NCCL.
+--impl reference : the CPU oracle (oracle/sim.py) executing the same IR on a bounded
+  sample of the same workload, on the host cores (the reference arm).
 """
 import argparse
 import json
@@ -31,6 +46,7 @@ sys.path.insert(0, ROOT)
 
 MIB = 1 << 20
 SEED_SAMPLES = 4096
+NVLINK_NOMINAL = 900.0  # GB/s per direction per GPU (NVLink 5)
 
 
 def parse():
@@ -50,7 +66,11 @@ def parse():
     ap.add_argument("--slot-kib", type=int, default=256)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu", action="store_true")
-    ap.add_argument("--quiet-extra", action="store_true", help="skip the small-message and AllToAll extras")
+    ap.add_argument("--no-nccl", action="store_true")
+    ap.add_argument("--no-register", action="store_true", help="N>1: do not register buffers (FIFO only)")
+    ap.add_argument("--quiet-extra", action="store_true", help="skip the extras")
+    ap.add_argument("--sweep", default=None, help="write per-size JSON lines to this path (and stdout)")
+    ap.add_argument("--sweep-max-mib", type=int, default=1024)
     return ap.parse_args()
 
 
@@ -155,17 +175,27 @@ def build_program(args, R):
     return P.alltoall_twostep(1, R, instances=args.instances, protocol=args.protocol)
 
 
-def simple_bytes_per_rank(algo, rank, S_per_chunk):
-    """Algorithmic HBM bytes of one launch for one rank under the FIFO protocol: each
-    instruction reads/writes its operands once per chunk."""
-    touches = {"s": 2, "r": 2, "cpy": 2, "re": 3, "rrc": 3, "rrs": 3, "rrcs": 4, "rcs": 3, "nop": 0}
-    g = algo.gpus[rank]
-    return sum(touches[st.op] * st.cnt for tb in g.tbs for st in tb.steps) * S_per_chunk
+def nop_ir(R):
+    """The smallest MSCCL-IR program: every rank one thread block with one nop. Its CUDA-graph
+    replay time is the interpreter's launch-latency floor (cooperative launch + prologue +
+    epilogue), against which the 1 KiB latencies are read."""
+    g = "".join('<gpu id="%d" i_chunks="1" o_chunks="1" s_chunks="0"><tb id="0" send="-1" recv="-1" chan="0">'
+                '<step s="0" type="nop" srcbuf="-" srcoff="-1" dstbuf="-" dstoff="-1" cnt="1" depid="-1" '
+                'deps="-1" hasdep="0"/></tb></gpu>' % q for q in range(R))
+    return '<algo name="nop" coll="custom" ngpus="%d" proto="LL" inplace="0" nchannels="1">%s</algo>' % (R, g)
+
+
+def host_threads():
+    try:
+        return len(os.sched_getaffinity(0))
+    except Exception:
+        return os.cpu_count()
 
 
 # ----------------------------------------------------------------------------- CPU oracle
-def cpu_oracle_run(args, R, algo, sample_bytes, reps=3):
-    """Time oracle.sim.simulate on a bounded sample (same program, same dtype)."""
+def cpu_oracle_run(R, algo, sample_bytes, reps=5):
+    """Time oracle.sim.simulate on a bounded sample (same program, same dtype, same R);
+    median of `reps` runs, numpy in one Python thread."""
     import numpy as np
     import synth
     from oracle import irparse, sim
@@ -180,12 +210,14 @@ def cpu_oracle_run(args, R, algo, sample_bytes, reps=3):
         times.append(time.perf_counter() - t0)
     t = statistics.median(times)
     return {"value": round(busbw("allreduce", n * 2, t, R), 4), "unit": "GB/s", "cores": 1,
-            "host_cores": len(os.sched_getaffinity(0)), "kind": "oracle",
-            "sample": "ring AllReduce R=%d bf16, %d MiB per rank (median of %d runs of oracle.sim.simulate, "
-                      "numpy, 1 thread), %.2f s per run" % (R, n * 2 // MIB, reps, t)}
+            "host_cores": host_threads(), "kind": "oracle",
+            "sample": "the same IR program (%s, R=%d, bf16) on %d MiB per rank instead of the workload's size: "
+                      "median of %d runs of oracle.sim.simulate (numpy, 1 thread), %.2f s per run"
+                      % (algo.name, R, n * 2 // MIB, reps, t)}
 
 
 def run_reference(args):
+    """--impl reference: the CPU oracle as it stands, on a bounded sample of the workload."""
     rank = int(os.environ.get("RANK", "0"))
     if rank != 0:
         return
@@ -211,8 +243,10 @@ def run_reference(args):
            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
            "config": cfg,
            "cpu_baseline": {"value": round(v, 4), "unit": "GB/s", "cores": 1, "kind": "oracle",
-                            "host_cores": len(os.sched_getaffinity(0)),
-                            "sample": "oracle.sim.simulate of the same IR, %d MiB per rank per step" % (sample // MIB)},
+                            "host_cores": host_threads(),
+                            "sample": "each step: oracle.sim.simulate of the same IR on %d MiB per rank (the "
+                                      "workload is %d MiB per rank; busBW is size-independent for the oracle)"
+                                      % (sample // MIB, int(args.size_mib))},
            "e2e": {"value": round(v, 4), "unit": "GB/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(out), flush=True)
 
@@ -224,30 +258,38 @@ def metric_name(coll="allreduce"):
 
 
 def config_dict(args, R, N):
-    mode = "virtual ranks on 1 GPU" if N == 1 else "1 process per GPU, CUDA IPC peer memory"
-    what = {"ring": "BASELINE config 1: ring AllReduce", "allpairs": "BASELINE config 2: all-pairs AllReduce",
-            "oneshot": "BASELINE config 2: one-shot AllReduce",
-            "alltoall": "BASELINE config 3: direct AllToAll"}[args.program]
-    return {"workload": "%s MSCCL-IR, %d channels, %d instances, %s protocol, %d ranks (%s), %d MiB per rank"
-                        % (what, args.channels, args.instances, args.protocol, R, mode, int(args.size_mib)),
+    if N == 1:
+        base = {"ring": "largest single-GPU analogue of BASELINE configs[1] (ring AllReduce, bf16)",
+                "allpairs": "BASELINE configs[2] shape (all-pairs AllReduce)",
+                "oneshot": "BASELINE configs[2] shape (one-shot AllReduce)",
+                "alltoall": "BASELINE configs[3] shape (AllToAll)"}[args.program]
+        mode = "%d virtual ranks on 1 B200 (HBM-bound)" % R
+    else:
+        base = {"ring": "BASELINE configs[1]: ring AllReduce, bf16", "allpairs": "all-pairs AllReduce",
+                "oneshot": "one-shot AllReduce", "alltoall": "BASELINE configs[3]: AllToAll"}[args.program]
+        mode = "%d B200, 1 process per GPU, CUDA IPC over NVLink" % N
+    return {"workload": "%s -- MSCCL-IR %s, %d channel(s) x %d instance(s), %s protocol, %s, %d MiB per rank"
+                        % (base, args.program, args.channels, args.instances, args.protocol, mode,
+                           int(args.size_mib)),
             "program": args.program, "ranks": R, "bytes_per_rank": int(args.size_mib * MIB),
             "channels": args.channels, "instances": args.instances, "protocol": args.protocol,
             "threads": args.threads, "slots": args.slots, "slot_bytes": args.slot_kib * 1024,
-            "l2": "inputs (%d MiB total) larger than L2 (126 MB); no flush" % int(args.size_mib * R),
+            "l2": "inputs (%d MiB total) larger than L2 (126 MB); no flush" % int(args.size_mib * (R if N == 1 else 1)),
             "parallelism": "virtual%d" % R if N == 1 else "ranks%d" % N}
 
 
-# ----------------------------------------------------------------------------- GPU runs
+# ----------------------------------------------------------------------------- GPU helpers
 def set_params(rt, args):
     rt.set_param("MSCCL_SLOTS", args.slots)
     rt.set_param("MSCCL_SLOT_BYTES", args.slot_kib * 1024)
     rt.set_param("MSCCL_THREADS", args.threads)
     rt.set_param("MSCCL_MAX_CHANNELS", max(32, args.channels * args.instances))
-    rt.set_param("MSCCL_TIMEOUT_S", 30)
+    rt.set_param("MSCCL_TIMEOUT_S", 60)
 
 
-def sampled_parity(algo, recv_list, n, ranks_to_check):
-    """Bit-exact check of sampled outputs against the oracle's reduction trees."""
+def sampled_parity(algo, recv_list, n, ranks_to_check, local=None):
+    """Bit-exact check of sampled outputs against the oracle's reduction trees.
+    recv_list[i] is the output of rank (local[i] if local else i)."""
     import numpy as np
     import torch
     import synth
@@ -256,45 +298,313 @@ def sampled_parity(algo, recv_list, n, ranks_to_check):
     g = np.random.default_rng(1)
     idx = np.unique(np.concatenate([g.integers(0, n, SEED_SAMPLES), [0, n - 1, n // 2]]))
     bad = 0
-    for q in ranks_to_check:
-        want = sampled.reduction_at(al, lambda r, i: synth.hashed_numpy(r, i, "bfloat16"), n, "bfloat16", "sum",
-                                      idx, rank=q)
-        got = recv_list[q][torch.from_numpy(idx).to(recv_list[q].device)].view(torch.int16).cpu().numpy() \
-            .view(np.uint16)
+    for i, q in enumerate(ranks_to_check):
+        want = sampled.reduction_at(al, lambda r, ii: synth.hashed_numpy(r, ii, "bfloat16"), n, "bfloat16", "sum",
+                                    idx, rank=q)
+        out = recv_list[q if local is None else local.index(q)]
+        got = out[torch.from_numpy(idx).to(out.device)].view(torch.int16).cpu().numpy().view(np.uint16)
         bad += int(np.count_nonzero(got != want))
     return bad, idx.size * len(ranks_to_check)
 
 
+class Ranks:
+    """The ranks this process drives: all R virtual ranks (N = 1) or its one rank (N > 1).
+    call(progs, sends, recvs, count) issues one collective on every local rank in one group
+    (one cooperative launch per device)."""
+
+    def __init__(self, rt, comms, ranks, R, world, dev):
+        self.rt, self.comms, self.ranks, self.R, self.world, self.dev = rt, comms, ranks, R, world, dev
+
+    def load(self, algo, lo=0, hi=0):
+        return [c.load(algo.to_xml(), lo, hi) for c in self.comms]
+
+    def unload(self, progs):
+        for c, p in zip(self.comms, progs):
+            c.unload(p)
+
+    def call(self, progs, sends, recvs, count, stream=None):
+        with self.rt.group():
+            for c, p, s, r in zip(self.comms, progs, sends, recvs):
+                c.run(p, s, r, count, stream=stream)
+
+    def coll(self, coll, sends, recvs, stream=None):
+        with self.rt.group():
+            for c, s, r in zip(self.comms, sends, recvs):
+                getattr(c, coll)(s, r, stream=stream)
+
+    def tmax(self, t):
+        """max over ranks of a per-rank time (device-timed), via the plumbing group."""
+        if self.world == 1:
+            return t
+        import torch
+        import torch.distributed as dist
+        tt = torch.tensor([t], dtype=torch.float64)
+        if dist.get_backend() == "nccl":
+            tt = tt.to(self.dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        return float(tt.item())
+
+    def all_ok(self, ok):
+        if self.world == 1:
+            return bool(ok)
+        import torch
+        import torch.distributed as dist
+        tt = torch.tensor([1 if ok else 0], dtype=torch.int64)
+        if dist.get_backend() == "nccl":
+            tt = tt.to(self.dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MIN)
+        return bool(tt.item())
+
+    def barrier(self):
+        if self.world > 1:
+            import torch.distributed as dist
+            dist.barrier()
+
+
+def timed(fn, iters, warmup, stream, graph, R):
+    """Mean device time per call of fn() (CUDA events on `stream`, synchronised on both
+    sides, max over ranks). graph=True captures `iters` calls into one CUDA graph and times
+    its replay. Returns (seconds, mode)."""
+    import torch
+    for _ in range(warmup):
+        fn()
+    torch.cuda.synchronize()
+    mode = "eager"
+    run = None
+    if graph:
+        try:
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g, stream=stream):
+                for _ in range(iters):
+                    fn()
+            g.replay()
+            torch.cuda.synchronize()
+            run, mode = g.replay, "cuda-graph"
+        except Exception as e:
+            torch.cuda.synchronize()
+            print("graph capture failed: %s" % e, file=sys.stderr)
+            run = None
+    if run is None:
+        def run():
+            for _ in range(iters):
+                fn()
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    R.barrier()
+    torch.cuda.synchronize()
+    e0.record(stream)
+    run()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    return R.tmax(e0.elapsed_time(e1) / 1e3 / iters), mode
+
+
+# ----------------------------------------------------------------------------- extras
+def extras(R, stream, nccl=None, S=256 * MIB):
+    """BASELINE configs[2..4] on the same ranks: 1 KiB fp16 AllReduce latency (graph replay;
+    one-shot / two-shot / ring LL) and the launch floor, AllToAll at 256 MiB per rank, and
+    AllGather / ReduceScatter rings at 256 MiB per rank."""
+    import torch
+    import synth
+    from paper_conf_asplos_cowanmmsx23_b200 import programs as P
+    W = R.R
+    out = {}
+    lat = {}
+    n = 512  # 1 KiB of fp16 per rank
+    send = [synth.hashed(q, torch.arange(n, device=R.dev), "float16") for q in R.ranks]
+    recv = [torch.empty_like(x) for x in send]
+    for name, algo in (("floor_nop", None), ("oneshot_LL", P.oneshot_allreduce(W, protocol="LL")),
+                       ("allpairs_LL", P.allpairs_allreduce(W, protocol="LL")),
+                       ("ring_LL", P.ring_allreduce(W, protocol="LL")),
+                       ("ring_ch%d_LL" % W, P.ring_allreduce(W, channels=W, protocol="LL"))):
+        if algo is None:
+            progs = [c.load(nop_ir(W)) for c in R.comms]
+        else:
+            progs = R.load(algo, 0, 1 << 20)
+        try:
+            t, mode = timed(lambda: R.call(progs, send, recv, n, stream), 50, 5, stream, True, R)
+            lat[name] = round(t * 1e6, 2)
+            lat["mode"] = mode
+        except Exception as e:
+            lat[name] = "error: %s" % str(e)[:160]
+        R.unload(progs)
+    if nccl is not None:
+        t, mode = timed(lambda: nccl.allreduce(send[0], recv[0], "float16", stream=stream.cuda_stream), 50, 5,
+                        stream, True, R)
+        lat["nccl_allreduce"] = round(t * 1e6, 2)
+    lat["note"] = ("floor_nop = an MSCCL-IR program of one nop per rank: cooperative launch + prologue + "
+                   "epilogue under graph replay; the collective latencies are read against it")
+    out["allreduce_1KiB_fp16_latency_us"] = lat
+    del send, recv
+    # AllToAll (direct two-step N=1), AllGather and ReduceScatter rings: S per rank (256 MiB), bf16
+    n = S // 2
+    nb = n // W
+    specs = (("alltoall", P.alltoall_twostep(1, W, instances=2 if R.world == 1 else 4), n, n, nb),
+             ("allgather", P.ring_allgather(W, 1, 32 if R.world == 1 else 8), nb, n, nb),
+             ("reducescatter", P.ring_reducescatter(W, 1, 32 if R.world == 1 else 8), n, nb, nb))
+    for coll, algo, ins, outs, cnt in specs:
+        progs = R.load(algo)
+        send = [synth.hashed(q, torch.arange(ins, device=R.dev), "bfloat16") for q in R.ranks]
+        recv = [torch.empty(outs, dtype=torch.bfloat16, device=R.dev) for _ in R.ranks]
+        regs = register_all(R, send + recv)
+        t, mode = timed(lambda: R.call(progs, send, recv, cnt, stream), 5, 2, stream, False, R)
+        if coll == "alltoall":
+            ok = check_alltoall(R, recv, W, n)
+        elif coll == "allgather":
+            ok = check_allgather(R, recv, W, nb)
+        else:
+            ranks = [q for q in (0, W - 1) if q in R.ranks]
+            bad, _ = sampled_parity(algo, recv, nb, ranks, local=R.ranks)
+            ok = bad == 0
+        ent = {"busbw_GBps": round(busbw(coll, S, t, W), 2), "ms": round(t * 1e3, 3),
+               "ctas_per_rank": int(progs[0].info()["thread_blocks"]), "bit_exact": R.all_ok(ok)}
+        if nccl is not None:
+            fn = {"alltoall": lambda: nccl.alltoall(send[0], recv[0], "bfloat16", W, stream.cuda_stream),
+                  "allgather": lambda: nccl.allgather(send[0], recv[0], "bfloat16", stream.cuda_stream),
+                  "reducescatter": lambda: nccl.reducescatter(send[0], recv[0], "bfloat16", "sum",
+                                                              stream.cuda_stream)}[coll]
+            tn, _ = timed(fn, 5, 2, stream, False, R)
+            ent["nccl_busbw_GBps"] = round(busbw(coll, S, tn, W), 2)
+        out["%s_bf16_%dMiB" % (coll, S // MIB)] = ent
+        for r_ in regs:
+            r_.deregister()
+        R.unload(progs)
+        del send, recv
+        torch.cuda.empty_cache()
+    return out
+
+
+def check_alltoall(R, recv, W, n):
+    import torch
+    import synth
+    ok = True
+    for i, q in enumerate(R.ranks):
+        if q not in (0, W - 1):
+            continue
+        for p in range(W):
+            src = synth.hashed(p, torch.arange(q * (n // W), (q + 1) * (n // W), device=R.dev), "bfloat16")
+            ok = ok and torch.equal(recv[i].view(W, -1)[p], src)
+    return ok
+
+
+def check_allgather(R, recv, W, nb):
+    import torch
+    import synth
+    ok = True
+    for i, q in enumerate(R.ranks):
+        if q not in (0, W - 1):
+            continue
+        for p in range(W):
+            ok = ok and torch.equal(recv[i].view(W, -1)[p], synth.hashed(p, torch.arange(nb, device=R.dev),
+                                                                         "bfloat16"))
+    return ok
+
+
+def register_all(R, tensors):
+    """N > 1: register the user buffers for direct placement (reading R15b), collectively."""
+    if R.world == 1 or getattr(R, "no_register", False):
+        return []
+    from paper_conf_asplos_cowanmmsx23_b200 import dist as mdist
+    return [mdist.register(R.comms[0], t) for t in tensors]
+
+
+# ----------------------------------------------------------------------------- sweep
+def sweep(R, stream, path, max_mib, nccl=None):
+    """Per-size JSON lines: AllReduce (the size-range program set of
+    programs.tuned_allreduce) and AllToAll (programs.tuned_alltoall), 1 KiB .. max per rank,
+    eager and CUDA graph; 20 warm-up + 50 timed ops, and 1000 for the <= 64 KiB
+    latency mode. Correctness of the last op: bit-exact sampled parity (AllReduce, oracle
+    reduction trees) / exact permutation (AllToAll)."""
+    import torch
+    import synth
+    from paper_conf_asplos_cowanmmsx23_b200 import programs as P
+    W = R.R
+    f = open(path, "w") if path else None
+    impl_sets = {"allreduce": P.tuned_allreduce(W), "alltoall": P.tuned_alltoall(W)}
+    lines = []
+    for coll in ("allreduce", "alltoall"):
+        sets = [(algo, lo, hi, R.load(algo, lo, hi)) for algo, lo, hi in impl_sets[coll]]
+        size = 1024
+        while size <= max_mib * MIB:
+            n = size // 2
+            send = [synth.hashed(q, torch.arange(n, device=R.dev), "bfloat16") for q in R.ranks]
+            recv = [torch.empty_like(x) for x in send]
+            regs = register_all(R, send + recv)
+            per = (n // W) * 2 if coll == "alltoall" else size   # selection bytes (count * w)
+            chosen = next(a for a, lo, hi, _ in sets if lo <= per and (hi == 0 or per < hi))
+            impls = [("msccl", lambda: R.coll(coll, send, recv, stream))]
+            if nccl is not None:
+                impls.append(("nccl", (lambda: nccl.allreduce(send[0], recv[0], "bfloat16", stream=stream.cuda_stream))
+                              if coll == "allreduce" else
+                              (lambda: nccl.alltoall(send[0], recv[0], "bfloat16", W, stream.cuda_stream))))
+            for impl, fn in impls:
+                for graph in (False, True):
+                    iters = 50 if size <= 256 * MIB else 20
+                    t, mode = timed(fn, iters, 20, stream, graph, R)
+                    rec = {"impl": impl, "coll": coll, "program": chosen.name if impl == "msccl" else "nccl",
+                           "R": W, "dtype": "bf16", "op": "sum", "bytes": size, "count": n,
+                           "iters": iters, "warmup": 20, "graph": mode == "cuda-graph", "t_us_max": round(t * 1e6, 3),
+                           "algbw": round(size / t / 1e9, 3), "busbw": round(busbw(coll, size, t, W), 3)}
+                    if R.world > 1:
+                        rec["frac_nvlink"] = round(rec["busbw"] / NVLINK_NOMINAL, 4)
+                    if size <= 64 * 1024 and graph:
+                        tl, _ = timed(fn, 1000, 20, stream, True, R)
+                        rec["latency_mode_us"] = round(tl * 1e6, 3)
+                    if impl == "msccl":
+                        if coll == "allreduce":
+                            ranks = [q for q in (0, W - 1) if q in R.ranks]
+                            bad, _ = sampled_parity(chosen, recv, n, ranks, local=R.ranks)
+                            rec["correct"] = R.all_ok(bad == 0)
+                        else:
+                            rec["correct"] = R.all_ok(check_alltoall(R, recv, W, n))
+                    lines.append(rec)
+                    if int(os.environ.get("RANK", "0")) == 0:
+                        print(json.dumps(rec), flush=True)
+                        if f:
+                            f.write(json.dumps(rec) + "\n")
+                            f.flush()
+            for r_ in regs:
+                r_.deregister()
+            del send, recv
+            torch.cuda.empty_cache()
+            size *= 2
+        for _, _, _, progs in sets:
+            R.unload(progs)
+    if f:
+        f.close()
+    return lines
+
+
+# ----------------------------------------------------------------------------- N = 1
 def run_virtual(args):
     import torch
     import synth
     from paper_conf_asplos_cowanmmsx23_b200 import runtime as rt
-    R = args.ranks
+    W = args.ranks
     set_params(rt, args)
-    algo = build_program(args, R)
+    algo = build_program(args, W)
     ir_text = algo.to_xml()
     S = int(args.size_mib * MIB)
     n = S // 2
     dev = torch.device("cuda:0")
-    comms = rt.Comm.virtual(R, 0)
+    comms = rt.Comm.virtual(W, 0)
+    R = Ranks(rt, comms, list(range(W)), W, 1, dev)
+    stream = torch.cuda.current_stream()
+    if args.sweep:
+        rt.set_param("MSCCL_MAX_CHANNELS", 64)
+        sweep(R, stream, args.sweep, args.sweep_max_mib)
+        return None
     progs = [c.load(ir_text) for c in comms]
     direct = rt.get_param("MSCCL_DIRECT") != 0 and args.protocol == "Simple"
     touches = [p.touches(direct) for p in progs]
     idx = torch.arange(n, device=dev, dtype=torch.int64)
-    send = [synth.hashed(q, idx, "bfloat16") for q in range(R)]
+    send = [synth.hashed(q, idx, "bfloat16") for q in range(W)]
     del idx
-    recv = [torch.empty(n, dtype=torch.bfloat16, device=dev) for _ in range(R)]
-    stream = torch.cuda.current_stream()
-
+    recv = [torch.empty(n, dtype=torch.bfloat16, device=dev) for _ in range(W)]
     coll = "alltoall" if args.program == "alltoall" else "allreduce"
+    count = n // W if coll == "alltoall" else n
 
     def step():
-        with rt.group():
-            for q in range(R):
-                if coll == "alltoall":
-                    comms[q].alltoall(send[q], recv[q], stream=stream)
-                else:
-                    comms[q].allreduce(send[q], recv[q], stream=stream)
+        R.call(progs, send, recv, count, stream)
 
     for _ in range(args.warmup):
         step()
@@ -316,191 +626,140 @@ def run_virtual(args):
     for c in comms:
         if c.async_error():
             raise RuntimeError("watchdog fired during the bench")
-    if coll == "alltoall":  # bit-exact block permutation on the first and last rank
-        bad = sum(int(torch.count_nonzero(recv[q].view(R, -1)[p] != send[p].view(R, -1)[q]))
-                  for q in (0, R - 1) for p in range(R))
-        total = 2 * n
+    if coll == "alltoall":
+        ok = check_alltoall(R, recv, W, n)
+        bad, total = (0 if ok else 1), 2 * n
     else:
-        bad, total = sampled_parity(algo, recv, n, [0, R - 1])
+        bad, total = sampled_parity(algo, recv, n, [0, W - 1])
     res = {"t": t, "coll": coll, "launches": launches, "clocks": clk, "parity_bad": bad, "parity_total": total,
-           "algo": algo, "S": S, "R": R, "touches": touches, "direct": direct}
-    # end-to-end through the public API with host buffers (pinned), every step
+           "algo": algo, "S": S, "R": W, "touches": touches, "direct": direct}
     if not args.no_e2e:
-        host_in = [s.cpu().pin_memory() for s in send]
-        host_out = [torch.empty(n, dtype=torch.bfloat16).pin_memory() for _ in range(R)]
-        e2e_steps = max(2, min(5, args.steps))
-
-        def e2e_step():
-            for q in range(R):
-                send[q].copy_(host_in[q], non_blocking=True)
-            step()
-            for q in range(R):
-                host_out[q].copy_(recv[q], non_blocking=True)
-
-        e2e_step()
-        torch.cuda.synchronize()
-        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        for _ in range(e2e_steps):
-            e2e_step()
-        e1.record(stream)
-        torch.cuda.synchronize()
-        te = e0.elapsed_time(e1) / 1e3 / e2e_steps
-        res["e2e"] = {"value": round(busbw("allreduce", S, te, R), 3), "unit": "GB/s",
-                      "h2d_bytes_per_step": S * R, "d2h_bytes_per_step": S * R,
-                      "ms_per_step": round(te * 1e3, 3),
-                      "note": "C-ABI call with pinned host buffers: H2D of all %d ranks' inputs + AllReduce + "
-                              "D2H of all outputs per step (PCIe-bound)" % R}
+        res["e2e"] = e2e(R, send, recv, lambda: step(), S, coll, W, args.steps, stream)
+    R.unload(progs)
     if not args.quiet_extra:
         del send, recv
         torch.cuda.empty_cache()
-        res["extras"] = virtual_extras(comms, R, stream)
+        res["extras"] = extras(R, stream)
     for c in comms:
         c.destroy()
     return res
 
 
-def _timed(fn, iters, stream, graph=True):
-    """Mean device time per call of fn(); CUDA-graph replay of `iters` calls when possible."""
+def e2e(R, send, recv, step, S, coll, W, steps, stream):
+    """The same metric end to end through the public API: every step copies the step's
+    inputs from pinned host memory to the device, runs the collective, and reads the result
+    back (all local ranks); max over ranks."""
     import torch
-    fn()
+    host_in = [s.cpu().pin_memory() for s in send]
+    host_out = [torch.empty(r.numel(), dtype=r.dtype).pin_memory() for r in recv]
+    k = max(2, min(5, steps))
+
+    def e2e_step():
+        for s, h in zip(send, host_in):
+            s.copy_(h, non_blocking=True)
+        step()
+        for r, h in zip(recv, host_out):
+            h.copy_(r, non_blocking=True)
+
+    e2e_step()
     torch.cuda.synchronize()
-    mode = "eager"
-    if graph:
-        try:
-            g = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(g):
-                for _ in range(iters):
-                    fn()
-            g.replay()
-            torch.cuda.synchronize()
-            run = g.replay
-            mode = "cuda-graph"
-        except Exception as e:
-            torch.cuda.synchronize()
-            print("graph capture failed: %s" % e, file=sys.stderr)
-            run = None
-    if mode == "eager":
-        def run():
-            for _ in range(iters):
-                fn()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    run()
-    torch.cuda.synchronize()
+    R.barrier()
     e0.record(stream)
-    for _ in range(5):
-        run()
+    for _ in range(k):
+        e2e_step()
     e1.record(stream)
     torch.cuda.synchronize()
-    return e0.elapsed_time(e1) / 1e3 / (5 * iters), mode
+    te = R.tmax(e0.elapsed_time(e1) / 1e3 / k)
+    nl = len(send)
+    return {"value": round(busbw(coll, S, te, W), 3), "unit": "GB/s",
+            "h2d_bytes_per_step": S * nl, "d2h_bytes_per_step": S * nl, "ms_per_step": round(te * 1e3, 3),
+            "note": "C-ABI call with pinned host buffers: H2D of this process's %d rank input(s) + collective + "
+                    "D2H of the output(s) per step (PCIe-bound)" % nl}
 
 
-def virtual_extras(comms, R, stream):
-    """BASELINE configs 3 and 4 on the same virtual ranks: 1 KB AllReduce latency (LL
-    one-shot / two-shot / ring) and AllToAll busBW at 256 MiB per rank."""
+# ----------------------------------------------------------------------------- N > 1
+def peer_copy_peak(rank, world, dev):
+    """Measured one-direction peer copy GB/s between this GPU and the next (1 GiB, best of
+    5, CUDA events), the NVLink roofline denominator; None when GPUs are shared."""
     import torch
-    import synth
-    from paper_conf_asplos_cowanmmsx23_b200 import programs as P
-    from paper_conf_asplos_cowanmmsx23_b200 import runtime as rt
-    dev = torch.device("cuda:0")
-    out = {}
-    lat = {}
-    n = 512  # 1 KiB of fp16 per rank
-    send = [synth.hashed(q, torch.arange(n, device=dev), "float16") for q in range(R)]
-    recv = [torch.empty_like(x) for x in send]
-    for name, algo in (("oneshot_LL", P.oneshot_allreduce(R, protocol="LL")),
-                       ("allpairs_LL", P.allpairs_allreduce(R, protocol="LL")),
-                       ("ring_LL", P.ring_allreduce(R, protocol="LL"))):
-        progs = [c.load(algo.to_xml()) for c in comms]
-
-        def call():
-            with rt.group():
-                for q in range(R):
-                    comms[q].run(progs[q], send[q], recv[q], n)  # current stream (graph capture)
-        try:
-            t, mode = _timed(call, 50, stream)
-            lat[name] = round(t * 1e6, 2)
-            lat["mode"] = mode
-        except Exception as e:
-            lat[name] = "error: %s" % str(e)[:120]
-        for c, p in zip(comms, progs):
-            c.unload(p)
-    out["allreduce_1KiB_fp16_latency_us"] = lat
-    # AllToAll (direct, N=1 two-step), 256 MiB per rank, bf16
-    S = 256 * MIB
-    n = S // 2
-    algo = P.alltoall_twostep(1, R, instances=2)
-    progs = [c.load(algo.to_xml()) for c in comms]
-    send = [synth.hashed(q, torch.arange(n, device=dev), "bfloat16") for q in range(R)]
-    recv = [torch.empty_like(x) for x in send]
-
-    def a2a():
-        with rt.group():
-            for q in range(R):
-                comms[q].run(progs[q], send[q], recv[q], n // R, stream=stream)
-    t, mode = _timed(a2a, 3, stream, graph=False)
-    ok = all(torch.equal(recv[q].view(R, -1)[p], send[p].view(R, -1)[q]) for q in (0, R - 1) for p in range(R))
-    out["alltoall_bf16_256MiB"] = {"busbw_GBps": round(busbw("alltoall", S, t, R), 2), "ms": round(t * 1e3, 3),
-                                   "ctas": sum(p.info()["thread_blocks"] for p in progs), "bit_exact": bool(ok)}
-    for c, p in zip(comms, progs):
-        c.unload(p)
-    del send, recv
-    # AllGather / ReduceScatter rings (config 5), S = 256 MiB of output (AG) / input (RS) per rank
-    nb = n // R
-    for name, algo, coll in (("allgather", P.ring_allgather(R, 1, 32), "allgather"),
-                             ("reducescatter", P.ring_reducescatter(R, 1, 32), "reducescatter")):
-        progs = [c.load(algo.to_xml()) for c in comms]
-        ins = nb if coll == "allgather" else n
-        outs = n if coll == "allgather" else nb
-        send = [synth.hashed(q, torch.arange(ins, device=dev), "bfloat16") for q in range(R)]
-        recv = [torch.empty(outs, dtype=torch.bfloat16, device=dev) for _ in range(R)]
-
-        def call():
-            with rt.group():
-                for q in range(R):
-                    comms[q].run(progs[q], send[q], recv[q], nb)
-        t, mode = _timed(call, 3, stream, graph=False)
-        if coll == "allgather":
-            ok = all(torch.equal(recv[q].view(R, -1)[p], send[p]) for q in (0, R - 1) for p in range(R))
-        else:
-            bad, _ = sampled_parity(algo, recv, nb, [0, R - 1])
-            ok = bad == 0
-        out[name + "_bf16_256MiB"] = {"busbw_GBps": round(busbw(coll, S, t, R), 2), "ms": round(t * 1e3, 3),
-                                      "instances": 32, "bit_exact": ok}
-        for c, p in zip(comms, progs):
-            c.unload(p)
-        del send, recv
-    return out
+    if os.environ.get("MSCCL_FORCE_DEVICE") or torch.cuda.device_count() < 2:
+        return None
+    peer = (dev.index + 1) % torch.cuda.device_count()
+    a = torch.empty(1 << 30, dtype=torch.uint8, device=dev)
+    b = torch.empty(1 << 30, dtype=torch.uint8, device=torch.device("cuda", peer))
+    best = 0.0
+    for _ in range(5):
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record()
+        b.copy_(a, non_blocking=True)
+        e1.record()
+        torch.cuda.synchronize()
+        best = max(best, (1 << 30) / (e0.elapsed_time(e1) / 1e3) / 1e9)
+    del a, b
+    torch.cuda.empty_cache()
+    return round(best, 1)
 
 
 def run_multi(args, rank, world, local_rank):
     import torch
-    if os.environ.get("MSCCL_FORCE_DEVICE"):  # testing the multi-process path on one GPU only
-        local_rank = int(os.environ["MSCCL_FORCE_DEVICE"])
+    forced = os.environ.get("MSCCL_FORCE_DEVICE")
+    if forced:  # testing the multi-process path on one GPU only
+        local_rank = int(forced)
     import torch.distributed as dist
     import synth
     from paper_conf_asplos_cowanmmsx23_b200 import runtime as rt
     torch.cuda.set_device(local_rank)
-    if os.environ.get("MSCCL_FORCE_DEVICE"):  # NCCL refuses two ranks on one GPU; plumbing only anyway
+    dev = torch.device("cuda", local_rank)
+    if forced:  # NCCL refuses two ranks on one GPU; plumbing only anyway
         dist.init_process_group("gloo", rank=rank, world_size=world)
     else:
-        dist.init_process_group("nccl", rank=rank, world_size=world, device_id=torch.device("cuda", local_rank))
+        dist.init_process_group("nccl", rank=rank, world_size=world, device_id=dev)
     set_params(rt, args)
-    R = world
-    algo = build_program(args, R)
     from paper_conf_asplos_cowanmmsx23_b200 import dist as mdist
     comm = mdist.init_from_process_group(local_rank)
-    comm.load(algo.to_xml())
+    R = Ranks(rt, [comm], [rank], world, world, dev)
+    R.no_register = args.no_register
+    stream = torch.cuda.current_stream()
+    nccl, nccl_note = None, None
+    if args.no_nccl:
+        nccl_note = "skipped (--no-nccl)"
+    elif forced:
+        nccl_note = "skipped: every rank is on one GPU (MSCCL_FORCE_DEVICE); NCCL refuses duplicate GPUs"
+    else:
+        try:
+            sys.path.insert(0, os.path.join(ROOT, "tools"))
+            import nccl_arm
+            nccl = nccl_arm.Nccl().init(rank, world)
+            nccl_note = "NCCL %d via ctypes (torch-bundled libnccl.so.2), default env" % nccl.version
+        except Exception as e:
+            nccl, nccl_note = None, "unavailable: %s" % str(e)[:200]
+    if args.sweep:
+        rt.set_param("MSCCL_MAX_CHANNELS", 64)
+        sweep(R, stream, args.sweep if rank == 0 else None, args.sweep_max_mib, nccl)
+        if nccl:
+            nccl.destroy()
+        comm.destroy()
+        dist.destroy_process_group()
+        return None
+    peak_peer = peer_copy_peak(rank, world, dev)
+    algo = build_program(args, world)
+    progs = R.load(algo)
     S = int(args.size_mib * MIB)
     n = S // 2
-    dev = torch.device("cuda", local_rank)
-    send = synth.hashed(rank, torch.arange(n, device=dev, dtype=torch.int64), "bfloat16")
-    recv = torch.empty(n, dtype=torch.bfloat16, device=dev)
-    stream = torch.cuda.current_stream()
+    coll = "alltoall" if args.program == "alltoall" else "allreduce"
+    count = n // world if coll == "alltoall" else n
+    send = [synth.hashed(rank, torch.arange(n, device=dev, dtype=torch.int64), "bfloat16")]
+    recv = [torch.empty(n, dtype=torch.bfloat16, device=dev)]
+    regs = register_all(R, send + recv)
+    h0 = comm.stats()["cross_direct_handshakes"]
+
+    def step():
+        R.call(progs, send, recv, count, stream)
+
     for _ in range(args.warmup):
-        comm.allreduce(send, recv, stream=stream)
+        step()
     torch.cuda.synchronize()
-    dist.barrier()
     clocks = Clocks(local_rank) if rank == 0 else None
     if clocks:
         clocks.start()
@@ -511,37 +770,53 @@ def run_multi(args, rank, world, local_rank):
     dist.barrier()
     ev0.record(stream)
     for _ in range(args.steps):
-        comm.allreduce(send, recv, stream=stream)
+        step()
     ev1.record(stream)
     torch.cuda.synchronize()
     dist.barrier()
-    t = ev0.elapsed_time(ev1) / 1e3 / args.steps
-    tt = torch.tensor([t], dtype=torch.float64)  # host tensor: works with any plumbing backend
-    if dist.get_backend() == "nccl":
-        tt = tt.to(dev)
-    dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-    t = float(tt.item())
+    t = R.tmax(ev0.elapsed_time(ev1) / 1e3 / args.steps)
     launches = rt.launch_count() - l0
     clk = clocks.stop() if clocks else None
-    # sampled parity on this rank
-    import numpy as np
-    from oracle import irparse, sampled
-    g = np.random.default_rng(1)
-    idx = np.unique(g.integers(0, n, SEED_SAMPLES))
-    want = sampled.allreduce_at(irparse.parse(algo.to_xml()), lambda r, i: synth.hashed_numpy(r, i, "bfloat16"),
-                                n, "bfloat16", "sum", idx, rank=rank)
-    got = recv[torch.from_numpy(idx).to(dev)].view(torch.int16).cpu().numpy().view(np.uint16)
-    bad = torch.tensor([int(np.count_nonzero(got != want))])
+    handshakes = comm.stats()["cross_direct_handshakes"] - h0
+    if coll == "alltoall":
+        ok = check_alltoall(R, recv, world, n)
+        bad, total = (0 if ok else 1), n
+    else:
+        bad, total = sampled_parity(algo, recv, n, [rank], local=[rank])
+    bt = torch.tensor([bad, total, handshakes], dtype=torch.int64)
     if dist.get_backend() == "nccl":
-        bad = bad.to(dev)
-    dist.all_reduce(bad)
-    res = {"t": t, "launches": launches, "clocks": clk, "parity_bad": int(bad.item()),
-           "parity_total": idx.size * R, "algo": algo, "S": S, "R": R}
+        bt = bt.to(dev)
+    dist.all_reduce(bt)
+    bad, total, handshakes = (int(x) for x in bt.tolist())
+    res = {"t": t, "coll": coll, "launches": launches, "clocks": clk, "parity_bad": bad, "parity_total": total,
+           "algo": algo, "S": S, "R": world, "peak_peer": peak_peer, "nccl_note": nccl_note,
+           "direct_handshakes": handshakes, "registered": not args.no_register}
+    if nccl is not None:
+        fn = (lambda: nccl.allreduce(send[0], recv[0], "bfloat16", stream=stream.cuda_stream)) \
+            if coll == "allreduce" else (lambda: nccl.alltoall(send[0], recv[0], "bfloat16", world,
+                                                               stream.cuda_stream))
+        tn, _ = timed(fn, args.steps, args.warmup, stream, False, R)
+        res["nccl"] = {"value": round(busbw(coll, S, tn, world), 3), "ms_per_step": round(tn * 1e3, 4),
+                       "note": nccl_note}
+    if not args.no_e2e:
+        res["e2e"] = e2e(R, send, recv, step, S, coll, world, args.steps, stream)
+    for r_ in regs:
+        r_.deregister()
+    R.unload(progs)
+    del send, recv
+    torch.cuda.empty_cache()
+    if not args.quiet_extra:
+        res["extras"] = extras(R, stream, nccl, S)
+    if rank == 0 and not args.no_cpu:
+        res["cpu_baseline"] = cpu_oracle_run(world, algo, 32 * MIB)
+    if nccl:
+        nccl.destroy()
     comm.destroy()
     dist.destroy_process_group()
     return res if rank == 0 else None
 
 
+# ----------------------------------------------------------------------------- main
 def main():
     args = parse()
     if args.impl == "reference":
@@ -553,76 +828,84 @@ def main():
     N = world if world > 1 else args.gpus
     if world > 1:
         res = run_multi(args, rank, world, local_rank)
-        if rank != 0:
+        if rank != 0 or res is None:
             return
-        R = world
     else:
         res = run_virtual(args)
-        R = args.ranks
+        if res is None:
+            return
+    R = res["R"]
     S, t, algo = res["S"], res["t"], res["algo"]
     coll = res.get("coll", "allreduce")
     value = busbw(coll, S, t, R)
-    peak, peak_src = measured_peak()
-    per_chunk = S / algo.gpus[0].i_chunks
-    nranks_launch = R if world == 1 else 1
-    if "touches" in res:
-        alg_bytes = sum(res["touches"]) * per_chunk
-    else:
-        alg_bytes = sum(simple_bytes_per_rank(algo, q, per_chunk) for q in range(R)) / R * nranks_launch
     launches_per_step = max(1, res["launches"] // args.steps)
-    achieved = alg_bytes / t / 1e9
-    traffic, prof = ncu_traffic()
-    if world > 1:
-        # one rank per GPU: the ring's bytes cross NVLink; roofline = measured peer copy 770 GB/s
-        # per direction (B200_PROFILING.md; 900 nominal). Egress per rank per step = busBW * t.
-        roof = {"bound": "nvlink", "achieved": round(value, 1), "peak": 770.0, "unit": "GB/s",
-                "frac": round(value / 770.0, 4), "traffic": None,
-                "peak_source": "measured peer copy per direction (B200_PROFILING.md)",
-                "kernel": "mscclInterpreter<bf16,sum>", "algorithmic_bytes_per_launch": int(S * 2 * (R - 1) / R),
-                "launch_ms": round(t * 1e3 / launches_per_step, 4)}
-    else:
-        # All R ranks run in one launch on one GPU: the HBM bytes any implementation must move are
-        # every rank's input read once and its output written once.
-        launch_s = t / launches_per_step
-        compulsory = 2 * S * R
-        hbm_achieved = compulsory / launch_s / 1e9
-        l2peak, l2src = l2_peak()
-        is_default = (args.program, args.instances, args.channels, args.slot_kib, args.threads, args.protocol) == \
-            ("ring", 32, 1, 256, 256, "Simple")
-        roof = {"bound": "hbm", "achieved": round(hbm_achieved, 1), "peak": peak, "unit": "GB/s",
-                "frac": round(hbm_achieved / peak, 4), "traffic": traffic if is_default else None,
-                "peak_source": peak_src,
-                "kernel": "mscclInterpreter<bf16,%s,Simple>" % ("copy" if coll == "alltoall" else "sum"),
-                "algorithmic_bytes_per_launch": int(compulsory), "launch_ms": round(launch_s * 1e3, 4),
-                "note": "algorithmic = compulsory HBM bytes of one launch covering all %d ranks: every input read "
-                        "once + every output written once (2 S R); traffic = ncu dram read+write bytes per launch "
-                        "(profiles/ncu_summary.json, default config only)" % R,
-                "l2": {"touched_bytes_per_launch": int(alg_bytes), "achieved": round(achieved, 1),
-                       "peak": l2peak, "frac": round(achieved / l2peak, 4) if l2peak else None,
-                       "peak_source": l2src,
-                       "note": "touched = the program's per-instruction operand bytes (send 2, recv 2, copy 2, "
-                               "reduce/rrc/rrs 3, rrcs 4, rcs 3 chunks; a direct recv 0, a direct rcs 2), i.e. "
-                               "the L2-level traffic of the interpreter; FIFO slots live mostly in L2"},
-                "direct_placement": res.get("direct")}
     out = {
         "metric": metric_name(coll), "value": round(value, 3), "unit": "GB/s", "n_gpus": N,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 4),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
         "data": "synthetic (counter-based uniform[-1,1) bf16, seed 20230325+rank)",
         "config": config_dict(args, R, N),
-        "frac_nvlink": round(value / 900.0, 4),
-        "roofline": roof,
-        "gpu_launches": res["launches"],
-        "parity": {"sampled_outputs": res["parity_total"], "mismatches": res["parity_bad"],
-                   "against": "oracle reduction trees (oracle/sampled.py), bit-exact"},
-        "clocks": res["clocks"],
     }
+    if world > 1:
+        # one rank per GPU: the bytes cross NVLink. Egress per rank per step = busBW * t, so
+        # busBW is the achieved per-direction link bandwidth.
+        pk = res.get("peak_peer")
+        peak, src = (pk, "measured peer copy (1 GiB cudaMemcpyPeer, this box)") if pk else \
+            (770.0, "fallback: B200_PROFILING.md measured peer copy per direction (no 2nd GPU to measure)")
+        out["roofline"] = {"bound": "nvlink", "achieved": round(value, 1), "peak": peak, "unit": "GB/s",
+                           "frac": round(value / peak, 4), "traffic": None, "peak_source": src,
+                           "frac_nominal_900": round(value / NVLINK_NOMINAL, 4),
+                           "kernel": "mscclInterpreter<bf16,%s,Simple>" % ("copy" if coll == "alltoall" else "sum"),
+                           "algorithmic_bytes_per_launch": int(S * (2 if coll == "allreduce" else 1) * (R - 1) / R),
+                           "launch_ms": round(t * 1e3 / launches_per_step, 4)}
+        out["frac_nvlink"] = round(value / NVLINK_NOMINAL, 4)
+        out["direct_placement"] = {"registered_buffers": res["registered"],
+                                   "cross_launch_handshakes": res["direct_handshakes"]}
+        out["nccl"] = res.get("nccl", {"note": res.get("nccl_note")})
+    else:
+        # All R virtual ranks run in one launch on one GPU: the HBM bytes any implementation
+        # must move are every rank's input read once and its output written once.
+        peak, peak_src = measured_peak()
+        per_chunk = S / algo.gpus[0].i_chunks
+        alg_bytes = sum(res["touches"]) * per_chunk
+        launch_s = t / launches_per_step
+        compulsory = 2 * S * R
+        hbm_achieved = compulsory / launch_s / 1e9
+        achieved = alg_bytes / launch_s / 1e9
+        traffic, prof = ncu_traffic()
+        l2peak, l2src = l2_peak()
+        is_default = (args.program, args.instances, args.channels, args.slot_kib, args.threads, args.protocol) == \
+            ("ring", 32, 1, 256, 256, "Simple")
+        out["roofline"] = {
+            "bound": "hbm", "achieved": round(hbm_achieved, 1), "peak": peak, "unit": "GB/s",
+            "frac": round(hbm_achieved / peak, 4), "traffic": traffic if is_default else None,
+            "peak_source": peak_src,
+            "kernel": "mscclInterpreter<bf16,%s,Simple>" % ("copy" if coll == "alltoall" else "sum"),
+            "algorithmic_bytes_per_launch": int(compulsory), "launch_ms": round(launch_s * 1e3, 4),
+            "note": "algorithmic = compulsory HBM bytes of one launch covering all %d ranks: every input read "
+                    "once + every output written once (2 S R); traffic = ncu dram read+write bytes per launch "
+                    "(profiles/ncu_summary.json, default config only)" % R,
+            "l2": {"touched_bytes_per_launch": int(alg_bytes), "achieved": round(achieved, 1),
+                   "peak": l2peak, "frac": round(achieved / l2peak, 4) if l2peak else None,
+                   "peak_source": l2src,
+                   "note": "touched = the program's per-instruction operand bytes (send 2, recv 2, copy 2, "
+                           "reduce/rrc/rrs 3, rrcs 4, rcs 3 chunks; a direct recv 0, a direct rcs 2), i.e. "
+                           "the L2-level traffic of the interpreter; FIFO slots live mostly in L2"},
+            "direct_placement": res.get("direct")}
+        out["nccl"] = {"note": "skipped: one GPU (NCCL cannot run 8 ranks on one device); the NCCL arm runs "
+                               "under torchrun with N > 1"}
+    out["gpu_launches"] = res["launches"]
+    out["parity"] = {"sampled_outputs": res["parity_total"], "mismatches": res["parity_bad"],
+                     "against": "oracle reduction trees (oracle/sampled.py), bit-exact"}
+    out["clocks"] = res["clocks"]
     if "e2e" in res:
         out["e2e"] = res["e2e"]
     if "extras" in res:
         out["extras"] = res["extras"]
     if world == 1 and not args.no_cpu:
-        out["cpu_baseline"] = cpu_oracle_run(args, R, algo, 32 * MIB)
+        out["cpu_baseline"] = cpu_oracle_run(R, algo, 32 * MIB)
+    elif "cpu_baseline" in res:
+        out["cpu_baseline"] = res["cpu_baseline"]
     print(json.dumps(out), flush=True)
 
 

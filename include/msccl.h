@@ -92,6 +92,13 @@ mscclResult_t mscclCommConnect(mscclComm_t comm, const void* allHandles);
 mscclResult_t mscclCommDestroy(mscclComm_t comm);
 
 mscclResult_t mscclCommCount(const mscclComm_t comm, int* count);
+
+/* Counters of this rank (synchronises with the device to read them), up to n of:
+ * [0] cross-launch ready handshakes in which a sender of this rank found a reachable
+ *     destination and stored directly into a peer (device-side count, reading R15b);
+ * [1] launches with one-launch direct placement (every rank in the launch, reading R15);
+ * [2] launches in which this rank published a reachable destination (cross-launch mode). */
+mscclResult_t mscclCommGetStats(mscclComm_t comm, int64_t* stats, int n);
 mscclResult_t mscclCommUserRank(const mscclComm_t comm, int* rank);
 mscclResult_t mscclCommCuDevice(const mscclComm_t comm, int* device);
 

@@ -73,6 +73,8 @@ struct RankArgs {
   char* const* regMap;
   int32_t regMax;
   int32_t directMask;
+  unsigned long long* stats;  // this rank's counters (region): [0] cross-launch handshakes that
+                              // resolved a direct destination (mscclCommGetStats)
 };
 
 struct KernelArgs {

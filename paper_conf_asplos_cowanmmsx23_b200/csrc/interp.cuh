@@ -699,11 +699,18 @@ __device__ __forceinline__ char* resolveRef(const RankArgs& ra, int peer, uint64
 __device__ __forceinline__ bool waitReady(const Ctx& c, const DevTB& tb) {
   uint64_t seen;
   if (!waitGE(tb.sendReady, c.sendL, c.a->sysScope != 0, c, seen)) return false;
+  bool any = false;
 #pragma unroll
   for (int b = 0; b < 3; b++) {
     const uint64_t ref = *(volatile const uint64_t*)(tb.sendReady + 1 + b);
     c.peerDst[b] = resolveRef(*c.ra, tb.sendPeer, ref);
+    if (ref && !c.peerDst[b]) {  // published but not mapped here: the receiver expects a direct store
+      raiseAbort(*c.a);          // that this sender cannot make (registration not connected)
+      return false;
+    }
+    any = any || c.peerDst[b] != nullptr;
   }
+  if (any) atomicAdd(c.ra->stats, 1ull);
   return true;
 }
 

@@ -118,6 +118,7 @@ struct mscclComm {
   std::vector<mscclProgram*> programs;
   std::string lastError;
   int maxCoResident = 0;
+  uint64_t launchesDirect1 = 0, launchesDirect2 = 0;  // launches this rank took part in, by direct mode
   std::vector<mscclReg*> regs;         // by index (nullptr = free)
   char** dRegMap = nullptr;            // device [nranks][regMax]: peers' registered buffers, mapped here
   std::vector<char*> hRegMap;
@@ -143,6 +144,7 @@ struct mscclComm {
     return flagsOff + (((size_t)kind * nranks + peer) * prm.maxChannels + ch) * MSCCL_FLAG_STRIDE * sizeof(uint64_t);
   }
   size_t abortOff() const { return flagOff(5, 0, 0); }
+  size_t statsOff() const { return abortOff() + 128; }
 };
 
 struct mscclProgram {
@@ -210,7 +212,7 @@ mscclResult_t allocRegion(mscclComm* c) {
   DeviceGuard g(c->dev);
   c->fifoBytes = c->fifoBase(3);
   c->flagsOff = c->fifoBytes;
-  c->regionBytes = c->abortOff() + 256;
+  c->regionBytes = c->statsOff() + 128;
   CUDACHECK(c, cudaMalloc(&c->region, c->regionBytes));
   CUDACHECK(c, cudaMemset(c->region, 0, c->regionBytes));
   c->hRegMap.assign((size_t)c->nranks * c->prm.regMax, nullptr);
@@ -473,6 +475,7 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
       ra.abortFlag = (uint32_t*)(cl->comm->region + cl->comm->abortOff());
       ra.hostAbort = cl->comm->hostAbortDev;
       ra.regMap = cl->comm->dRegMap;
+      ra.stats = (unsigned long long*)(cl->comm->region + cl->comm->statsOff());
       ra.regMax = (int32_t)cl->comm->prm.regMax;
       if (direct == 1) {
         ra.directMask = 7;
@@ -487,6 +490,8 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
       }
       cta += p->nTB;
       if (cl->comm->sysScope) ka.sysScope = 1;
+      if (direct == 1) cl->comm->launchesDirect1++;
+      if (direct == 2 && ra.directMask) cl->comm->launchesDirect2++;
     }
     if (cta == 0) continue;
     const void* fn = p0->hasReduce ? interpreterKernel(v[0]->dtype, v[0]->op, ka.proto)
@@ -906,6 +911,16 @@ mscclResult_t mscclDebugDirectPlacement(const char* ir, size_t irBytes, int rank
     setErr(nullptr, mscclInvalidProgram, e.what());
     return mscclInvalidProgram;
   }
+  return mscclSuccess;
+}
+
+mscclResult_t mscclCommGetStats(mscclComm_t c, int64_t* stats, int n) {
+  if (!c || !stats || n < 1) return mscclInvalidArgument;
+  DeviceGuard g(c->dev);
+  uint64_t dev[1] = {0};
+  CUDACHECK(c, cudaMemcpy(dev, c->region + c->statsOff(), sizeof(dev), cudaMemcpyDeviceToHost));
+  const int64_t v[3] = {(int64_t)dev[0], (int64_t)c->launchesDirect1, (int64_t)c->launchesDirect2};
+  for (int i = 0; i < n && i < 3; i++) stats[i] = v[i];
   return mscclSuccess;
 }
 

@@ -56,6 +56,7 @@ SIGNATURES = {
     "mscclSetParam": (_i, [_c.c_char_p, _i64]),
     "mscclGetParam": (_i, [_c.c_char_p, _c.POINTER(_i64)]),
     "mscclLaunchCount": (_c.c_uint64, []),
+    "mscclCommGetStats": (_i, [_vp, _c.POINTER(_i64), _i]),
     "mscclCommRegister": (_i, [_vp, _vp, _sz, _c.POINTER(_vp)]),
     "mscclRegExport": (_i, [_vp, _vp]),
     "mscclRegConnect": (_i, [_vp, _vp]),
@@ -251,6 +252,12 @@ class Comm:
         v = _i()
         _check(lib.mscclCommGetAsyncError(self.handle, _c.byref(v)))
         return v.value
+
+    def stats(self):
+        """mscclCommGetStats: {"cross_direct_handshakes", "launches_direct1", "launches_direct2"}."""
+        v = (_i64 * 3)()
+        _check(lib.mscclCommGetStats(self.handle, v, 3), self.handle)
+        return {"cross_direct_handshakes": v[0], "launches_direct1": v[1], "launches_direct2": v[2]}
 
     def last_error(self):
         return lib.mscclGetLastError(self.handle).decode(errors="replace")
