@@ -57,7 +57,8 @@ def parse():
     ap.add_argument("--impl", default="msccl", choices=["msccl", "reference"])
     ap.add_argument("--ranks", type=int, default=8, help="virtual ranks when N=1")
     ap.add_argument("--size-mib", type=float, default=256.0, help="bytes per rank (MiB)")
-    ap.add_argument("--program", default="ring", choices=["ring", "allpairs", "oneshot", "alltoall"])
+    ap.add_argument("--program", default="ring",
+                    choices=["ring", "allpairs", "oneshot", "alltoall", "allgather", "reducescatter"])
     ap.add_argument("--channels", type=int, default=1)
     ap.add_argument("--instances", type=int, default=32)
     ap.add_argument("--protocol", default="Simple")
@@ -172,7 +173,27 @@ def build_program(args, R):
         return P.allpairs_allreduce(R, instances=args.instances, protocol=args.protocol)
     if args.program == "oneshot":
         return P.oneshot_allreduce(R, instances=args.instances, protocol=args.protocol)
+    if args.program == "allgather":
+        return P.ring_allgather(R, args.channels, args.instances, protocol=args.protocol)
+    if args.program == "reducescatter":
+        return P.ring_reducescatter(R, args.channels, args.instances, protocol=args.protocol)
     return P.alltoall_twostep(1, R, instances=args.instances, protocol=args.protocol)
+
+
+def coll_of(program):
+    return {"alltoall": "alltoall", "allgather": "allgather", "reducescatter": "reducescatter"}.get(program,
+                                                                                                  "allreduce")
+
+
+def shapes(coll, n, W):
+    """(send elems, recv elems, count) for S = n elements per rank (S = the larger buffer)."""
+    if coll == "allgather":
+        return n // W, n, n // W
+    if coll == "reducescatter":
+        return n, n // W, n // W
+    if coll == "alltoall":
+        return n, n, n // W
+    return n, n, n
 
 
 def nop_ir(R):
@@ -254,6 +275,8 @@ def run_reference(args):
 def metric_name(coll="allreduce"):
     if coll == "alltoall":
         return "AllToAll busBW (GB/s), direct MSCCL-IR (two-step N=1), bf16"
+    if coll in ("allgather", "reducescatter"):
+        return "%s busBW (GB/s), ring MSCCL-IR, bf16" % {"allgather": "AllGather", "reducescatter": "ReduceScatter"}[coll]
     return "AllReduce busBW (GB/s), ring MSCCL-IR, bf16"
 
 
@@ -361,10 +384,16 @@ class Ranks:
             dist.barrier()
 
 
+def cur():
+    """The current CUDA stream handle (the capture stream while a graph is being captured)."""
+    import torch
+    return torch.cuda.current_stream().cuda_stream
+
+
 def timed(fn, iters, warmup, stream, graph, R):
     """Mean device time per call of fn() (CUDA events on `stream`, synchronised on both
-    sides, max over ranks). graph=True captures `iters` calls into one CUDA graph and times
-    its replay. Returns (seconds, mode)."""
+    sides, max over ranks). fn() must issue its work on the current stream. graph=True
+    captures `iters` calls into one CUDA graph and times its replay. Returns (seconds, mode)."""
     import torch
     for _ in range(warmup):
         fn()
@@ -374,7 +403,7 @@ def timed(fn, iters, warmup, stream, graph, R):
     if graph:
         try:
             g = torch.cuda.CUDAGraph()
-            with torch.cuda.graph(g, stream=stream):
+            with torch.cuda.graph(g):   # torch's capture stream; fn() issues on the current stream
                 for _ in range(iters):
                     fn()
             g.replay()
@@ -421,15 +450,14 @@ def extras(R, stream, nccl=None, S=256 * MIB):
         else:
             progs = R.load(algo, 0, 1 << 20)
         try:
-            t, mode = timed(lambda: R.call(progs, send, recv, n, stream), 50, 5, stream, True, R)
+            t, mode = timed(lambda: R.call(progs, send, recv, n), 50, 5, stream, True, R)
             lat[name] = round(t * 1e6, 2)
             lat["mode"] = mode
         except Exception as e:
             lat[name] = "error: %s" % str(e)[:160]
         R.unload(progs)
     if nccl is not None:
-        t, mode = timed(lambda: nccl.allreduce(send[0], recv[0], "float16", stream=stream.cuda_stream), 50, 5,
-                        stream, True, R)
+        t, mode = timed(lambda: nccl.allreduce(send[0], recv[0], "float16", stream=cur()), 50, 5, stream, True, R)
         lat["nccl_allreduce"] = round(t * 1e6, 2)
     lat["note"] = ("floor_nop = an MSCCL-IR program of one nop per rank: cooperative launch + prologue + "
                    "epilogue under graph replay; the collective latencies are read against it")
@@ -446,7 +474,7 @@ def extras(R, stream, nccl=None, S=256 * MIB):
         send = [synth.hashed(q, torch.arange(ins, device=R.dev), "bfloat16") for q in R.ranks]
         recv = [torch.empty(outs, dtype=torch.bfloat16, device=R.dev) for _ in R.ranks]
         regs = register_all(R, send + recv)
-        t, mode = timed(lambda: R.call(progs, send, recv, cnt, stream), 5, 2, stream, False, R)
+        t, mode = timed(lambda: R.call(progs, send, recv, cnt), 5, 2, stream, False, R)
         if coll == "alltoall":
             ok = check_alltoall(R, recv, W, n)
         elif coll == "allgather":
@@ -458,10 +486,9 @@ def extras(R, stream, nccl=None, S=256 * MIB):
         ent = {"busbw_GBps": round(busbw(coll, S, t, W), 2), "ms": round(t * 1e3, 3),
                "ctas_per_rank": int(progs[0].info()["thread_blocks"]), "bit_exact": R.all_ok(ok)}
         if nccl is not None:
-            fn = {"alltoall": lambda: nccl.alltoall(send[0], recv[0], "bfloat16", W, stream.cuda_stream),
-                  "allgather": lambda: nccl.allgather(send[0], recv[0], "bfloat16", stream.cuda_stream),
-                  "reducescatter": lambda: nccl.reducescatter(send[0], recv[0], "bfloat16", "sum",
-                                                              stream.cuda_stream)}[coll]
+            fn = {"alltoall": lambda: nccl.alltoall(send[0], recv[0], "bfloat16", W, cur()),
+                  "allgather": lambda: nccl.allgather(send[0], recv[0], "bfloat16", cur()),
+                  "reducescatter": lambda: nccl.reducescatter(send[0], recv[0], "bfloat16", "sum", cur())}[coll]
             tn, _ = timed(fn, 5, 2, stream, False, R)
             ent["nccl_busbw_GBps"] = round(busbw(coll, S, tn, W), 2)
         out["%s_bf16_%dMiB" % (coll, S // MIB)] = ent
@@ -531,11 +558,11 @@ def sweep(R, stream, path, max_mib, nccl=None):
             regs = register_all(R, send + recv)
             per = (n // W) * 2 if coll == "alltoall" else size   # selection bytes (count * w)
             chosen = next(a for a, lo, hi, _ in sets if lo <= per and (hi == 0 or per < hi))
-            impls = [("msccl", lambda: R.coll(coll, send, recv, stream))]
+            impls = [("msccl", lambda: R.coll(coll, send, recv))]
             if nccl is not None:
-                impls.append(("nccl", (lambda: nccl.allreduce(send[0], recv[0], "bfloat16", stream=stream.cuda_stream))
+                impls.append(("nccl", (lambda: nccl.allreduce(send[0], recv[0], "bfloat16", stream=cur()))
                               if coll == "allreduce" else
-                              (lambda: nccl.alltoall(send[0], recv[0], "bfloat16", W, stream.cuda_stream))))
+                              (lambda: nccl.alltoall(send[0], recv[0], "bfloat16", W, cur()))))
             for impl, fn in impls:
                 for graph in (False, True):
                     iters = 50 if size <= 256 * MIB else 20
@@ -596,12 +623,12 @@ def run_virtual(args):
     progs = [c.load(ir_text) for c in comms]
     direct = rt.get_param("MSCCL_DIRECT") != 0 and args.protocol == "Simple"
     touches = [p.touches(direct) for p in progs]
-    idx = torch.arange(n, device=dev, dtype=torch.int64)
+    coll = coll_of(args.program)
+    ns, nr, count = shapes(coll, n, W)
+    idx = torch.arange(ns, device=dev, dtype=torch.int64)
     send = [synth.hashed(q, idx, "bfloat16") for q in range(W)]
     del idx
-    recv = [torch.empty(n, dtype=torch.bfloat16, device=dev) for _ in range(W)]
-    coll = "alltoall" if args.program == "alltoall" else "allreduce"
-    count = n // W if coll == "alltoall" else n
+    recv = [torch.empty(nr, dtype=torch.bfloat16, device=dev) for _ in range(W)]
 
     def step():
         R.call(progs, send, recv, count, stream)
@@ -629,8 +656,11 @@ def run_virtual(args):
     if coll == "alltoall":
         ok = check_alltoall(R, recv, W, n)
         bad, total = (0 if ok else 1), 2 * n
+    elif coll == "allgather":
+        ok = check_allgather(R, recv, W, count)
+        bad, total = (0 if ok else 1), 2 * n
     else:
-        bad, total = sampled_parity(algo, recv, n, [0, W - 1])
+        bad, total = sampled_parity(algo, recv, count, [0, W - 1])
     res = {"t": t, "coll": coll, "launches": launches, "clocks": clk, "parity_bad": bad, "parity_total": total,
            "algo": algo, "S": S, "R": W, "touches": touches, "direct": direct}
     if not args.no_e2e:
@@ -792,9 +822,8 @@ def run_multi(args, rank, world, local_rank):
            "algo": algo, "S": S, "R": world, "peak_peer": peak_peer, "nccl_note": nccl_note,
            "direct_handshakes": handshakes, "registered": not args.no_register}
     if nccl is not None:
-        fn = (lambda: nccl.allreduce(send[0], recv[0], "bfloat16", stream=stream.cuda_stream)) \
-            if coll == "allreduce" else (lambda: nccl.alltoall(send[0], recv[0], "bfloat16", world,
-                                                               stream.cuda_stream))
+        fn = (lambda: nccl.allreduce(send[0], recv[0], "bfloat16", stream=cur())) \
+            if coll == "allreduce" else (lambda: nccl.alltoall(send[0], recv[0], "bfloat16", world, cur()))
         tn, _ = timed(fn, args.steps, args.warmup, stream, False, R)
         res["nccl"] = {"value": round(busbw(coll, S, tn, world), 3), "ms_per_step": round(tn * 1e3, 4),
                        "note": nccl_note}
@@ -866,10 +895,11 @@ def main():
         # All R virtual ranks run in one launch on one GPU: the HBM bytes any implementation
         # must move are every rank's input read once and its output written once.
         peak, peak_src = measured_peak()
-        per_chunk = S / algo.gpus[0].i_chunks
+        ns, nr, _ = shapes(coll, S // 2, R)
+        per_chunk = ns * 2 / algo.gpus[0].i_chunks       # E * w: every buffer's chunk size
         alg_bytes = sum(res["touches"]) * per_chunk
         launch_s = t / launches_per_step
-        compulsory = 2 * S * R
+        compulsory = (ns + nr) * 2 * R                     # inputs read once + outputs written once
         hbm_achieved = compulsory / launch_s / 1e9
         achieved = alg_bytes / launch_s / 1e9
         traffic, prof = ncu_traffic()
@@ -883,7 +913,7 @@ def main():
             "kernel": "mscclInterpreter<bf16,%s,Simple>" % ("copy" if coll == "alltoall" else "sum"),
             "algorithmic_bytes_per_launch": int(compulsory), "launch_ms": round(launch_s * 1e3, 4),
             "note": "algorithmic = compulsory HBM bytes of one launch covering all %d ranks: every input read "
-                    "once + every output written once (2 S R); traffic = ncu dram read+write bytes per launch "
+                    "once + every output written once (2 S R for AllReduce); traffic = ncu dram read+write bytes per launch "
                     "(profiles/ncu_summary.json, default config only)" % R,
             "l2": {"touched_bytes_per_launch": int(alg_bytes), "achieved": round(achieved, 1),
                    "peak": l2peak, "frac": round(achieved / l2peak, 4) if l2peak else None,
