@@ -285,11 +285,15 @@ def config_dict(args, R, N):
         base = {"ring": "largest single-GPU analogue of BASELINE configs[1] (ring AllReduce, bf16)",
                 "allpairs": "BASELINE configs[2] shape (all-pairs AllReduce)",
                 "oneshot": "BASELINE configs[2] shape (one-shot AllReduce)",
-                "alltoall": "BASELINE configs[3] shape (AllToAll)"}[args.program]
+                "alltoall": "BASELINE configs[3] shape (AllToAll)",
+                "allgather": "BASELINE configs[4] shape (ring AllGather)",
+                "reducescatter": "BASELINE configs[4] shape (ring ReduceScatter)"}[args.program]
         mode = "%d virtual ranks on 1 B200 (HBM-bound)" % R
     else:
         base = {"ring": "BASELINE configs[1]: ring AllReduce, bf16", "allpairs": "all-pairs AllReduce",
-                "oneshot": "one-shot AllReduce", "alltoall": "BASELINE configs[3]: AllToAll"}[args.program]
+                "oneshot": "one-shot AllReduce", "alltoall": "BASELINE configs[3]: AllToAll",
+                "allgather": "BASELINE configs[4]: ring AllGather", "reducescatter": "BASELINE configs[4]: ring "
+                "ReduceScatter"}[args.program]
         mode = "%d B200, 1 process per GPU, CUDA IPC over NVLink" % N
     return {"workload": "%s -- MSCCL-IR %s, %d channel(s) x %d instance(s), %s protocol, %s, %d MiB per rank"
                         % (base, args.program, args.channels, args.instances, args.protocol, mode,
@@ -777,10 +781,10 @@ def run_multi(args, rank, world, local_rank):
     progs = R.load(algo)
     S = int(args.size_mib * MIB)
     n = S // 2
-    coll = "alltoall" if args.program == "alltoall" else "allreduce"
-    count = n // world if coll == "alltoall" else n
-    send = [synth.hashed(rank, torch.arange(n, device=dev, dtype=torch.int64), "bfloat16")]
-    recv = [torch.empty(n, dtype=torch.bfloat16, device=dev)]
+    coll = coll_of(args.program)
+    ns, nr, count = shapes(coll, n, world)
+    send = [synth.hashed(rank, torch.arange(ns, device=dev, dtype=torch.int64), "bfloat16")]
+    recv = [torch.empty(nr, dtype=torch.bfloat16, device=dev)]
     regs = register_all(R, send + recv)
     h0 = comm.stats()["cross_direct_handshakes"]
 
@@ -811,8 +815,11 @@ def run_multi(args, rank, world, local_rank):
     if coll == "alltoall":
         ok = check_alltoall(R, recv, world, n)
         bad, total = (0 if ok else 1), n
+    elif coll == "allgather":
+        ok = check_allgather(R, recv, world, count)
+        bad, total = (0 if ok else 1), n
     else:
-        bad, total = sampled_parity(algo, recv, n, [rank], local=[rank])
+        bad, total = sampled_parity(algo, recv, count, [rank], local=[rank])
     bt = torch.tensor([bad, total, handshakes], dtype=torch.int64)
     if dist.get_backend() == "nccl":
         bt = bt.to(dev)
@@ -822,8 +829,10 @@ def run_multi(args, rank, world, local_rank):
            "algo": algo, "S": S, "R": world, "peak_peer": peak_peer, "nccl_note": nccl_note,
            "direct_handshakes": handshakes, "registered": not args.no_register}
     if nccl is not None:
-        fn = (lambda: nccl.allreduce(send[0], recv[0], "bfloat16", stream=cur())) \
-            if coll == "allreduce" else (lambda: nccl.alltoall(send[0], recv[0], "bfloat16", world, cur()))
+        fn = {"allreduce": lambda: nccl.allreduce(send[0], recv[0], "bfloat16", stream=cur()),
+              "alltoall": lambda: nccl.alltoall(send[0], recv[0], "bfloat16", world, cur()),
+              "allgather": lambda: nccl.allgather(send[0], recv[0], "bfloat16", cur()),
+              "reducescatter": lambda: nccl.reducescatter(send[0], recv[0], "bfloat16", "sum", cur())}[coll]
         tn, _ = timed(fn, args.steps, args.warmup, stream, False, R)
         res["nccl"] = {"value": round(busbw(coll, S, tn, world), 3), "ms_per_step": round(tn * 1e3, 4),
                        "note": nccl_note}

@@ -24,7 +24,13 @@ OPS = {
     "rrs":  (True,  True,  True,  False, True),    # send(recv (+) src)
     "rrcs": (True,  True,  True,  True,  True),    # v = recv (+) src; dst <- v; send(v)
     "rcs":  (True,  True,  False, True,  False),   # v = recv; dst <- v; send(v)
+    # multimem ops (reading R23): src/dst name the same chunk on
+    # EVERY rank of the group (NVLS multicast address); no connection is used
+    "mrd":  (False, False, True,  True,  True),    # dst_q <- (+)_p src_p            (ld_reduce)
+    "mst":  (False, False, True,  True,  False),   # dst_p <- src_q for every p      (st)
+    "mrs":  (False, False, True,  True,  True),    # v = (+)_p src_p; dst_p <- v     (ld_reduce + st)
 }
+MULTIMEM = ("mrd", "mst", "mrs")
 BUFS = ("i", "o", "s")
 COLLS = ("allreduce", "allgather", "reducescatter", "alltoall", "custom")
 PROTOS = ("Simple", "LL", "LL128")
@@ -65,6 +71,18 @@ class Step:
     @property
     def reduces(self):
         return OPS[self.op][4]
+
+    @property
+    def multimem(self):
+        return self.op in MULTIMEM
+
+    @property
+    def reads_all(self):      # reads src on every rank
+        return self.op in ("mrd", "mrs")
+
+    @property
+    def writes_all(self):     # writes dst on every rank
+        return self.op in ("mst", "mrs")
 
 
 @dataclass

@@ -90,3 +90,30 @@ def poison(dtype, n):
     if dtype == "bfloat16":
         return np.full(n, 0x7FC1, dtype=np.uint16)
     return np.full(n, np.iinfo(storage(dtype)).max, dtype=storage(dtype))
+
+
+# ---------------------------------------------------------------- multimem reduction (N2)
+MULTIMEM_OPS = ("sum", "max", "min")
+
+
+def mreduce(vals, op, dtype):
+    """The value a multimem reduce returns for one element over the group's copies
+    (reading R23): the ranks' values folded in ascending rank
+    order; fp16/bf16 sums accumulate in fp32 and round ONCE to the dtype (the switch's
+    .acc::f32 reduction), fp32/fp64 sums round per add in the dtype, integers wrap, max/min
+    are exact. There is no multimem product (P:L908-909 names no operator; PTX multimem
+    has add/min/max only), so prod is rejected."""
+    if op not in MULTIMEM_OPS:
+        raise ValueError("multimem reduction supports sum/max/min, not %r" % op)
+    if dtype in ("bfloat16", "float16"):
+        w = [bf16_to_f32(v) if dtype == "bfloat16" else np.asarray(v, dtype=np.float16).astype(np.float32)
+             for v in vals]
+        acc = w[0].copy()
+        for x in w[1:]:
+            acc = _apply(op, acc, x).astype(np.float32)
+        return f32_to_bf16(acc) if dtype == "bfloat16" else acc.astype(np.float16)
+    acc = np.asarray(vals[0], dtype=storage(dtype)).copy()
+    for x in vals[1:]:
+        with np.errstate(over="ignore"):
+            acc = _apply(op, acc, np.asarray(x, dtype=storage(dtype))).astype(storage(dtype))
+    return acc

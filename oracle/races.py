@@ -23,6 +23,13 @@ Happens-before = transitive closure of
 FIFO-capacity edges (the (k-s)-th receive before the k-th send, §6.1) are
 left out on purpose: the verdict then holds for every slot count s >= 1.
 
+Multimem ops (mrd / mst / mrs, reading R23) read or write the same chunk on
+EVERY rank. Their thread block b synchronises with thread block b of every other rank at
+its start and its end (the group barrier of the runtime). So for every pair of ranks p, q,
+the start of (p, b) happens before the first instruction of (q, b), and the last
+instruction of (q, b) happens before the end of (p, b). Start and end are extra events
+with no accesses.
+
 One pipeline iteration is enough. Tiles of different iterations touch disjoint elements
 (reading R3), and every edge goes forward in time: program order leads from tile t to
 t+1, and dependency and message edges stay inside one tile (V7 makes the k-th message the
@@ -66,12 +73,25 @@ def _canon(algo, buf, alias):
     return buf
 
 
+def _multimem_groups(algo):
+    """thread block id -> [(rank, steps)] of the blocks that hold multimem ops."""
+    out = defaultdict(list)
+    for g in algo.gpus:
+        for tb in g.tbs:
+            if tb.steps and any(st.multimem for st in tb.steps):
+                out[tb.id].append((g.id, len(tb.steps)))
+    return out
+
+
 def _events(algo):
     ev = []
     for g in algo.gpus:
         for tb in g.tbs:
             for s, st in enumerate(tb.steps):
                 ev.append((g.id, tb.id, s))
+    for b, members in _multimem_groups(algo).items():
+        for (p, _) in members:
+            ev += [("B", p, b), ("E", p, b)]
     return ev
 
 
@@ -110,6 +130,14 @@ def happens_before(algo):
     for (sends, recvs) in _connections(algo).values():
         for a, b in zip(sends, recvs):
             edge(a, b)                                                     # k-th send -> k-th recv
+    for b, members in _multimem_groups(algo).items():                     # group barriers (R23)
+        for (p, n) in members:
+            edge(("B", p, b), (p, b, 0))
+            edge((p, b, n - 1), ("E", p, b))
+            for (q, m) in members:
+                if q != p:
+                    edge(("B", p, b), (q, b, 0))
+                    edge((q, b, m - 1), ("E", p, b))
     anc = [0] * len(ev)
     q = deque(i for i in range(len(ev)) if indeg[i] == 0)
     done = 0
@@ -138,6 +166,14 @@ def accesses(algo, alias=False, direct=None):
         for tb in g.tbs:
             for s, st in enumerate(tb.steps):
                 e = (q, tb.id, s)
+                if st.multimem:                        # the same chunk on every rank (R23)
+                    for p in range(algo.ngpus):
+                        for j in range(st.cnt):
+                            if st.reads_all or p == q:
+                                acc[e].append((p, _canon(algo, st.srcbuf, alias), st.srcoff + j, "r"))
+                            if st.writes_all or p == q:
+                                acc[e].append((p, _canon(algo, st.dstbuf, alias), st.dstoff + j, "w"))
+                    continue
                 if st.reads_src:
                     for j in range(st.cnt):
                         acc[e].append((q, _canon(algo, st.srcbuf, alias), st.srcoff + j, "r"))

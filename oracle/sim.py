@@ -141,7 +141,25 @@ class NumericDomain:
     def _len(self, buf, k):
         return self.geo.span(buf, k)[1]
 
+    def _multimem(self, q, st, j, t):
+        """mrd / mst / mrs (reading R23): the same chunk span on every rank's buffer."""
+        L = min(self._len(st.srcbuf, st.srcoff + j), self._len(st.dstbuf, st.dstoff + j))
+        a = t * self.T
+        m = max(0, min(a + self.T, L) - a)
+        s0 = self.geo.span(st.srcbuf, st.srcoff + j)[0] + a
+        d0 = self.geo.span(st.dstbuf, st.dstoff + j)[0] + a
+        if st.reads_all:
+            v = nm.mreduce([b[st.srcbuf][s0:s0 + m].copy() for b in self.bufs], self.op, self.dtype)
+        else:
+            v = self.bufs[q][st.srcbuf][s0:s0 + m].copy()
+        for p, b in enumerate(self.bufs):
+            if st.writes_all or p == q:
+                b[st.dstbuf][d0:d0 + m] = v
+        return None
+
     def exec_piece(self, q, st, j, t, incoming):
+        if st.multimem:
+            return self._multimem(q, st, j, t)
         B = self.bufs[q]
         lens = []
         if st.reads_src:

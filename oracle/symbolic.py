@@ -62,6 +62,18 @@ class SymbolicDomain:
     def exec_piece(self, q, st, j, t, incoming):
         if st.op == "nop":
             return None
+        if st.multimem:  # reading R23: the same chunk on every rank, folded in ascending rank order
+            if st.reads_all:
+                vals = [self.get(p, st.srcbuf, st.srcoff + j) for p in range(len(self.bufs))]
+                v = vals[0]
+                for x in vals[1:]:
+                    v = combine(v, x)
+            else:
+                v = self.get(q, st.srcbuf, st.srcoff + j)
+            for p in range(len(self.bufs)):
+                if st.writes_all or p == q:
+                    self.bufs[p][self._key(st.dstbuf, st.dstoff + j)] = v
+            return None
         if st.recvs and incoming is UNINIT:
             raise SymbolicError("rank %d receives an uninitialized chunk" % q)
         src = self.get(q, st.srcbuf, st.srcoff + j) if st.reads_src else None

@@ -15,6 +15,9 @@ V8 deps name an existing (tb, step) of another thread block on the same GPU, and
    referenced step sets hasdep (Fig. 5 lines 25-27)
 V9 no deadlock in the abstract machine with the protocol's FIFO slot count, run for >= 2
    pipeline iterations (§5.2; §6.1)
+V11 multimem ops (mrd/mst/mrs, reading R23) address only the i/o buffers, and the thread
+   blocks that hold them have the same ids on every rank (their start/end group barrier
+   pairs thread block b of every rank)
 V10 (races=True) no happens-before race between instructions (oracle/races.py; §3.3
    P:L859-867, §5.2); with `marking` (the loader's direct placement) also none
    after the direct writes are moved to the sends
@@ -103,6 +106,8 @@ def validate(algo, nranks=None, slots=8, max_tbs=148, max_channels=64, iters=2, 
                     _fail("V6", "%s: reduce needs src and dst" % w)
                 if st.writes_dst and st.dstbuf == "i" and not algo.inplace:
                     _fail("V3", "%s: out-of-place program writes the input buffer" % w)
+                if st.multimem and ("s" in (st.srcbuf, st.dstbuf)):
+                    _fail("V11", "%s: multimem op on the scratch buffer (per-rank sizes)" % w)
                 for (b, s) in st.deps:
                     if b == tb.id:
                         _fail("V8", "%s: depends on its own thread block" % w)
@@ -120,6 +125,10 @@ def validate(algo, nranks=None, slots=8, max_tbs=148, max_channels=64, iters=2, 
         for k, (a, b) in enumerate(zip(sc, rc)):
             if a != b:
                 _fail("V7", "connection %s message %d: send cnt %d != recv cnt %d" % (key, k, a, b))
+    mm = [sorted(tb.id for tb in g.tbs if any(st.multimem for st in tb.steps)) for g in algo.gpus]
+    for g, ids in zip(algo.gpus, mm):
+        if ids != mm[0]:
+            _fail("V11", "rank %d holds multimem ops in thread blocks %s, rank 0 in %s" % (g.id, ids, mm[0]))
     try:
         Machine(algo, NullDomain(), slots=slots, iters=iters).run()
     except Deadlock as e:

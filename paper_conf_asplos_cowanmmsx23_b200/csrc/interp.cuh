@@ -235,6 +235,16 @@ __device__ __forceinline__ void stRelaxedGpu(uint64_t* p, uint64_t v) {
 }
 __device__ __forceinline__ void fenceSys() { asm volatile("fence.acq_rel.sys;" ::: "memory"); }
 __device__ __forceinline__ void fenceGpu() { asm volatile("fence.acq_rel.gpu;" ::: "memory"); }
+#ifndef MSCCL_WARP_FENCE
+#define MSCCL_WARP_FENCE 0
+#endif
+#ifndef MSCCL_REL_STORE
+#define MSCCL_REL_STORE 0
+#endif
+__device__ __forceinline__ void postRelease(uint64_t* p, uint64_t v, bool sys) {
+  if (sys) asm volatile("st.release.sys.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+  else asm volatile("st.release.gpu.global.u64 [%0], %1;" ::"l"(p), "l"(v) : "memory");
+}
 // post a connection counter (one u64 word in its own 128-byte line)
 __device__ __forceinline__ void postFlag(uint64_t* p, uint64_t v, bool sys) {
   if (sys) stRelaxedSys(p, v);
@@ -841,6 +851,14 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
   // each protocol's data path is its own non-inlined function (separate register allocation)
   if constexpr (!ll || (!RECV && !SEND)) {
     movePiecesSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, tb, in, t, rslot, sslot);
+#if MSCCL_WARP_FENCE
+    // every warp drains its own stores before the block barrier, in parallel, so the poster's
+    // fence after the barrier has (almost) nothing left to wait for
+    if constexpr (SEND) {
+      if (sys) fenceSys();
+      else fenceGpu();
+    }
+#endif
   } else if constexpr (PROTO == 2) {
     if (!movePiecesLL128<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, in, t, rslot, sslot, recvd + 1, sent + 1)) *sAbort = 1;
   } else {
@@ -859,10 +877,15 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
   } else if (c.tid == (MSCCL_POST_LAST_WARP ? c.nt - 32 : 0) && (RECV || SEND) && !ll) {
     // Simple: lane 0 of the last warp posts, so thread 0 (the head poller) goes straight to the
     // next step's wait and the fence latency overlaps it (option MSCCL_POST_LAST_WARP)
+#if MSCCL_REL_STORE
+    if (SEND) postRelease(tb.sendHead, sent + 1, sys);
+    if (RECV) postRelease(tb.recvAck, recvd + 1, sys);
+#else
     if (sys) fenceSys();
     else fenceGpu();
     if (SEND) postFlag(tb.sendHead, sent + 1, sys);
     if (RECV) postFlag(tb.recvAck, recvd + 1, sys);
+#endif
   }
 #if MSCCL_TRACE
   if (c.tid == 0 && a.trace) {

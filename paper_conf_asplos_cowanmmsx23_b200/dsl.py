@@ -30,7 +30,10 @@ Lowering follows §4-§5:
 Extensions: ``c1.reduce(c2, buffer=, index=)`` names the destination of the
 result (the rrc instruction already has separate src/dst), which lets
 out-of-place programs keep the input buffer read-only; ``parallelize(k)`` splits each
-op of a fragment into k ops of count/k on channels ch+i.
+op of a fragment into k ops of count/k on channels ch+i (P:L1149-1164);
+``c.multimem_reduce(...)`` / ``c.multimem_store(...)`` are the NVSwitch multicast ops of
+reading R23 (not in the paper): one instruction on the issuing rank that
+reads or writes the same chunks on EVERY rank.
 """
 import heapq
 from contextlib import contextmanager
@@ -151,6 +154,36 @@ class Ref:
         return p._write(self.rank, b, idx, self.count)
 
 
+    # ---- multimem (NVLS) ops, reading R23 ----
+    def multimem_reduce(self, buffer, index=None, store_all=True, ch=None):
+        """Reduce these chunks over every rank (the same buffer and index on each) and write
+        the result to (buffer, index) on this rank (``mrd``) or on every rank (``mrs``).
+        The sources must still hold the precondition's input on every rank, and results
+        stored on other ranks are final (nothing may read them later): the group barrier of
+        the multimem thread block orders only the multimem ops themselves."""
+        p = self.prog
+        p._mm_sources(self)
+        b = BUFNAME[buffer]
+        idx = self.index if index is None else p._index(index)
+        p._record("mrs" if store_all else "mrd", (self.rank, self.buf, self.index), None, (self.rank, b, idx),
+                  self.count, ch)
+        if store_all:
+            return p._mm_final(b, idx, self.count, self.rank)
+        return p._write(self.rank, b, idx, self.count)
+
+    def multimem_store(self, buffer, index, ch=None):
+        """Store these chunks to (buffer, index) on every rank (``mst``); results are final."""
+        p = self.prog
+        self._check()
+        b = BUFNAME[buffer]
+        idx = p._index(index)
+        p._record("mst", (self.rank, self.buf, self.index), None, (self.rank, b, idx), self.count, ch)
+        return p._mm_final(b, idx, self.count, self.rank)
+
+
+FINAL = -1  # version of a chunk written on a remote rank by a multimem op (reading R23)
+
+
 def chunk(rank, buffer, index, count=1, sz=None):
     """Reference to the chunks currently at (rank, buffer, index) (Table 1)."""
     p = _prog()
@@ -162,6 +195,9 @@ def chunk(rank, buffer, index, count=1, sz=None):
     if any(v is None for v in vers):
         raise DSLError("chunk(%d, %s, %d, %d) accesses an uninitialized chunk (P:L847-848)"
                        % (rank, buffer, index, count))
+    if any(v == FINAL for v in vers):
+        raise DSLError("chunk(%d, %s, %d, %d) was written by a multimem op: multimem results are final "
+                       "(reading R23)" % (rank, buffer, index, count))
     return Ref(p, rank, b, index, count, vers)
 
 
@@ -262,6 +298,22 @@ class Program:
             vers.append(v)
         return Ref(self, rank, b, index, count, tuple(vers))
 
+    def _mm_sources(self, ref):
+        """Multimem sources: the same chunks on every rank, still holding the input."""
+        ref._check()
+        for r in range(self.R):
+            v = self._versions(r, ref.buf, ref.index, ref.count)
+            if any(x != 0 for x in v):
+                raise DSLError("multimem reduce of %s[%d:%d] needs the unmodified input on every rank "
+                               "(rank %d's was written)" % (ref.buf, ref.index, ref.index + ref.count, r))
+
+    def _mm_final(self, b, index, count, rank):
+        self._check_bounds(b, index, count)
+        for r in range(self.R):
+            for k in range(index, index + count):
+                self._ver[self._key(r, b, k)] = FINAL
+        return None
+
     def _check_bounds(self, b, index, count):
         lim = {"i": self.collective.i_chunks, "o": self.collective.o_chunks}.get(b)
         if b == "o" and self.collective.inplace:
@@ -312,6 +364,9 @@ class Program:
         for op in self._ops:
             s_r, s_b, s_i = op.src
             d_r, d_b, d_i = op.dst
+            if op.kind in ir.MULTIMEM_OPS:  # one instruction on the issuing rank (reading R23)
+                new(s_r, op.kind, (s_b, s_i), (d_b, d_i), op.count, ch=op.ch)
+                continue
             if op.kind == "copy":
                 if s_r == d_r:
                     new(s_r, "cpy", (s_b, s_i), (d_b, d_i), op.count, ch=op.ch)
@@ -456,7 +511,7 @@ class Program:
         for x in ins:
             if x.ch is None:
                 x.ch = 0
-        return 1 + max([x.ch for x in ins if x.sp >= 0 or x.rp >= 0] + [0])
+        return 1 + max([x.ch for x in ins if x.sp >= 0 or x.rp >= 0 or x.op in ir.MULTIMEM_OPS] + [0])
 
     # step 5: whole-program instances (reading R5: interleaved sub-chunks)
     def _replicate(self, ins, nch):
@@ -512,6 +567,10 @@ class Program:
                         merged.append(t)
                 tuples = merged + list(recv_only.values())
             lst = [_TB(t[0], t[1], t[2]) for t in tuples]
+            # multimem ops run on their own thread block per channel (its group barrier pairs
+            # it with the same block on every rank, reading R23)
+            for ch in sorted({x.ch for x in ins if x.rank == r and x.op in ir.MULTIMEM_OPS}):
+                lst.append(_TB(-1, -1, ch))
             if not lst and any(x.rank == r for x in ins):
                 lst.append(_TB(-1, -1, 0))
             for i, tb in enumerate(lst):
@@ -620,6 +679,8 @@ class _TB:
 
 
 def _fits(tb, x):
+    if x.op in ir.MULTIMEM_OPS:
+        return tb.send == -1 and tb.recv == -1 and tb.ch == x.ch
     if x.sp >= 0 and (tb.send != x.sp or tb.ch != x.ch):
         return False
     if x.rp >= 0 and (tb.recv != x.rp or tb.ch != x.ch):

@@ -12,17 +12,21 @@ Text syntax (DESIGN.md reading R0)::
         <tb id send recv chan>
           <step s type srcbuf srcoff dstbuf dstoff cnt depid deps hasdep/>
 
-``type`` is one of nop s r cpy re rrc rrs rrcs rcs; buffers are i/o/s ('-' = unused);
+``type`` is one of nop s r cpy re rrc rrs rrcs rcs, or a multimem op mrd mst mrs (reading
+R23); buffers are i/o/s ('-' = unused);
 ``depid``/``deps`` are equal-length comma lists ('-1' = none).
 """
 from dataclasses import dataclass, field
 import xml.etree.ElementTree as ET
 
-OPCODES = {"nop": 0, "s": 1, "r": 2, "cpy": 3, "re": 4, "rrc": 5, "rrs": 6, "rrcs": 7, "rcs": 8}
+OPCODES = {"nop": 0, "s": 1, "r": 2, "cpy": 3, "re": 4, "rrc": 5, "rrs": 6, "rrcs": 7, "rcs": 8,
+           "mrd": 9, "mst": 10, "mrs": 11}
 RECV_OPS = {"r", "rrc", "rrs", "rrcs", "rcs"}
 SEND_OPS = {"s", "rrs", "rrcs", "rcs"}
-SRC_OPS = {"s", "cpy", "re", "rrc", "rrs", "rrcs"}
-DST_OPS = {"r", "cpy", "re", "rrc", "rrcs", "rcs"}
+SRC_OPS = {"s", "cpy", "re", "rrc", "rrs", "rrcs", "mrd", "mst", "mrs"}
+DST_OPS = {"r", "cpy", "re", "rrc", "rrcs", "rcs", "mrd", "mst", "mrs"}
+# multimem (NVLS) ops, DESIGN.md reading R23: the same chunk on every rank of the group
+MULTIMEM_OPS = {"mrd", "mst", "mrs"}
 
 
 @dataclass
