@@ -15,8 +15,8 @@ V8 deps name an existing (tb, step) of another thread block on the same GPU, and
    referenced step sets hasdep (Fig. 5 lines 25-27)
 V9 no deadlock in the abstract machine with the protocol's FIFO slot count, run for >= 2
    pipeline iterations (§5.2; §6.1)
-V11 multimem ops (mrd/mst/mrs, reading R23) address only the i/o buffers, and the thread
-   blocks that hold them have the same ids on every rank (their start/end group barrier
+V11 multimem ops (mrd/mst/mrs, reading R23) address only the i/o buffers, the program uses
+   the Simple protocol, and the thread blocks that hold them have the same ids on every rank (their start/end group barrier
    pairs thread block b of every rank)
 V10 (races=True) no happens-before race between instructions (oracle/races.py; §3.3
    P:L859-867, §5.2); with `marking` (the loader's direct placement) also none
@@ -126,6 +126,8 @@ def validate(algo, nranks=None, slots=8, max_tbs=148, max_channels=64, iters=2, 
             if a != b:
                 _fail("V7", "connection %s message %d: send cnt %d != recv cnt %d" % (key, k, a, b))
     mm = [sorted(tb.id for tb in g.tbs if any(st.multimem for st in tb.steps)) for g in algo.gpus]
+    if any(mm) and algo.proto != "Simple":
+        _fail("V11", "multimem programs use the Simple protocol")
     for g, ids in zip(algo.gpus, mm):
         if ids != mm[0]:
             _fail("V11", "rank %d holds multimem ops in thread blocks %s, rank 0 in %s" % (g.id, ids, mm[0]))

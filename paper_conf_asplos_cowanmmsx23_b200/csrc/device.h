@@ -11,6 +11,8 @@ namespace msccl {
 #define MSCCL_MAX_LOCAL 16   // ranks that one kernel launch may cover (virtual ranks)
 #define MSCCL_FLAG_STRIDE 16 // u64 words between connection counters (one 128-byte line each)
 #define MSCCL_REF_REG (1ull << 63)  // destination reference: registered-buffer (index, offset) form
+#define MSCCL_MM_MAX_TB 64   // thread-block ids that may hold multimem ops (group-barrier lines)
+#define MSCCL_MM_MAX_RANKS 16
 #ifndef MSCCL_MAX_THREADS
 #define MSCCL_MAX_THREADS 256  // threads per CTA (MSCCL_THREADS <= this); 2 CTAs per SM at 256
 #endif
@@ -51,6 +53,9 @@ struct DevTB {
   uint64_t* recvAck;          // peer: messages I consumed
   uint64_t* recvCnt;          // mine: [0] messages I consumed, [1] launches on this connection
   uint64_t* recvReady;        // peer: the sender's ready line for this connection (I write it)
+  int32_t mmId;               // multimem thread block: its group-barrier line index (tb id), else -1
+  uint32_t mmTag;             // the program's load ordinal on this communicator (group-barrier epoch)
+  int32_t pad[2];
 };
 static_assert(sizeof(DevTB) % 16 == 0, "DevTB is staged with 16-byte loads");
 
@@ -75,6 +80,8 @@ struct RankArgs {
   int32_t directMask;
   unsigned long long* stats;  // this rank's counters (region): [0] cross-launch handshakes that
                               // resolved a direct destination (mscclCommGetStats)
+  char* const* peerRegion;    // every rank's shared region in this address space (group barriers)
+  int32_t myRank, nRanks;
 };
 
 struct KernelArgs {
@@ -94,7 +101,11 @@ struct KernelArgs {
   // 2 cross-launch (ranks in other launches / processes, ready handshake per connection)
   int32_t direct;
   int32_t directHints;        // bit 0: terminal direct sends store L2 evict_first (cache hint)
-  int32_t pad0;
+  // multimem ops (reading R23): 0 none; 1 every rank in this launch (slot r = rank r, buffers
+  // from the launch arguments, no barrier); 2 cross-launch (group barrier lines publish the
+  // ranks' buffer references at the start and completion at the end)
+  int32_t mm;
+  int64_t mmLineOff;          // offset of the group-barrier lines in every region
   uint64_t timeoutNs;         // device watchdog; 0 = disabled
   uint64_t* trace;            // MSCCL_TRACE builds: per-CTA phase times (ns), else null
 };

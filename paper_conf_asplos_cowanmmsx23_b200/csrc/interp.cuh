@@ -32,7 +32,8 @@ namespace msccl {
 enum { R_SUM = 0, R_PROD = 1, R_MAX = 2, R_MIN = 3, R_COPY = 4 };
 enum { DT_I8 = 0, DT_U8 = 1, DT_I32 = 2, DT_U32 = 3, DT_I64 = 4, DT_U64 = 5, DT_F16 = 6, DT_F32 = 7, DT_F64 = 8,
        DT_BF16 = 9 };
-enum { K_NOP = 0, K_SEND = 1, K_RECV = 2, K_COPY = 3, K_REDUCE = 4, K_RRC = 5, K_RRS = 6, K_RRCS = 7, K_RCS = 8 };
+enum { K_NOP = 0, K_SEND = 1, K_RECV = 2, K_COPY = 3, K_REDUCE = 4, K_RRC = 5, K_RRS = 6, K_RRCS = 7, K_RCS = 8,
+       K_MRD = 9, K_MST = 10, K_MRS = 11 };
 enum { KB_IN = 0, KB_OUT = 1, KB_SC = 2 };
 
 struct V32 {  // 32-byte vector (one 256-bit LDG/STG on sm_100)
@@ -272,6 +273,7 @@ struct Ctx {
   char** peerDst;
   mutable bool readyDone;
   uint64_t sendL;  // thread 32: this launch's ordinal on the send connection
+  char* (*mmBuf)[2];  // multimem ops: every rank's in/out base in this address space (shared memory)
 };
 
 static __device__ __noinline__ void raiseAbort(const KernelArgs& a) {
@@ -904,18 +906,222 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
   return true;
 }
 
-template <int DT, int OP, int PROTO>
+// ------------------------------------------------------------------ multimem ops (reading R23)
+// mrd / mst / mrs address the same chunk of every rank's buffer. With NVSwitch multicast
+// they are one multimem.ld_reduce / multimem.st per vector on the multicast address; this
+// interpreter path is the unicast form of the same semantics: loads from every rank's copy
+// (peer memory over NVLink, or the same HBM for virtual ranks), folded in ascending rank order
+// with fp32 accumulation and one rounding for fp16 / bf16 sums (what the switch's .acc::f32
+// reduction computes), and one store per rank.
+template <int DT, int OP>
+struct MMAcc {  // fold of R 16-byte vectors in ascending rank order
+  static constexpr bool kHalfSum = (DT == DT_BF16 || DT == DT_F16) && OP == R_SUM;
+  float f[8];
+  uint4 v;
+  static __device__ __forceinline__ float widen(uint16_t x) {
+    if constexpr (DT == DT_BF16) return __uint_as_float(((uint32_t)x) << 16);
+    else return __half2float(__ushort_as_half(x));
+  }
+  static __device__ __forceinline__ uint16_t narrow(float x) {
+    if constexpr (DT == DT_BF16) return __bfloat16_as_ushort(__float2bfloat16_rn(x));
+    else return __half_as_ushort(__float2half_rn(x));
+  }
+  __device__ __forceinline__ void first(const uint4& x) {
+    if constexpr (kHalfSum) {
+      const uint16_t* h = reinterpret_cast<const uint16_t*>(&x);
+#pragma unroll
+      for (int k = 0; k < 8; k++) f[k] = widen(h[k]);
+    } else {
+      v = x;
+    }
+  }
+  __device__ __forceinline__ void add(const uint4& x) {
+    if constexpr (kHalfSum) {
+      const uint16_t* h = reinterpret_cast<const uint16_t*>(&x);
+#pragma unroll
+      for (int k = 0; k < 8; k++) f[k] = f[k] + widen(h[k]);
+    } else {
+      v = vop<DT, OP>(v, x);
+    }
+  }
+  __device__ __forceinline__ uint4 result() const {
+    if constexpr (kHalfSum) {
+      uint4 r;
+      uint16_t* h = reinterpret_cast<uint16_t*>(&r);
+#pragma unroll
+      for (int k = 0; k < 8; k++) h[k] = narrow(f[k]);
+      return r;
+    } else {
+      return v;
+    }
+  }
+};
+
+template <int DT, int OP, int KIND>
+__device__ __noinline__ void runMultimem(const Ctx& c, const DevInstr& in, int t) {
+  typedef typename DType<DT>::T T;
+  const KernelArgs& a = *c.a;
+  const RankArgs& ra = *c.ra;
+  constexpr bool RALL = KIND != K_MST, WALL = KIND != K_MRD;
+  const int R = ra.nRanks, me = ra.myRank;
+  const int64_t w = sizeof(T), a0 = (int64_t)t * a.T;
+  const uint64_t pol = policyEvictFirst();
+  for (int j = 0; j < in.cnt; j++) {
+    int64_t ss, sl, ds, dl;
+    chunkSpan(a, in.srcBuf, (int64_t)in.srcOff + j, ss, sl);
+    chunkSpan(a, in.dstBuf, (int64_t)in.dstOff + j, ds, dl);
+    const int64_t L = sl < dl ? sl : dl;
+    const int64_t m = (a0 + a.T < L ? a0 + a.T : L) - a0;
+    if (m <= 0) continue;
+    const int64_t so = (ss + a0) * w, dof = (ds + a0) * w;
+    uintptr_t al = (uintptr_t)so | (uintptr_t)dof;
+    for (int p = 0; p < R; p++) al |= (uintptr_t)c.mmBuf[p][in.srcBuf] | (uintptr_t)c.mmBuf[p][in.dstBuf];
+    const int64_t nvec = (al & 15) ? 0 : m * w / 16;
+    for (int64_t i = c.tid; i < nvec; i += c.nt) {
+      MMAcc<DT, OP> acc;
+      if constexpr (RALL) {  // 4 ranks' loads in flight, folded in ascending rank order
+        for (int p0 = 0; p0 < R; p0 += 4) {
+          uint4 x[4];
+#pragma unroll
+          for (int u = 0; u < 4; u++)
+            if (p0 + u < R) ldStream(x[u], c.mmBuf[p0 + u][in.srcBuf] + so + i * 16, pol);
+#pragma unroll
+          for (int u = 0; u < 4; u++) {
+            if (p0 + u >= R) break;
+            if (p0 + u == 0) acc.first(x[u]);
+            else acc.add(x[u]);
+          }
+        }
+      } else {
+        uint4 x;
+        ldStream(x, c.mmBuf[me][in.srcBuf] + so + i * 16, pol);
+        acc.first(x);
+      }
+      const uint4 v = acc.result();
+      for (int p = 0; p < R; p++)
+        if (WALL || p == me) stHint(c.mmBuf[p][in.dstBuf] + dof + i * 16, v, pol);
+    }
+    for (int64_t e = nvec * 16 / w + c.tid; e < m; e += c.nt) {  // scalar tail (ragged or unaligned)
+      T v;
+      if constexpr (RALL) {
+        if constexpr (MMAcc<DT, OP>::kHalfSum) {
+          float f = MMAcc<DT, OP>::widen(*(const T*)(c.mmBuf[0][in.srcBuf] + so + e * w));
+          for (int p = 1; p < R; p++) f = f + MMAcc<DT, OP>::widen(*(const T*)(c.mmBuf[p][in.srcBuf] + so + e * w));
+          v = MMAcc<DT, OP>::narrow(f);
+        } else {
+          v = *(const T*)(c.mmBuf[0][in.srcBuf] + so + e * w);
+          for (int p = 1; p < R; p++) v = DType<DT>::op(OP, v, *(const T*)(c.mmBuf[p][in.srcBuf] + so + e * w));
+        }
+      } else {
+        v = *(const T*)(c.mmBuf[me][in.srcBuf] + so + e * w);
+      }
+      for (int p = 0; p < R; p++)
+        if (WALL || p == me) *(T*)(c.mmBuf[p][in.dstBuf] + dof + e * w) = v;
+    }
+  }
+}
+
+// Group barrier of a multimem thread block in cross-launch mode (reading R23): at its start,
+// thread block b of this rank publishes {epoch, in ref, out ref} to line (start, b, me) of
+// every rank and waits until every rank's line (start, b, p) here carries the same epoch,
+// then resolves their buffer references; at its end it publishes (done, b, me) after a
+// system-scope fence and waits for every rank's. Epoch = (program load tag, launch gen):
+// equal on every rank for the same launch, never reused, compared for equality.
+__device__ __forceinline__ uint64_t* mmLine(const KernelArgs& a, char* region, int kind, int b, int src, int R) {
+  return (uint64_t*)(region + a.mmLineOff + ((size_t)(kind * MSCCL_MM_MAX_TB + b) * R + src) * 128);
+}
+
+__device__ __forceinline__ bool waitEq(const uint64_t* p, uint64_t v, const Ctx& c) {
+  uint64_t t0 = 0;
+  for (uint32_t it = 0;; it++) {
+    if (ldAcquireSys(p) == v) return true;
+    if ((it & 1023u) == 1023u) {
+      const uint64_t now = globaltimer();
+      if (t0 == 0) t0 = now;
+      if (*(volatile uint32_t*)c.ra->abortFlag) return false;
+      if (c.a->timeoutNs && now - t0 > c.a->timeoutNs) {
+        raiseAbort(*c.a);
+        return false;
+      }
+    }
+  }
+}
+
+// returns false on watchdog / abort; every thread calls it (block-uniform)
+static __device__ __noinline__ bool mmBarrier(const Ctx& c, const DevTB& tb, uint64_t gen, bool start) {
+  const uint64_t epoch = ((uint64_t)tb.mmTag << 40) | ((gen + 1) & ((1ull << 40) - 1));
+  const KernelArgs& a = *c.a;
+  const RankArgs& ra = *c.ra;
+  const int R = ra.nRanks, me = ra.myRank;
+  bool ok = true;
+  if (!start) {
+    __syncthreads();                       // every thread's multimem stores are issued
+    if (c.tid == 0) fenceSys();            // ... and visible system-wide before "done"
+    __syncthreads();
+  }
+  if (c.tid < R && c.tid != me) {
+    uint64_t* l = mmLine(a, ra.peerRegion[c.tid], start ? 0 : 1, tb.mmId, me, R);
+    if (start) {
+      stRelaxedSys(l + 1, ra.bufRef[0]);
+      stRelaxedSys(l + 2, ra.bufRef[1]);
+      fenceSys();
+    }
+    stRelaxedSys(l, epoch);
+    const uint64_t* mine = mmLine(a, ra.peerRegion[me], start ? 0 : 1, tb.mmId, c.tid, R);
+    ok = waitEq(mine, epoch, c);
+    if (ok && start) {
+      for (int b = 0; b < 2; b++) {
+        const uint64_t ref = *(volatile const uint64_t*)(mine + 1 + b);
+        char* ptr = resolveRef(ra, c.tid, ref);
+        if (!ptr) {  // a peer's buffer this process cannot reach: no multimem without it
+          raiseAbort(a);
+          ok = false;
+        }
+        c.mmBuf[c.tid][b] = ptr;
+      }
+    }
+  }
+  if (start && c.tid == me) {
+    c.mmBuf[me][0] = ra.buf[0];
+    c.mmBuf[me][1] = ra.buf[1];
+  }
+  return __syncthreads_and(ok) != 0;
+}
+
+template <int DT, int OP>
+__device__ __noinline__ void multimemOp(const Ctx& c, const DevInstr& in, int t) {
+  if (in.op == K_MST) runMultimem<DT, OP, K_MST>(c, in, t);
+  if constexpr (OP != R_COPY) {
+    if (in.op == K_MRD) runMultimem<DT, OP, K_MRD>(c, in, t);
+    if (in.op == K_MRS) runMultimem<DT, OP, K_MRS>(c, in, t);
+  }
+}
+
+// MM: the kernel variant for programs with multimem ops (reading R23). Their code lives only
+// in that variant: a call into it from the kernel body raised the register pressure of every
+// other data path of the kernel (ptxas -v: spills in every movePieces / runOp), so programs
+// without multimem ops run kernels that do not contain it.
+template <int DT, int OP, int PROTO, bool MM>
 __device__ __forceinline__ bool dispatch(const Ctx& c, const DevTB& tb, const DevInstr& in, int t, uint64_t& sent,
                                          uint64_t& recvd, volatile int* sAbort) {
+  if constexpr (MM) {
+    if (in.op >= K_MRD) {
+      multimemOp<DT, OP>(c, in, t);
+      __syncthreads();
+      return true;
+    }
+  }
   switch (in.op) {  // Fig. 5 line 18; every case ends (the figure's fall-through is reading R10)
     case K_SEND: return runOp<DT, OP, PROTO, false, true, true, false, false>(c, tb, in, t, sent, recvd, sAbort);
     case K_RECV: return runOp<DT, OP, PROTO, true, false, false, true, false>(c, tb, in, t, sent, recvd, sAbort);
     case K_COPY: return runOp<DT, OP, PROTO, false, false, true, true, false>(c, tb, in, t, sent, recvd, sAbort);
     case K_RCS: return runOp<DT, OP, PROTO, true, true, false, true, false>(c, tb, in, t, sent, recvd, sAbort);
+
     default: break;
   }
   if (OP != R_COPY) {
     switch (in.op) {
+
       case K_REDUCE: return runOp<DT, OP, PROTO, false, false, true, true, true>(c, tb, in, t, sent, recvd, sAbort);
       case K_RRC: return runOp<DT, OP, PROTO, true, false, true, true, false>(c, tb, in, t, sent, recvd, sAbort);
       case K_RRS: return runOp<DT, OP, PROTO, true, true, true, false, false>(c, tb, in, t, sent, recvd, sAbort);
@@ -1090,7 +1296,7 @@ __device__ __noinline__ void chainExecSimple(const Ctx& c, const DevInstr* mem, 
 #define MSCCL_SMEM_INSTR 64  // instructions per thread block staged in shared memory (LL / LL128)
 #endif
 
-template <int DT, int OP, int PROTO>
+template <int DT, int OP, int PROTO, bool MM = false>
 __global__ void __launch_bounds__(MSCCL_MAX_THREADS, MSCCL_MIN_BLOCKS) mscclInterpreter(const __grid_constant__ KernelArgs aParam) {
   __shared__ int sAbort;
   // The launch arguments (all ranks' base pointers and tables, geometry) are copied from the
@@ -1129,8 +1335,13 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, MSCCL_MIN_BLOCKS) mscclInte
   }
   __shared__ uint64_t sAck;
   __shared__ char* sPeerDst[3];
+  __shared__ char* sMM[MSCCL_MM_MAX_RANKS][2];
   __shared__ ChainSmem sChain;
-  Ctx c{&a, &ra, (int)threadIdx.x, (int)blockDim.x, 0, &sAck, sPeerDst, false, 0};
+  Ctx c{&a, &ra, (int)threadIdx.x, (int)blockDim.x, 0, &sAck, sPeerDst, false, 0, sMM};
+  if (MM && a.mm == 1 && (int)threadIdx.x < a.nLocal) {  // every rank in this launch: slot r = rank r
+    sMM[threadIdx.x][0] = a.rank[threadIdx.x].buf[0];
+    sMM[threadIdx.x][1] = a.rank[threadIdx.x].buf[1];
+  }
   if (threadIdx.x == 0) {
     sAbort = 0;
     // one-launch direct placement: the send peer is local rank tb.sendPeer of this launch
@@ -1161,6 +1372,9 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, MSCCL_MIN_BLOCKS) mscclInte
   // head / dependencies meanwhile; every post follows a block barrier (option MSCCL_POST_LAST_WARP)
   const int kPoster = MSCCL_POST_LAST_WARP ? (int)blockDim.x - 32 : 0;
   __syncthreads();
+  if constexpr (MM) {
+    if (a.mm == 2 && tb.mmId >= 0 && !mmBarrier(c, tb, gen, true)) return;
+  }
   for (int t = 0; t < a.I; t++) {
     for (int s = 0; s < tb.nSteps; s++) {
       const DevInstr in = ins[s];
@@ -1214,7 +1428,7 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, MSCCL_MIN_BLOCKS) mscclInte
         __syncthreads();
         if (sAbort) return;
       }
-      if (!dispatch<DT, OP, PROTO>(c, tb, in, t, sent, recvd, &sAbort)) return;
+      if (!dispatch<DT, OP, PROTO, MM>(c, tb, in, t, sent, recvd, &sAbort)) return;
       if (in.hasDep) {  // Fig. 5 lines 25-27: the step is complete before the semaphore moves
         if (c.tid == kPoster) {
           fenceGpu();
@@ -1222,6 +1436,9 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, MSCCL_MIN_BLOCKS) mscclInte
         }
       }
     }
+  }
+  if constexpr (MM) {
+    if (a.mm == 2 && tb.mmId >= 0 && !mmBarrier(c, tb, gen, false)) return;
   }
   if (threadIdx.x == 0) {  // epilogue: persist the connection counters and the generation
     if (tb.sendFifo) *(volatile uint64_t*)tb.sendCnt = sent;

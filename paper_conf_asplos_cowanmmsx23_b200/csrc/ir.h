@@ -16,7 +16,13 @@ enum Proto { PROTO_SIMPLE = 0, PROTO_LL = 1, PROTO_LL128 = 2 };
 
 // opcodes (also the device encoding)
 enum OpCode { OP_NOP = 0, OP_SEND = 1, OP_RECV = 2, OP_COPY = 3, OP_REDUCE = 4, OP_RRC = 5, OP_RRS = 6,
-              OP_RRCS = 7, OP_RCS = 8, OP_COUNT = 9 };
+              OP_RRCS = 7, OP_RCS = 8,
+              // multimem (NVLS) ops, reading R23: the same chunk on every rank of the group
+              OP_MRD = 9,    // dst_q <- (+)_p src_p                 (multimem.ld_reduce)
+              OP_MST = 10,   // dst_p <- src_q for every rank p      (multimem.st)
+              OP_MRS = 11,   // v = (+)_p src_p; dst_p <- v           (ld_reduce + st)
+              OP_COUNT = 12 };
+inline bool isMultimem(int op) { return op == OP_MRD || op == OP_MST || op == OP_MRS; }
 enum BufId { BUF_IN = 0, BUF_OUT = 1, BUF_SC = 2, BUF_NONE = 3 };
 
 // per-op roles (§4.2): receives, sends, reads src, writes dst
@@ -32,6 +38,9 @@ inline OpRole opRole(int op) {
       {true, true, true, false},     // rrs
       {true, true, true, true},      // rrcs
       {true, true, false, true},     // rcs
+      {false, false, true, true},    // mrd
+      {false, false, true, true},    // mst
+      {false, false, true, true},    // mrs
   };
   return t[op];
 }
@@ -63,6 +72,7 @@ struct Algo {
   std::vector<GpuProgram> gpus;
   int maxCnt() const;
   bool hasReduce() const;
+  bool hasMultimem() const;
 };
 
 Algo parseIR(const char* text, size_t len);  // throws IRError (rule V1)

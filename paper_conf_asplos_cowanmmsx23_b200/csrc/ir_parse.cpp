@@ -148,7 +148,7 @@ int bufOf(const std::string& s) {
 }
 
 int opOf(const std::string& s) {
-  static const char* names[OP_COUNT] = {"nop", "s", "r", "cpy", "re", "rrc", "rrs", "rrcs", "rcs"};
+  static const char* names[OP_COUNT] = {"nop", "s", "r", "cpy", "re", "rrc", "rrs", "rrcs", "rcs", "mrd", "mst", "mrs"};
   for (int i = 0; i < OP_COUNT; i++)
     if (s == names[i]) return i;
   throw IRError("V1: unknown instruction type '" + s + "'");
@@ -250,7 +250,17 @@ bool Algo::hasReduce() const {
   for (auto& g : gpus)
     for (auto& tb : g.tbs)
       for (auto& s : tb.steps)
-        if (s.op == OP_REDUCE || s.op == OP_RRC || s.op == OP_RRS || s.op == OP_RRCS) return true;
+        if (s.op == OP_REDUCE || s.op == OP_RRC || s.op == OP_RRS || s.op == OP_RRCS || s.op == OP_MRD ||
+            s.op == OP_MRS)
+          return true;
+  return false;
+}
+
+bool Algo::hasMultimem() const {
+  for (auto& g : gpus)
+    for (auto& tb : g.tbs)
+      for (auto& s : tb.steps)
+        if (isMultimem(s.op)) return true;
   return false;
 }
 

@@ -4,4 +4,7 @@
 namespace msccl {
 const void* interpreterKernel(int dtype, int op, int proto);  // op 0..3 sum/prod/max/min; proto 0 Simple 1 LL 2 LL128
 const void* copyKernel(int elemBytes, int proto);             // programs with no reduction
+// programs with multimem ops (reading R23; Simple protocol): separate kernel variants
+const void* interpreterKernelMM(int dtype, int op);
+const void* copyKernelMM(int elemBytes);
 }  // namespace msccl

@@ -119,6 +119,8 @@ struct mscclComm {
   std::string lastError;
   int maxCoResident = 0;
   uint64_t launchesDirect1 = 0, launchesDirect2 = 0;  // launches this rank took part in, by direct mode
+  uint32_t loadCounter = 0;            // programs loaded so far (multimem group-barrier epochs)
+  char** dPeerRegion = nullptr;        // device [nranks]: every rank's region in this address space
   std::vector<mscclReg*> regs;         // by index (nullptr = free)
   char** dRegMap = nullptr;            // device [nranks][regMax]: peers' registered buffers, mapped here
   std::vector<char*> hRegMap;
@@ -145,6 +147,9 @@ struct mscclComm {
   }
   size_t abortOff() const { return flagOff(5, 0, 0); }
   size_t statsOff() const { return abortOff() + 128; }
+  // multimem group-barrier lines (reading R23): [start|done][thread block][source rank]
+  size_t mmLineOff() const { return statsOff() + 128; }
+  size_t mmBytes() const { return (size_t)2 * MSCCL_MM_MAX_TB * nranks * 128; }
 };
 
 struct mscclProgram {
@@ -164,6 +169,7 @@ struct mscclProgram {
   bool hasReduce = false;
   bool allDirect = true;  // every message of this rank's program is a direct placement (R15)
   std::set<int> v9Iters;  // pipeline depths I at which V9 (deadlock freedom) has been verified
+  bool hasMultimem = false;
 };
 
 namespace {
@@ -212,7 +218,7 @@ mscclResult_t allocRegion(mscclComm* c) {
   DeviceGuard g(c->dev);
   c->fifoBytes = c->fifoBase(3);
   c->flagsOff = c->fifoBytes;
-  c->regionBytes = c->statsOff() + 128;
+  c->regionBytes = c->mmLineOff() + c->mmBytes();
   CUDACHECK(c, cudaMalloc(&c->region, c->regionBytes));
   CUDACHECK(c, cudaMemset(c->region, 0, c->regionBytes));
   c->hRegMap.assign((size_t)c->nranks * c->prm.regMax, nullptr);
@@ -277,6 +283,14 @@ mscclResult_t coResident(mscclComm* c, const void* fn, int threads, int smem, in
   CUDACHECK(c, cudaOccupancyMaxActiveBlocksPerMultiprocessor(&nb, fn, threads, smem));
   out = nsm * nb;
   cache[key] = out;
+  return mscclSuccess;
+}
+
+// the device copy of peerBase (multimem group barriers address every rank's region)
+mscclResult_t uploadPeerRegions(mscclComm* c) {
+  DeviceGuard g(c->dev);
+  if (!c->dPeerRegion) CUDACHECK(c, cudaMalloc(&c->dPeerRegion, c->nranks * sizeof(char*)));
+  CUDACHECK(c, cudaMemcpy(c->dPeerRegion, c->peerBase.data(), c->nranks * sizeof(char*), cudaMemcpyHostToDevice));
   return mscclSuccess;
 }
 
@@ -431,6 +445,11 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
     bool aliasedAny = false;
     for (auto* cl : v) aliasedAny = aliasedAny || cl->aliased;
     if (direct == 1 && aliasedAny) direct = 0;  // ADVICE: in-place call of an out-of-place program
+    // multimem ops (reading R23): buffers of every rank from this launch (mode 1) or through the
+    // group barrier's published references (mode 2)
+    const int mm = p0->hasMultimem ? (allHere ? 1 : 2) : 0;
+    if (mm && v[0]->op == mscclProd && p0->hasReduce)
+      return setErr(c0, mscclInvalidArgument, "multimem reductions support sum/max/min (no product, reading R23)");
     bool noFifo = direct == 1 && c0->prm.directTile;
     for (auto* cl : v) noFifo = noFifo && cl->prog->allDirect;
     Geometry g{};
@@ -451,6 +470,8 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
     ka.trace = traceBuffer();
     ka.direct = direct;
     ka.directHints = (int32_t)c0->prm.directHints;
+    ka.mm = mm;
+    ka.mmLineOff = (int64_t)c0->mmLineOff();
     int cta = 0;
     for (int i = 0; i < (int)v.size(); i++) {
       Call* cl = v[i];
@@ -475,27 +496,36 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
       ra.abortFlag = (uint32_t*)(cl->comm->region + cl->comm->abortOff());
       ra.hostAbort = cl->comm->hostAbortDev;
       ra.regMap = cl->comm->dRegMap;
+      ra.peerRegion = cl->comm->dPeerRegion;
+      ra.myRank = cl->comm->rank;
+      ra.nRanks = cl->comm->nranks;
       ra.stats = (unsigned long long*)(cl->comm->region + cl->comm->statsOff());
       ra.regMax = (int32_t)cl->comm->prm.regMax;
       if (direct == 1) {
         ra.directMask = 7;
-      } else if (direct == 2 && !cl->aliased) {
+      } else if ((direct == 2 || mm == 2) && !cl->aliased) {
         const int Rr = cl->comm->nranks;
         const size_t bytes[3] = {(size_t)g.n * blocksOf(p->algo.coll, BUF_IN, Rr) * w,
                                  (size_t)g.n * blocksOf(p->algo.coll, BUF_OUT, Rr) * w, need};
         for (int b = 0; b < 3; b++) {
           ra.bufRef[b] = bufferRef(cl->comm, ra.buf[b], bytes[b]);
-          if (ra.bufRef[b]) ra.directMask |= 1 << b;
+          if (ra.bufRef[b] && direct == 2) ra.directMask |= 1 << b;
         }
       }
+      if (mm == 2 && (!ra.bufRef[0] || !ra.bufRef[1]))
+        return setErr(cl->comm, mscclInvalidUsage,
+                      "a multimem program across processes needs sendbuff and recvbuff inside registered buffers "
+                      "(mscclCommRegister; reading R23)");
       cta += p->nTB;
       if (cl->comm->sysScope) ka.sysScope = 1;
       if (direct == 1) cl->comm->launchesDirect1++;
       if (direct == 2 && ra.directMask) cl->comm->launchesDirect2++;
     }
     if (cta == 0) continue;
-    const void* fn = p0->hasReduce ? interpreterKernel(v[0]->dtype, v[0]->op, ka.proto)
-                                   : copyKernel(elemBytes(v[0]->dtype), ka.proto);
+    const void* fn = p0->hasMultimem ? (p0->hasReduce ? interpreterKernelMM(v[0]->dtype, v[0]->op)
+                                                      : copyKernelMM(elemBytes(v[0]->dtype)))
+                     : p0->hasReduce ? interpreterKernel(v[0]->dtype, v[0]->op, ka.proto)
+                                     : copyKernel(elemBytes(v[0]->dtype), ka.proto);
     int maxCta = 0;
     r = coResident(c0, fn, (int)c0->prm.threads, 0, maxCta);
     if (r != mscclSuccess) return r;
@@ -681,6 +711,8 @@ mscclResult_t mscclCommInitAll(mscclComm_t* comms, int ndev, const int* devlist)
       }
     }
     c->connected = true;
+    mscclResult_t ur = uploadPeerRegions(c);
+    if (ur != mscclSuccess) return ur;
   }
   for (int i = 0; i < ndev; i++) comms[i] = clique->comms[i];
   return mscclSuccess;
@@ -697,7 +729,11 @@ mscclResult_t mscclCommInitRank(mscclComm_t* comm, int nranks, int rank, int cud
     delete c;
     return r;
   }
-  if (nranks == 1) c->connected = true;
+  if (nranks == 1) {
+    c->connected = true;
+    r = uploadPeerRegions(c);
+    if (r != mscclSuccess) return r;
+  }
   *comm = c;
   return mscclSuccess;
 }
@@ -748,7 +784,7 @@ mscclResult_t mscclCommConnect(mscclComm_t c, const void* allHandles) {
     c->sysScope = true;
   }
   c->connected = true;
-  return mscclSuccess;
+  return uploadPeerRegions(c);
 }
 
 mscclResult_t mscclCommDestroy(mscclComm_t c) {
@@ -762,6 +798,7 @@ mscclResult_t mscclCommDestroy(mscclComm_t c) {
       if (r) releaseReg(c, r);
     c->regs.clear();
     cudaFree(c->dRegMap);
+    cudaFree(c->dPeerRegion);
     for (int p = 0; p < c->nranks; p++)
       if (c->peerIpc[p]) cudaIpcCloseMemHandle(c->peerBase[p]);
     cudaFree(c->region);
@@ -983,6 +1020,10 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
   p->hasReduce = p->algo.hasReduce();
   const GpuProgram& g = p->algo.gpus[c->rank];
   p->nTB = (int)g.tbs.size();
+  p->hasMultimem = p->algo.hasMultimem();
+  if (p->hasMultimem && c->nranks > MSCCL_MM_MAX_RANKS)
+    return setErr(c, mscclInvalidProgram, "V11: multimem programs support at most 16 ranks");
+  const uint32_t tag = ++c->loadCounter;
   const DirectInfo dinfo = directPlacement(p->algo, c->rank);
   std::vector<DevTB> tbs(p->nTB);
   std::vector<DevInstr> ins;
@@ -995,6 +1036,12 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
     d.instrStart = (uint32_t)ins.size();
     d.tbId = tb.id;
     d.sendPeer = tb.send;
+    d.mmId = -1;
+    d.mmTag = tag;
+    for (auto& in : tb.steps)
+      if (isMultimem(in.op)) d.mmId = tb.id;
+    if (d.mmId >= MSCCL_MM_MAX_TB)
+      return setErr(c, mscclInvalidProgram, "V11: a multimem thread block id must be < 64 (group-barrier lines)");
     const int pr = p->algo.proto;
     if (tb.send >= 0) {
       d.sendFifo = c->peerBase[tb.send] + c->fifoOff(pr, c->rank, tb.chan);

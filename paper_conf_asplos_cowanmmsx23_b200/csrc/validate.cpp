@@ -151,6 +151,8 @@ void validateIR(Algo& a, int nranks, int slots, int maxTbs, int maxChannels, int
           if (x.off < 0 || (long long)x.off + in.cnt > nch[x.buf]) fail("V6", w + ": chunk range exceeds the buffer");
         }
         if (ro.dst && in.dstBuf == BUF_IN && !a.inplace) fail("V3", w + ": out-of-place program writes the input buffer");
+        if (isMultimem(in.op) && (in.srcBuf == BUF_SC || in.dstBuf == BUF_SC))
+          fail("V11", w + ": multimem op on the scratch buffer (per-rank sizes)");
         for (auto& d : in.deps) {
           if (d.first == tb.id) fail("V8", w + ": depends on its own thread block");
           if (d.first < 0 || d.first >= (int)g.tbs.size() || d.second < 0 ||
@@ -177,6 +179,21 @@ void validateIR(Algo& a, int nranks, int slots, int maxTbs, int maxChannels, int
     if (sc.size() != rc.size()) fail("V7", "connection: number of sends differs from number of receives");
     for (size_t k = 0; k < sc.size(); k++)
       if (sc[k] != rc[k]) fail("V7", "connection: k-th send and k-th receive carry different cnt");
+  }
+  // V11: the thread blocks holding multimem ops have the same ids on every rank (their
+  // start / end group barrier pairs block b of every rank, reading R23)
+  std::vector<int> mm0;
+  for (auto& g : a.gpus) {
+    std::vector<int> mm;
+    for (auto& tb : g.tbs)
+      for (auto& in : tb.steps)
+        if (isMultimem(in.op)) {
+          mm.push_back(tb.id);
+          break;
+        }
+    if (!mm.empty() && a.proto != PROTO_SIMPLE) fail("V11", "multimem programs use the Simple protocol");
+    if (g.id == 0) mm0 = mm;
+    else if (mm != mm0) fail("V11", where(g.id, mm.empty() ? 0 : mm[0]) + ": multimem thread blocks differ from rank 0's");
   }
   deadlockCheck(a, slots, iters);
 }

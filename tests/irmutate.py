@@ -129,7 +129,8 @@ def random_bases():
     return [(P.ring_allreduce(4).to_xml(), 4), (P.allpairs_allreduce(4).to_xml(), 4),
             (P.ring_allgather(4, 1, 2).to_xml(), 4), (P.ring_reducescatter(4, 1, 1).to_xml(), 4),
             (P.alltoall_twostep(2, 2).to_xml(), 4), (P.hierarchical_allreduce(2, 2).to_xml(), 4),
-            (P.ring_allreduce(4, inplace=True).to_xml(), 4), (P.oneshot_allreduce(4).to_xml(), 4)]
+            (P.ring_allreduce(4, inplace=True).to_xml(), 4), (P.oneshot_allreduce(4).to_xml(), 4),
+            (P.nvls_allreduce(4, 2).to_xml(), 4), (P.nvls_allgather(4).to_xml(), 4)]
 
 
 def mutate(text, rng):
@@ -140,7 +141,7 @@ def mutate(text, rng):
     vals = ["-2", "-1", "0", "1", "2", "3", "4", "7", "65536", "x", "-"]
     if kind == 0 and steps:
         st = rng.choice(steps); a = rng.choice(["type","srcbuf","srcoff","dstbuf","dstoff","cnt","depid","deps","hasdep"])
-        if a == "type": st.set(a, rng.choice(["s","r","cpy","re","rrc","rrs","rrcs","rcs","nop","zz"]))
+        if a == "type": st.set(a, rng.choice(["s","r","cpy","re","rrc","rrs","rrcs","rcs","nop","zz","mrd","mst","mrs"]))
         elif a.endswith("buf"): st.set(a, rng.choice(["i","o","s","-","q"]))
         else: st.set(a, rng.choice(vals))
     elif kind == 1:

@@ -53,6 +53,12 @@ def _algo(name, W, proto):
         return P.ring_allgather(W, 1, 2, protocol=proto)
     if name == "reducescatter":
         return P.ring_reducescatter(W, 1, 2, protocol=proto)
+    if name == "nvls_ar":
+        return P.nvls_allreduce(W, 2)
+    if name == "nvls_rs":
+        return P.nvls_reducescatter(W, 2)
+    if name == "nvls_ag":
+        return P.nvls_allgather(W, 2)
     raise KeyError(name)
 
 
@@ -79,6 +85,11 @@ CASES = [
     ("allgather", "LL128", "uint8", None, 3333, False),
     ("reducescatter", "Simple", "float32", "sum", 5001, True),
     ("reducescatter", "LL", "float32", "prod", 1201, False),
+    # multimem (NVLS) programs across processes: group barrier + registered buffers (reading R23)
+    ("nvls_ar", "Simple", "bfloat16", "sum", 20011, True),
+    ("nvls_ar", "Simple", "int32", "max", 7001, True),
+    ("nvls_rs", "Simple", "float32", "sum", 9001, True),
+    ("nvls_ag", "Simple", "int32", None, 5003, True),
 ]
 
 
@@ -90,8 +101,8 @@ def _inputs(name, W, n, dtype):
     import synth
     from oracle import geometry
     algo = _algo(name, W, "Simple")
-    coll = {"a2a": "alltoall", "a2a_2step": "alltoall", "allgather": "allgather",
-            "reducescatter": "reducescatter"}.get(name, "allreduce")
+    coll = {"a2a": "alltoall", "a2a_2step": "alltoall", "allgather": "allgather", "nvls_ag": "allgather",
+            "reducescatter": "reducescatter", "nvls_rs": "reducescatter"}.get(name, "allreduce")
     elems = geometry.buffer_elems(coll, "i", W, n)
     del algo
     dist = "pattern" if coll in ("alltoall", "allgather") else ("uniform" if dtype.startswith(("float", "bf"))
@@ -189,7 +200,7 @@ def _run_world(world, cases, timeout):
             handshakes += hs
         # device-side evidence of cross-launch direct placement (reading R15b): senders found
         # a registered destination exactly when the buffers were registered
-        if not reg or proto != "Simple":
+        if not reg or proto != "Simple" or name.startswith("nvls"):
             assert handshakes == 0, (name, proto, handshakes)
         elif name in DIRECT_EXPECTED:
             assert handshakes > 0, (name, proto, handshakes)

@@ -1,0 +1,72 @@
+"""GPU parity of the multimem (NVLS) ops (reading R23) on virtual
+ranks: every rank of the group is in one launch, so the interpreter reaches every rank's
+buffer directly (the unicast form of multimem ld_reduce / st). Outputs are compared bit for
+bit with the oracle simulator (fp32 accumulation and one rounding for fp16 / bf16 sums,
+ascending-rank fold), and with the MPI definitions on integer-valued inputs. The
+cross-process form (group barrier, registered buffers) is covered by
+tests/test_gpu_multiprocess.py."""
+import numpy as np
+import pytest
+
+import synth
+from oracle import irparse, mpi_ref, sim
+from paper_conf_asplos_cowanmmsx23_b200 import programs as P
+
+pytestmark = pytest.mark.gpu
+
+
+def _run(algo, xs, n, dtype, op, out_elems=None):
+    import gpu_util
+    return gpu_util.run_program(algo.to_xml(), xs, n, dtype, op, out_elems=out_elems)
+
+
+@pytest.mark.parametrize("R", [2, 4, 8])
+@pytest.mark.parametrize("r", [1, 2, 4])
+@pytest.mark.parametrize("dtype,op", [("bfloat16", "sum"), ("float16", "sum"), ("float32", "sum"),
+                                      ("float32", "max"), ("int32", "sum"), ("bfloat16", "min"),
+                                      ("float64", "sum"), ("uint8", "max")])
+def test_nvls_allreduce_bit_exact(R, r, dtype, op):
+    n = 4097 * r + 13
+    dist = "uniform" if dtype.startswith(("float", "bf")) else "int"
+    xs = synth.inputs(R, n, dtype, dist)
+    algo = P.nvls_allreduce(R, r)
+    want = sim.simulate(irparse.parse(algo.to_xml()), xs, n, dtype, op)
+    got = _run(algo, xs, n, dtype, op)
+    for g, w in zip(got, want):
+        assert np.array_equal(np.asarray(g).view(np.uint8), np.asarray(w).view(np.uint8))
+
+
+@pytest.mark.parametrize("R", [4, 8])
+def test_nvls_allreduce_integer_valued_matches_mpi(R):
+    n = 100003
+    xs = synth.inputs(R, n, "bfloat16", "intval")
+    got = _run(P.nvls_allreduce(R, 2), xs, n, "bfloat16", "sum")
+    from oracle import numerics as nm
+    ref = mpi_ref.allreduce(xs, "sum", "bfloat16")[0]
+    for g in got:
+        assert np.array_equal(nm.to_f64(g, "bfloat16"), ref)
+
+
+@pytest.mark.parametrize("R", [2, 4, 8])
+def test_nvls_reducescatter_and_allgather(R):
+    n = 30011
+    xs = synth.inputs(R, R * n, "float32", "uniform")
+    algo = P.nvls_reducescatter(R, 2)
+    want = sim.simulate(irparse.parse(algo.to_xml()), xs, n, "float32", "sum")
+    got = _run(algo, xs, n, "float32", "sum", out_elems=n)
+    for g, w in zip(got, want):
+        assert np.array_equal(g.view(np.uint32), w.view(np.uint32))
+    xs = synth.inputs(R, n, "int32", "pattern")
+    got = _run(P.nvls_allgather(R, 2), xs, n, "int32", out_elems=R * n)
+    for g, w in zip(got, mpi_ref.allgather(xs)):
+        assert np.array_equal(g, w)
+
+
+def test_nvls_prod_rejected():
+    import gpu_util
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    R, n = 4, 1000
+    xs = synth.inputs(R, n, "float32", "uniform")
+    with pytest.raises(runtime.MscclError) as ei:
+        gpu_util.run_program(P.nvls_allreduce(R).to_xml(), xs, n, "float32", "prod")
+    assert ei.value.code == 4

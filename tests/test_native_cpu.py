@@ -47,6 +47,9 @@ VALID = [
     ("rs", lambda: P.ring_reducescatter(8, 2, 1), 8),
     ("a2a", lambda: P.alltoall_twostep(2, 4), 8),
     ("a2n", lambda: P.alltonext(2, 3), 6),
+    ("nvls_ar", lambda: P.nvls_allreduce(8, 4), 8),
+    ("nvls_rs", lambda: P.nvls_reducescatter(4, 2), 4),
+    ("nvls_ag", lambda: P.nvls_allgather(8), 8),
 ]
 
 
@@ -117,3 +120,19 @@ def test_cpp_and_python_validators_agree_on_random_mutants(rt, seed):
             accepted += 1
     assert {"V1", "V2", "V3", "V4", "V5", "V6", "V7", "V8"} <= seen, seen  # V9: deadlock fixtures above
     assert 50 < accepted < 900
+
+
+def test_cpp_v11_multimem_rules(rt):
+    """V11 in the loader: multimem programs use the Simple protocol, never touch scratch, and
+    hold their multimem ops in the same thread blocks on every rank (reading R23)."""
+    ll = P.nvls_allreduce(4).to_xml().replace('proto="Simple"', 'proto="LL"')
+    ok, msg = rt.validate(ll, 4)
+    assert not ok and msg.startswith("V11"), msg
+    sc = P.nvls_allreduce(4).to_xml().replace('type="mrs" srcbuf="i"', 'type="mrs" srcbuf="s"', 1).replace(
+        's_chunks="0"', 's_chunks="4"')
+    ok, msg = rt.validate(sc, 4)
+    assert not ok and msg.startswith("V11"), msg
+    from oracle import validate as pv
+    for text in (ll, sc):
+        with pytest.raises(pv.ValidationError, match="^V11"):
+            pv.validate(irparse.parse(text), nranks=4)
