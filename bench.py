@@ -58,7 +58,7 @@ def parse():
     ap.add_argument("--ranks", type=int, default=8, help="virtual ranks when N=1")
     ap.add_argument("--size-mib", type=float, default=256.0, help="bytes per rank (MiB)")
     ap.add_argument("--program", default="ring",
-                    choices=["ring", "allpairs", "oneshot", "alltoall", "allgather", "reducescatter"])
+                    choices=["ring", "allpairs", "oneshot", "alltoall", "allgather", "reducescatter", "nvls"])
     ap.add_argument("--channels", type=int, default=1)
     ap.add_argument("--instances", type=int, default=32)
     ap.add_argument("--protocol", default="Simple")
@@ -173,6 +173,8 @@ def build_program(args, R):
         return P.allpairs_allreduce(R, instances=args.instances, protocol=args.protocol)
     if args.program == "oneshot":
         return P.oneshot_allreduce(R, instances=args.instances, protocol=args.protocol)
+    if args.program == "nvls":
+        return P.nvls_allreduce(R, args.instances)
     if args.program == "allgather":
         return P.ring_allgather(R, args.channels, args.instances, protocol=args.protocol)
     if args.program == "reducescatter":
@@ -287,11 +289,13 @@ def config_dict(args, R, N):
                 "oneshot": "BASELINE configs[2] shape (one-shot AllReduce)",
                 "alltoall": "BASELINE configs[3] shape (AllToAll)",
                 "allgather": "BASELINE configs[4] shape (ring AllGather)",
+                "nvls": "BASELINE configs[1] shape with the multimem (NVLS) AllReduce program",
                 "reducescatter": "BASELINE configs[4] shape (ring ReduceScatter)"}[args.program]
         mode = "%d virtual ranks on 1 B200 (HBM-bound)" % R
     else:
         base = {"ring": "BASELINE configs[1]: ring AllReduce, bf16", "allpairs": "all-pairs AllReduce",
                 "oneshot": "one-shot AllReduce", "alltoall": "BASELINE configs[3]: AllToAll",
+                "nvls": "multimem (NVLS) AllReduce",
                 "allgather": "BASELINE configs[4]: ring AllGather", "reducescatter": "BASELINE configs[4]: ring "
                 "ReduceScatter"}[args.program]
         mode = "%d B200, 1 process per GPU, CUDA IPC over NVLink" % N
@@ -470,7 +474,8 @@ def extras(R, stream, nccl=None, S=256 * MIB):
     # AllToAll (direct two-step N=1), AllGather and ReduceScatter rings: S per rank (256 MiB), bf16
     n = S // 2
     nb = n // W
-    specs = (("alltoall", P.alltoall_twostep(1, W, instances=2 if R.world == 1 else 4), n, n, nb),
+    specs = (("nvls_allreduce", P.nvls_allreduce(W, 32 if R.world == 1 else 8), n, n, n),
+             ("alltoall", P.alltoall_twostep(1, W, instances=2 if R.world == 1 else 4), n, n, nb),
              ("allgather", P.ring_allgather(W, 1, 32 if R.world == 1 else 8), nb, n, nb),
              ("reducescatter", P.ring_reducescatter(W, 1, 32 if R.world == 1 else 8), n, nb, nb))
     for coll, algo, ins, outs, cnt in specs:
@@ -483,13 +488,18 @@ def extras(R, stream, nccl=None, S=256 * MIB):
             ok = check_alltoall(R, recv, W, n)
         elif coll == "allgather":
             ok = check_allgather(R, recv, W, nb)
+        elif coll == "nvls_allreduce":
+            ranks = [q for q in (0, W - 1) if q in R.ranks]
+            bad, _ = sampled_parity(algo, recv, n, ranks, local=R.ranks)
+            ok = bad == 0
         else:
             ranks = [q for q in (0, W - 1) if q in R.ranks]
             bad, _ = sampled_parity(algo, recv, nb, ranks, local=R.ranks)
             ok = bad == 0
-        ent = {"busbw_GBps": round(busbw(coll, S, t, W), 2), "ms": round(t * 1e3, 3),
+        ent = {"busbw_GBps": round(busbw("allreduce" if coll == "nvls_allreduce" else coll, S, t, W), 2),
+               "ms": round(t * 1e3, 3),
                "ctas_per_rank": int(progs[0].info()["thread_blocks"]), "bit_exact": R.all_ok(ok)}
-        if nccl is not None:
+        if nccl is not None and coll != "nvls_allreduce":
             fn = {"alltoall": lambda: nccl.alltoall(send[0], recv[0], "bfloat16", W, cur()),
                   "allgather": lambda: nccl.allgather(send[0], recv[0], "bfloat16", cur()),
                   "reducescatter": lambda: nccl.reducescatter(send[0], recv[0], "bfloat16", "sum", cur())}[coll]

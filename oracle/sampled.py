@@ -16,6 +16,8 @@ from .symbolic import check
 def _eval(tree, leafval, op, dtype):
     if tree[0] == "in":
         return leafval(tree[1], tree[2])
+    if tree[0] == "m+":  # multimem fold over the ranks (reading R23): one rounding
+        return nm.mreduce([_eval(x, leafval, op, dtype) for x in tree[1:]], op, dtype)
     _, a, b = tree
     return nm.reduce(_eval(a, leafval, op, dtype), _eval(b, leafval, op, dtype), op, dtype)
 

@@ -63,11 +63,9 @@ class SymbolicDomain:
         if st.op == "nop":
             return None
         if st.multimem:  # reading R23: the same chunk on every rank, folded in ascending rank order
-            if st.reads_all:
+            if st.reads_all:  # one multimem node: the fold is evaluated with one rounding
                 vals = [self.get(p, st.srcbuf, st.srcoff + j) for p in range(len(self.bufs))]
-                v = vals[0]
-                for x in vals[1:]:
-                    v = combine(v, x)
+                v = (tuple(sorted(sum((x[0] for x in vals), ()))), ("m+",) + tuple(x[1] for x in vals))
             else:
                 v = self.get(q, st.srcbuf, st.srcoff + j)
             for p in range(len(self.bufs)):

@@ -190,3 +190,17 @@ def test_dsl_multimem_rules():
         with dsl.Program("y", dsl.AllReduce(2, 2, inplace=True)):
             c = dsl.chunk(1, "in", 0).copy(0, "in", 0)
             dsl.chunk(0, "in", 0).multimem_reduce("out", 0)
+
+
+def test_sampled_oracle_evaluates_multimem_nodes():
+    """oracle/sampled.py (used at bench sizes) agrees with the full simulation of the NVLS
+    AllReduce bit for bit, including the single rounding of the multimem fold."""
+    from oracle import sampled
+    R, n = 8, 5000
+    xs = synth.inputs(R, n, "bfloat16", "uniform")
+    al = _al(P.nvls_allreduce(R, 2))
+    full = sim.simulate(al, xs, n, "bfloat16", "sum")
+    idx = np.arange(0, n, 7)
+    for q in (0, 5):
+        got = sampled.allreduce_at(al, lambda r, i: xs[r][i], n, "bfloat16", "sum", idx, rank=q)
+        assert np.array_equal(got, full[q][idx])
