@@ -15,7 +15,7 @@ from paper_conf_asplos_cowanmmsx23_b200 import programs as P
 pytestmark = pytest.mark.gpu
 
 
-def _run(algo, xs, n, dtype, op, out_elems=None):
+def _run(algo, xs, n, dtype, op="sum", out_elems=None):
     import gpu_util
     return gpu_util.run_program(algo.to_xml(), xs, n, dtype, op, out_elems=out_elems)
 
