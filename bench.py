@@ -208,6 +208,25 @@ def nop_ir(R):
     return '<algo name="nop" coll="custom" ngpus="%d" proto="LL" inplace="0" nchannels="1">%s</algo>' % (R, g)
 
 
+def hop_ir(R, proto="LL"):
+    """One message hop: rank r sends its chunk to rank r+1 (AllToNext without the cross-node
+    relay, §7.4). Its latency minus the launch floor is the cost of one hop of the
+    protocol; the 1 KiB breakdown in DESIGN.md §7 reads the one-shot and ring latencies
+    against floor + hops."""
+    g = []
+    for q in range(R):
+        tbs = []
+        if q + 1 < R:
+            tbs.append('<tb id="%d" send="%d" recv="-1" chan="0"><step s="0" type="s" srcbuf="i" srcoff="0" '
+                       'dstbuf="-" dstoff="-1" cnt="1" depid="-1" deps="-1" hasdep="0"/></tb>' % (len(tbs), q + 1))
+        if q > 0:
+            tbs.append('<tb id="%d" send="-1" recv="%d" chan="0"><step s="0" type="r" srcbuf="-" srcoff="-1" '
+                       'dstbuf="o" dstoff="0" cnt="1" depid="-1" deps="-1" hasdep="0"/></tb>' % (len(tbs), q - 1))
+        g.append('<gpu id="%d" i_chunks="1" o_chunks="1" s_chunks="0">%s</gpu>' % (q, "".join(tbs)))
+    return '<algo name="hop" coll="custom" ngpus="%d" proto="%s" inplace="0" nchannels="1">%s</algo>' % (
+        R, proto, "".join(g))
+
+
 def host_threads():
     try:
         return len(os.sched_getaffinity(0))
@@ -449,12 +468,15 @@ def extras(R, stream, nccl=None, S=256 * MIB):
     n = 512  # 1 KiB of fp16 per rank
     send = [synth.hashed(q, torch.arange(n, device=R.dev), "float16") for q in R.ranks]
     recv = [torch.empty_like(x) for x in send]
-    for name, algo in (("floor_nop", None), ("oneshot_LL", P.oneshot_allreduce(W, protocol="LL")),
+    for name, algo in (("floor_nop", None), ("one_hop_LL", "hop"), ("one_hop_LL128", "hop128"),
+                       ("oneshot_LL", P.oneshot_allreduce(W, protocol="LL")),
                        ("allpairs_LL", P.allpairs_allreduce(W, protocol="LL")),
                        ("ring_LL", P.ring_allreduce(W, protocol="LL")),
                        ("ring_ch%d_LL" % W, P.ring_allreduce(W, channels=W, protocol="LL"))):
         if algo is None:
             progs = [c.load(nop_ir(W)) for c in R.comms]
+        elif algo in ("hop", "hop128"):
+            progs = [c.load(hop_ir(W, "LL" if algo == "hop" else "LL128")) for c in R.comms]
         else:
             progs = R.load(algo, 0, 1 << 20)
         try:
@@ -468,7 +490,8 @@ def extras(R, stream, nccl=None, S=256 * MIB):
         t, mode = timed(lambda: nccl.allreduce(send[0], recv[0], "float16", stream=cur()), 50, 5, stream, True, R)
         lat["nccl_allreduce"] = round(t * 1e6, 2)
     lat["note"] = ("floor_nop = an MSCCL-IR program of one nop per rank: cooperative launch + prologue + "
-                   "epilogue under graph replay; the collective latencies are read against it")
+                   "epilogue under graph replay; one_hop = rank r sends 1 KiB to rank r+1 (one message of the "
+                   "protocol); the collective latencies are read against floor + hops")
     out["allreduce_1KiB_fp16_latency_us"] = lat
     del send, recv
     # AllToAll (direct two-step N=1), AllGather and ReduceScatter rings: S per rank (256 MiB), bf16

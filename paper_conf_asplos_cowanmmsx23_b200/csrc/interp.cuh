@@ -914,10 +914,10 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
 // with fp32 accumulation and one rounding for fp16 / bf16 sums (what the switch's .acc::f32
 // reduction computes), and one store per rank.
 template <int DT, int OP>
-struct MMAcc {  // fold of R 16-byte vectors in ascending rank order
+struct MMAcc {  // fold of R 32-byte vectors in ascending rank order
   static constexpr bool kHalfSum = (DT == DT_BF16 || DT == DT_F16) && OP == R_SUM;
-  float f[8];
-  uint4 v;
+  float f[16];
+  V32 v;
   static __device__ __forceinline__ float widen(uint16_t x) {
     if constexpr (DT == DT_BF16) return __uint_as_float(((uint32_t)x) << 16);
     else return __half2float(__ushort_as_half(x));
@@ -926,30 +926,30 @@ struct MMAcc {  // fold of R 16-byte vectors in ascending rank order
     if constexpr (DT == DT_BF16) return __bfloat16_as_ushort(__float2bfloat16_rn(x));
     else return __half_as_ushort(__float2half_rn(x));
   }
-  __device__ __forceinline__ void first(const uint4& x) {
+  __device__ __forceinline__ void first(const V32& x) {
     if constexpr (kHalfSum) {
       const uint16_t* h = reinterpret_cast<const uint16_t*>(&x);
 #pragma unroll
-      for (int k = 0; k < 8; k++) f[k] = widen(h[k]);
+      for (int k = 0; k < 16; k++) f[k] = widen(h[k]);
     } else {
       v = x;
     }
   }
-  __device__ __forceinline__ void add(const uint4& x) {
+  __device__ __forceinline__ void add(const V32& x) {
     if constexpr (kHalfSum) {
       const uint16_t* h = reinterpret_cast<const uint16_t*>(&x);
 #pragma unroll
-      for (int k = 0; k < 8; k++) f[k] = f[k] + widen(h[k]);
+      for (int k = 0; k < 16; k++) f[k] = f[k] + widen(h[k]);
     } else {
       v = vop<DT, OP>(v, x);
     }
   }
-  __device__ __forceinline__ uint4 result() const {
+  __device__ __forceinline__ V32 result() const {
     if constexpr (kHalfSum) {
-      uint4 r;
+      V32 r;
       uint16_t* h = reinterpret_cast<uint16_t*>(&r);
 #pragma unroll
-      for (int k = 0; k < 8; k++) h[k] = narrow(f[k]);
+      for (int k = 0; k < 16; k++) h[k] = narrow(f[k]);
       return r;
     } else {
       return v;
@@ -957,12 +957,17 @@ struct MMAcc {  // fold of R 16-byte vectors in ascending rank order
   }
 };
 
+#ifndef MSCCL_MM_BATCH
+#define MSCCL_MM_BATCH 4  // ranks whose 32-byte loads are in flight together (multimem path)
+#endif
+
 template <int DT, int OP, int KIND>
 __device__ __noinline__ void runMultimem(const Ctx& c, const DevInstr& in, int t) {
   typedef typename DType<DT>::T T;
   const KernelArgs& a = *c.a;
   const RankArgs& ra = *c.ra;
   constexpr bool RALL = KIND != K_MST, WALL = KIND != K_MRD;
+  constexpr int B = MSCCL_MM_BATCH;
   const int R = ra.nRanks, me = ra.myRank;
   const int64_t w = sizeof(T), a0 = (int64_t)t * a.T;
   const uint64_t pol = policyEvictFirst();
@@ -976,32 +981,32 @@ __device__ __noinline__ void runMultimem(const Ctx& c, const DevInstr& in, int t
     const int64_t so = (ss + a0) * w, dof = (ds + a0) * w;
     uintptr_t al = (uintptr_t)so | (uintptr_t)dof;
     for (int p = 0; p < R; p++) al |= (uintptr_t)c.mmBuf[p][in.srcBuf] | (uintptr_t)c.mmBuf[p][in.dstBuf];
-    const int64_t nvec = (al & 15) ? 0 : m * w / 16;
+    const int64_t nvec = (al & 31) ? 0 : m * w / 32;
     for (int64_t i = c.tid; i < nvec; i += c.nt) {
       MMAcc<DT, OP> acc;
-      if constexpr (RALL) {  // 4 ranks' loads in flight, folded in ascending rank order
-        for (int p0 = 0; p0 < R; p0 += 4) {
-          uint4 x[4];
+      if constexpr (RALL) {  // B ranks' 256-bit loads in flight, folded in ascending rank order
+        for (int p0 = 0; p0 < R; p0 += B) {
+          V32 x[B];
 #pragma unroll
-          for (int u = 0; u < 4; u++)
-            if (p0 + u < R) ldStream(x[u], c.mmBuf[p0 + u][in.srcBuf] + so + i * 16, pol);
+          for (int u = 0; u < B; u++)
+            if (p0 + u < R) ldStream(x[u], c.mmBuf[p0 + u][in.srcBuf] + so + i * 32, pol);
 #pragma unroll
-          for (int u = 0; u < 4; u++) {
+          for (int u = 0; u < B; u++) {
             if (p0 + u >= R) break;
             if (p0 + u == 0) acc.first(x[u]);
             else acc.add(x[u]);
           }
         }
       } else {
-        uint4 x;
-        ldStream(x, c.mmBuf[me][in.srcBuf] + so + i * 16, pol);
+        V32 x;
+        ldStream(x, c.mmBuf[me][in.srcBuf] + so + i * 32, pol);
         acc.first(x);
       }
-      const uint4 v = acc.result();
+      const V32 v = acc.result();
       for (int p = 0; p < R; p++)
-        if (WALL || p == me) stHint(c.mmBuf[p][in.dstBuf] + dof + i * 16, v, pol);
+        if (WALL || p == me) stHint(c.mmBuf[p][in.dstBuf] + dof + i * 32, v, pol);
     }
-    for (int64_t e = nvec * 16 / w + c.tid; e < m; e += c.nt) {  // scalar tail (ragged or unaligned)
+    for (int64_t e = nvec * 32 / w + c.tid; e < m; e += c.nt) {  // scalar tail (ragged or unaligned)
       T v;
       if constexpr (RALL) {
         if constexpr (MMAcc<DT, OP>::kHalfSum) {
