@@ -97,7 +97,8 @@ mscclResult_t mscclCommCount(const mscclComm_t comm, int* count);
  * [0] cross-launch ready handshakes in which a sender of this rank found a reachable
  *     destination and stored directly into a peer (device-side count, reading R15b);
  * [1] launches with one-launch direct placement (every rank in the launch, reading R15);
- * [2] launches in which this rank published a reachable destination (cross-launch mode). */
+ * [2] launches in which this rank published a reachable destination (cross-launch mode);
+ * [3] multimem pieces executed through an NVSwitch multicast address (device-side count). */
 mscclResult_t mscclCommGetStats(mscclComm_t comm, int64_t* stats, int n);
 mscclResult_t mscclCommUserRank(const mscclComm_t comm, int* rank);
 mscclResult_t mscclCommCuDevice(const mscclComm_t comm, int* device);
@@ -130,6 +131,22 @@ mscclResult_t mscclCommRegister(mscclComm_t comm, void* buff, size_t size, msccl
 mscclResult_t mscclRegExport(mscclReg_t reg, void* desc);
 mscclResult_t mscclRegConnect(mscclReg_t reg, const void* allDescs);
 mscclResult_t mscclCommDeregister(mscclComm_t comm, mscclReg_t reg);
+
+/* ---------------------------------------------------------------- NVLS buffers
+ * NVSwitch multicast (reading R23). mscclNvlsAlloc allocates
+ * `bytes` on every rank's GPU of one single-process communicator set (mscclCommInitAll, one
+ * rank per distinct device, comms in rank order), binds all of them to one multicast
+ * object, and writes each rank's (unicast) pointer to ptrs[rank]. A multimem program whose
+ * sendbuff / recvbuff lie inside such a buffer (at the same offset on every rank) runs its
+ * mrd / mst / mrs instructions as multimem.ld_reduce / multimem.st on the multicast address
+ * (fp16 / bf16 / fp32 sums, and stores of any type; other dtype / op pairs and buffers
+ * outside NVLS buffers use the unicast form). Not capturable (allocates). Errors:
+ * InvalidArgument (not a full rank-ordered clique), InvalidUsage (two ranks on one device),
+ * SystemError (no multicast support), UnhandledCudaError. mscclNvlsSupported reports
+ * CU_DEVICE_ATTRIBUTE_MULTICAST_SUPPORTED of a device (0 when the driver lacks the API). */
+mscclResult_t mscclNvlsSupported(int cudaDev, int* supported);
+mscclResult_t mscclNvlsAlloc(mscclComm_t* comms, int ncomms, size_t bytes, void** ptrs);
+mscclResult_t mscclNvlsFree(mscclComm_t* comms, int ncomms, void** ptrs);
 
 /* ---------------------------------------------------------------- programs */
 

@@ -82,6 +82,10 @@ struct RankArgs {
                               // resolved a direct destination (mscclCommGetStats)
   char* const* peerRegion;    // every rank's shared region in this address space (group barriers)
   int32_t myRank, nRanks;
+  // NVSwitch multicast addresses of this rank's in / out buffers when they lie inside an
+  // NVLS buffer (mscclNvlsAlloc), else null: multimem ops on them use multimem.ld_reduce /
+  // multimem.st (the hardware form of reading R23)
+  char* mcBuf[2];
 };
 
 struct KernelArgs {

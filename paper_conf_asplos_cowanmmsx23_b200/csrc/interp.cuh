@@ -961,6 +961,56 @@ struct MMAcc {  // fold of R 32-byte vectors in ascending rank order
 #define MSCCL_MM_BATCH 4  // ranks whose 32-byte loads are in flight together (multimem path)
 #endif
 
+// Hardware multicast (NVLS): one multimem.ld_reduce returns the reduction of the 16 bytes at
+// this address over every GPU bound to the multicast object; multimem.st writes 16 bytes to
+// all of them. fp16 / bf16 sums accumulate in fp32 inside the switch (.acc::f32, reading R23).
+template <int DT, int OP>
+struct MCOps {
+  static constexpr bool kReduce = (DT == DT_BF16 || DT == DT_F16 || DT == DT_F32) && OP == R_SUM;
+  static __device__ __forceinline__ uint4 ldReduce(const char* p) {
+    uint4 v;
+    if constexpr (DT == DT_BF16) {
+      asm volatile("multimem.ld_reduce.relaxed.sys.global.add.acc::f32.v4.bf16x2 {%0,%1,%2,%3}, [%4];"
+                   : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
+    } else if constexpr (DT == DT_F16) {
+      asm volatile("multimem.ld_reduce.relaxed.sys.global.add.acc::f32.v4.f16x2 {%0,%1,%2,%3}, [%4];"
+                   : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
+    } else {
+      asm volatile("multimem.ld_reduce.relaxed.sys.global.add.v4.f32 {%0,%1,%2,%3}, [%4];"
+                   : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "l"(p) : "memory");
+    }
+    return v;
+  }
+  static __device__ __forceinline__ void st(char* p, const uint4& v) {  // bit pattern, any dtype
+    asm volatile("multimem.st.relaxed.sys.global.v4.f32 [%0], {%1,%2,%3,%4};" ::"l"(p), "r"(v.x), "r"(v.y),
+                 "r"(v.z), "r"(v.w) : "memory");
+  }
+};
+
+// returns true when the piece was done through the multicast addresses
+template <int DT, int OP, int KIND>
+__device__ __forceinline__ bool multicastPiece(const Ctx& c, const DevInstr& in, int64_t so, int64_t dof, int64_t m) {
+  typedef typename DType<DT>::T T;
+  constexpr bool RALL = KIND != K_MST, WALL = KIND != K_MRD;
+  const RankArgs& ra = *c.ra;
+  const char* ms = ra.mcBuf[in.srcBuf];
+  char* md = ra.mcBuf[in.dstBuf];
+  if (RALL && (!MCOps<DT, OP>::kReduce || !ms)) return false;
+  if (WALL && !md) return false;
+  const int64_t bytes = m * (int64_t)sizeof(T);
+  if ((bytes & 15) || ((so | dof) & 15)) return false;
+  const int64_t nvec = bytes / 16;
+  for (int64_t i = c.tid; i < nvec; i += c.nt) {
+    uint4 v;
+    if constexpr (RALL) v = MCOps<DT, OP>::ldReduce(ms + so + i * 16);
+    else v = ldcg(c.mmBuf[ra.myRank][in.srcBuf] + so + i * 16);
+    if constexpr (WALL) MCOps<DT, OP>::st(md + dof + i * 16, v);
+    else stg(c.mmBuf[ra.myRank][in.dstBuf] + dof + i * 16, v);
+  }
+  if (c.tid == 0) atomicAdd(ra.stats + 1, 1ull);  // evidence: pieces done on the multicast path
+  return true;
+}
+
 template <int DT, int OP, int KIND>
 __device__ __noinline__ void runMultimem(const Ctx& c, const DevInstr& in, int t) {
   typedef typename DType<DT>::T T;
@@ -979,6 +1029,7 @@ __device__ __noinline__ void runMultimem(const Ctx& c, const DevInstr& in, int t
     const int64_t m = (a0 + a.T < L ? a0 + a.T : L) - a0;
     if (m <= 0) continue;
     const int64_t so = (ss + a0) * w, dof = (ds + a0) * w;
+    if (multicastPiece<DT, OP, KIND>(c, in, so, dof, m)) continue;
     uintptr_t al = (uintptr_t)so | (uintptr_t)dof;
     for (int p = 0; p < R; p++) al |= (uintptr_t)c.mmBuf[p][in.srcBuf] | (uintptr_t)c.mmBuf[p][in.dstBuf];
     const int64_t nvec = (al & 31) ? 0 : m * w / 32;
@@ -1066,14 +1117,20 @@ static __device__ __noinline__ bool mmBarrier(const Ctx& c, const DevTB& tb, uin
   }
   if (c.tid < R && c.tid != me) {
     uint64_t* l = mmLine(a, ra.peerRegion[c.tid], start ? 0 : 1, tb.mmId, me, R);
+    const uint64_t mcMask = (ra.mcBuf[0] ? 1u : 0u) | (ra.mcBuf[1] ? 2u : 0u);
     if (start) {
       stRelaxedSys(l + 1, ra.bufRef[0]);
       stRelaxedSys(l + 2, ra.bufRef[1]);
+      stRelaxedSys(l + 3, mcMask);
       fenceSys();
     }
     stRelaxedSys(l, epoch);
     const uint64_t* mine = mmLine(a, ra.peerRegion[me], start ? 0 : 1, tb.mmId, c.tid, R);
     ok = waitEq(mine, epoch, c);
+    if (ok && start && *(volatile const uint64_t*)(mine + 3) != mcMask) {  // NVLS buffers must be symmetric
+      raiseAbort(a);
+      ok = false;
+    }
     if (ok && start) {
       for (int b = 0; b < 2; b++) {
         const uint64_t ref = *(volatile const uint64_t*)(mine + 1 + b);

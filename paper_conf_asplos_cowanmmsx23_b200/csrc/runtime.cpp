@@ -120,6 +120,16 @@ struct mscclComm {
   int maxCoResident = 0;
   uint64_t launchesDirect1 = 0, launchesDirect2 = 0;  // launches this rank took part in, by direct mode
   uint32_t loadCounter = 0;            // programs loaded so far (multimem group-barrier epochs)
+  // NVLS buffers (mscclNvlsAlloc): this rank's unicast range and the multicast address of it
+  struct Nvls {
+    char* uc;
+    char* mc;
+    size_t size;
+    unsigned long long phys;     // CUmemGenericAllocationHandle of this rank's memory
+    unsigned long long mcHandle; // the multicast object (shared by the clique)
+    bool owner;                  // this rank maps / releases the multicast VA
+  };
+  std::vector<Nvls> nvls;
   char** dPeerRegion = nullptr;        // device [nranks]: every rank's region in this address space
   std::vector<mscclReg*> regs;         // by index (nullptr = free)
   char** dRegMap = nullptr;            // device [nranks][regMax]: peers' registered buffers, mapped here
@@ -504,6 +514,14 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
       ra.peerRegion = cl->comm->dPeerRegion;
       ra.myRank = cl->comm->rank;
       ra.nRanks = cl->comm->nranks;
+      if (mm) {  // NVSwitch multicast addresses of in / out (reading R23, hardware form)
+        const int Rr = cl->comm->nranks;
+        const size_t bytes[2] = {(size_t)g.n * blocksOf(p->algo.coll, BUF_IN, Rr) * w,
+                                 (size_t)g.n * blocksOf(p->algo.coll, BUF_OUT, Rr) * w};
+        for (int b = 0; b < 2; b++)
+          for (auto& nv : cl->comm->nvls)
+            if (ra.buf[b] >= nv.uc && ra.buf[b] + bytes[b] <= nv.uc + nv.size) ra.mcBuf[b] = nv.mc + (ra.buf[b] - nv.uc);
+      }
       ra.stats = (unsigned long long*)(cl->comm->region + cl->comm->statsOff());
       ra.regMax = (int32_t)cl->comm->prm.regMax;
       if (direct == 1) {
@@ -631,6 +649,69 @@ mscclResult_t runColl(mscclProgram* p, int coll, const void* sendbuff, void* rec
   return enqueue(cl);
 }
 
+}  // namespace
+
+// ------------------------------------------------------------------ NVLS buffers (reading R23)
+namespace {
+template <typename F>
+F driverFn(const char* name) {
+  void* fn = nullptr;
+  cudaDriverEntryPointQueryResult q;
+  if (cudaGetDriverEntryPoint(name, &fn, cudaEnableDefault, &q) != cudaSuccess || q != cudaDriverEntryPointSuccess)
+    return nullptr;
+  return (F)fn;
+}
+struct Drv {
+  CUresult (*devAttr)(int*, CUdevice_attribute, CUdevice) = nullptr;
+  CUresult (*mcCreate)(CUmemGenericAllocationHandle*, const CUmulticastObjectProp*) = nullptr;
+  CUresult (*mcAddDevice)(CUmemGenericAllocationHandle, CUdevice) = nullptr;
+  CUresult (*mcGran)(size_t*, const CUmulticastObjectProp*, CUmulticastGranularity_flags) = nullptr;
+  CUresult (*mcBindMem)(CUmemGenericAllocationHandle, size_t, CUmemGenericAllocationHandle, size_t, size_t,
+                        unsigned long long) = nullptr;
+  CUresult (*mcUnbind)(CUmemGenericAllocationHandle, CUdevice, size_t, size_t) = nullptr;
+  CUresult (*memCreate)(CUmemGenericAllocationHandle*, size_t, const CUmemAllocationProp*, unsigned long long) = nullptr;
+  CUresult (*memRelease)(CUmemGenericAllocationHandle) = nullptr;
+  CUresult (*memGran)(size_t*, const CUmemAllocationProp*, CUmemAllocationGranularity_flags) = nullptr;
+  CUresult (*addrReserve)(CUdeviceptr*, size_t, size_t, CUdeviceptr, unsigned long long) = nullptr;
+  CUresult (*addrFree)(CUdeviceptr, size_t) = nullptr;
+  CUresult (*memMap)(CUdeviceptr, size_t, size_t, CUmemGenericAllocationHandle, unsigned long long) = nullptr;
+  CUresult (*memUnmap)(CUdeviceptr, size_t) = nullptr;
+  CUresult (*setAccess)(CUdeviceptr, size_t, const CUmemAccessDesc*, size_t) = nullptr;
+  bool ok = false;
+};
+const Drv& drv() {
+  static Drv d;
+  static bool init = false;
+  if (!init) {
+    init = true;
+    d.devAttr = driverFn<decltype(d.devAttr)>("cuDeviceGetAttribute");
+    d.mcCreate = driverFn<decltype(d.mcCreate)>("cuMulticastCreate");
+    d.mcAddDevice = driverFn<decltype(d.mcAddDevice)>("cuMulticastAddDevice");
+    d.mcGran = driverFn<decltype(d.mcGran)>("cuMulticastGetGranularity");
+    d.mcBindMem = driverFn<decltype(d.mcBindMem)>("cuMulticastBindMem");
+    d.mcUnbind = driverFn<decltype(d.mcUnbind)>("cuMulticastUnbind");
+    d.memCreate = driverFn<decltype(d.memCreate)>("cuMemCreate");
+    d.memRelease = driverFn<decltype(d.memRelease)>("cuMemRelease");
+    d.memGran = driverFn<decltype(d.memGran)>("cuMemGetAllocationGranularity");
+    d.addrReserve = driverFn<decltype(d.addrReserve)>("cuMemAddressReserve");
+    d.addrFree = driverFn<decltype(d.addrFree)>("cuMemAddressFree");
+    d.memMap = driverFn<decltype(d.memMap)>("cuMemMap");
+    d.memUnmap = driverFn<decltype(d.memUnmap)>("cuMemUnmap");
+    d.setAccess = driverFn<decltype(d.setAccess)>("cuMemSetAccess");
+    d.ok = d.devAttr && d.mcCreate && d.mcAddDevice && d.mcGran && d.mcBindMem && d.mcUnbind && d.memCreate &&
+           d.memRelease && d.memGran && d.addrReserve && d.addrFree && d.memMap && d.memUnmap && d.setAccess;
+  }
+  return d;
+}
+#define CUCHECK(c, call)                                                                   \
+  do {                                                                                     \
+    CUresult e_ = (call);                                                                  \
+    if (e_ != CUDA_SUCCESS) {                                                              \
+      std::ostringstream o_;                                                               \
+      o_ << #call << " failed with CUresult " << (int)e_;                                  \
+      return setErr((c), e_ == CUDA_ERROR_NOT_SUPPORTED ? mscclSystemError : mscclUnhandledCudaError, o_.str()); \
+    }                                                                                      \
+  } while (0)
 }  // namespace
 
 // ================================================================== C ABI
@@ -956,13 +1037,126 @@ mscclResult_t mscclDebugDirectPlacement(const char* ir, size_t irBytes, int rank
   return mscclSuccess;
 }
 
+
+mscclResult_t mscclNvlsSupported(int cudaDev, int* supported) {
+  if (!supported) return mscclInvalidArgument;
+  *supported = 0;
+  const Drv& d = drv();
+  if (!d.ok) return mscclSuccess;
+  cudaFree(nullptr);  // a current context
+  int v = 0;
+  if (d.devAttr(&v, CU_DEVICE_ATTRIBUTE_MULTICAST_SUPPORTED, (CUdevice)cudaDev) == CUDA_SUCCESS) *supported = v;
+  return mscclSuccess;
+}
+
+mscclResult_t mscclNvlsAlloc(mscclComm_t* comms, int n, size_t bytes, void** ptrs) {
+  if (!comms || n < 1 || !bytes || !ptrs) return setErr(nullptr, mscclInvalidArgument, "mscclNvlsAlloc: bad arguments");
+  mscclComm* c0 = comms[0];
+  for (int i = 0; i < n; i++) {
+    if (!comms[i] || comms[i]->rank != i || comms[i]->nranks != n || (n > 1 && comms[i]->clique != c0->clique) ||
+        (n > 1 && !c0->clique))
+      return setErr(comms[i], mscclInvalidArgument,
+                    "mscclNvlsAlloc: pass every rank of one mscclCommInitAll communicator set, in rank order");
+    for (int j = 0; j < i; j++)
+      if (comms[j]->dev == comms[i]->dev)
+        return setErr(comms[i], mscclInvalidUsage, "mscclNvlsAlloc: a multicast object binds one buffer per GPU "
+                                                   "(virtual ranks cannot share one)");
+  }
+  const Drv& d = drv();
+  if (!d.ok) return setErr(c0, mscclSystemError, "CUDA driver has no multicast API");
+  for (int i = 0; i < n; i++) {
+    int sup = 0;
+    mscclNvlsSupported(comms[i]->dev, &sup);
+    if (!sup) return setErr(comms[i], mscclSystemError, "device does not support NVSwitch multicast");
+  }
+  CUmulticastObjectProp mp;
+  memset(&mp, 0, sizeof(mp));
+  mp.numDevices = (unsigned)n;
+  mp.size = bytes;
+  mp.handleTypes = 0;
+  size_t gran = 0, ugran = 0;
+  {
+    DeviceGuard g(c0->dev);
+    cudaFree(nullptr);
+    CUCHECK(c0, d.mcGran(&gran, &mp, CU_MULTICAST_GRANULARITY_RECOMMENDED));
+  }
+  CUmemAllocationProp ap;
+  memset(&ap, 0, sizeof(ap));
+  ap.type = CU_MEM_ALLOCATION_TYPE_PINNED;
+  ap.location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+  ap.location.id = c0->dev;
+  CUCHECK(c0, d.memGran(&ugran, &ap, CU_MEM_ALLOC_GRANULARITY_RECOMMENDED));
+  size_t g2 = std::max(gran, ugran);
+  const size_t size = (bytes + g2 - 1) / g2 * g2;
+  mp.size = size;
+  CUmemGenericAllocationHandle mc = 0;
+  {
+    DeviceGuard g(c0->dev);
+    CUCHECK(c0, d.mcCreate(&mc, &mp));
+  }
+  for (int i = 0; i < n; i++) CUCHECK(comms[i], d.mcAddDevice(mc, (CUdevice)comms[i]->dev));
+  // the multicast address, mapped once and accessible from every device
+  CUdeviceptr mcva = 0;
+  std::vector<CUmemAccessDesc> acc(n);
+  for (int i = 0; i < n; i++) {
+    acc[i].location.type = CU_MEM_LOCATION_TYPE_DEVICE;
+    acc[i].location.id = comms[i]->dev;
+    acc[i].flags = CU_MEM_ACCESS_FLAGS_PROT_READWRITE;
+  }
+  for (int i = 0; i < n; i++) {
+    DeviceGuard g(comms[i]->dev);
+    cudaFree(nullptr);
+    ap.location.id = comms[i]->dev;
+    CUmemGenericAllocationHandle phys = 0;
+    CUCHECK(comms[i], d.memCreate(&phys, size, &ap, 0));
+    CUCHECK(comms[i], d.mcBindMem(mc, 0, phys, 0, size, 0));
+    CUdeviceptr uc = 0;
+    CUCHECK(comms[i], d.addrReserve(&uc, size, g2, 0, 0));
+    CUCHECK(comms[i], d.memMap(uc, size, 0, phys, 0));
+    CUCHECK(comms[i], d.setAccess(uc, size, acc.data(), acc.size()));  // peers reach it too (unicast form)
+    if (i == 0) {
+      CUCHECK(comms[i], d.addrReserve(&mcva, size, g2, 0, 0));
+      CUCHECK(comms[i], d.memMap(mcva, size, 0, mc, 0));
+      CUCHECK(comms[i], d.setAccess(mcva, size, acc.data(), acc.size()));
+    }
+    mscclComm::Nvls nv{(char*)uc, nullptr, size, (unsigned long long)phys, (unsigned long long)mc, i == 0};
+    comms[i]->nvls.push_back(nv);
+    ptrs[i] = (void*)uc;
+  }
+  for (int i = 0; i < n; i++) comms[i]->nvls.back().mc = (char*)mcva;
+  return mscclSuccess;
+}
+
+mscclResult_t mscclNvlsFree(mscclComm_t* comms, int n, void** ptrs) {
+  if (!comms || n < 1 || !ptrs) return mscclInvalidArgument;
+  const Drv& d = drv();
+  for (int i = 0; i < n; i++) {
+    mscclComm* c = comms[i];
+    DeviceGuard g(c->dev);
+    CUDACHECK(c, cudaDeviceSynchronize());
+    auto it = std::find_if(c->nvls.begin(), c->nvls.end(), [&](const mscclComm::Nvls& x) { return x.uc == ptrs[i]; });
+    if (it == c->nvls.end()) return setErr(c, mscclInvalidArgument, "mscclNvlsFree: not an NVLS buffer of this rank");
+    d.memUnmap((CUdeviceptr)it->uc, it->size);
+    d.addrFree((CUdeviceptr)it->uc, it->size);
+    d.mcUnbind((CUmemGenericAllocationHandle)it->mcHandle, (CUdevice)c->dev, 0, it->size);
+    d.memRelease((CUmemGenericAllocationHandle)it->phys);
+    if (it->owner) {
+      d.memUnmap((CUdeviceptr)it->mc, it->size);
+      d.addrFree((CUdeviceptr)it->mc, it->size);
+      d.memRelease((CUmemGenericAllocationHandle)it->mcHandle);
+    }
+    c->nvls.erase(it);
+  }
+  return mscclSuccess;
+}
+
 mscclResult_t mscclCommGetStats(mscclComm_t c, int64_t* stats, int n) {
   if (!c || !stats || n < 1) return mscclInvalidArgument;
   DeviceGuard g(c->dev);
-  uint64_t dev[1] = {0};
+  uint64_t dev[2] = {0, 0};
   CUDACHECK(c, cudaMemcpy(dev, c->region + c->statsOff(), sizeof(dev), cudaMemcpyDeviceToHost));
-  const int64_t v[3] = {(int64_t)dev[0], (int64_t)c->launchesDirect1, (int64_t)c->launchesDirect2};
-  for (int i = 0; i < n && i < 3; i++) stats[i] = v[i];
+  const int64_t v[4] = {(int64_t)dev[0], (int64_t)c->launchesDirect1, (int64_t)c->launchesDirect2, (int64_t)dev[1]};
+  for (int i = 0; i < n && i < 4; i++) stats[i] = v[i];
   return mscclSuccess;
 }
 

@@ -58,6 +58,9 @@ SIGNATURES = {
     "mscclLaunchCount": (_c.c_uint64, []),
     "mscclCommGetStats": (_i, [_vp, _c.POINTER(_i64), _i]),
     "mscclCommRegister": (_i, [_vp, _vp, _sz, _c.POINTER(_vp)]),
+    "mscclNvlsSupported": (_i, [_i, _c.POINTER(_i)]),
+    "mscclNvlsAlloc": (_i, [_c.POINTER(_vp), _i, _sz, _c.POINTER(_vp)]),
+    "mscclNvlsFree": (_i, [_c.POINTER(_vp), _i, _c.POINTER(_vp)]),
     "mscclRegExport": (_i, [_vp, _vp]),
     "mscclRegConnect": (_i, [_vp, _vp]),
     "mscclCommDeregister": (_i, [_vp, _vp]),
@@ -115,6 +118,49 @@ def direct_placement(ir_text, rank):
     rdst = (_c.c_int32 * max(2, 2 * n.value))()
     _check(lib.mscclDebugDirectPlacement(b, len(b), rank, flags, rdst, n.value, _c.byref(n)))
     return [(flags[k], rdst[2 * k], rdst[2 * k + 1]) for k in range(n.value)]
+
+
+def nvls_supported(device):
+    """mscclNvlsSupported: NVSwitch multicast support of a device (bool)."""
+    v = _i()
+    _check(lib.mscclNvlsSupported(device, _c.byref(v)))
+    return bool(v.value)
+
+
+class _DeviceMemory:
+    """A raw device range exposed through __cuda_array_interface__ (zero-copy torch view)."""
+
+    def __init__(self, ptr, nbytes):
+        self.__cuda_array_interface__ = {"shape": (nbytes,), "typestr": "|u1", "data": (ptr, False),
+                                         "version": 3, "strides": None}
+
+
+def nvls_alloc(comms, nbytes):
+    """mscclNvlsAlloc over a full rank-ordered communicator set: one uint8 torch tensor per
+    rank (views of the multicast-bound memory; free with nvls_free)."""
+    import torch
+    n = len(comms)
+    arr = (_vp * n)(*[c.handle for c in comms])
+    ptrs = (_vp * n)()
+    _check(lib.mscclNvlsAlloc(arr, n, nbytes, ptrs), comms[0].handle)
+    out = []
+    for i, c in enumerate(comms):
+        with torch.cuda.device(_device_of(c)):
+            out.append(torch.as_tensor(_DeviceMemory(ptrs[i], nbytes), device="cuda"))
+    return out, [ptrs[i] for i in range(n)]
+
+
+def nvls_free(comms, ptrs):
+    n = len(comms)
+    arr = (_vp * n)(*[c.handle for c in comms])
+    p = (_vp * n)(*ptrs)
+    _check(lib.mscclNvlsFree(arr, n, p), comms[0].handle)
+
+
+def _device_of(comm):
+    v = _i()
+    _check(lib.mscclCommCuDevice(comm.handle, _c.byref(v)))
+    return v.value
 
 
 _TORCH_DT = None
@@ -254,10 +300,12 @@ class Comm:
         return v.value
 
     def stats(self):
-        """mscclCommGetStats: {"cross_direct_handshakes", "launches_direct1", "launches_direct2"}."""
-        v = (_i64 * 3)()
-        _check(lib.mscclCommGetStats(self.handle, v, 3), self.handle)
-        return {"cross_direct_handshakes": v[0], "launches_direct1": v[1], "launches_direct2": v[2]}
+        """mscclCommGetStats: {"cross_direct_handshakes", "launches_direct1", "launches_direct2",
+        "multicast_pieces"}."""
+        v = (_i64 * 4)()
+        _check(lib.mscclCommGetStats(self.handle, v, 4), self.handle)
+        return {"cross_direct_handshakes": v[0], "launches_direct1": v[1], "launches_direct2": v[2],
+                "multicast_pieces": v[3]}
 
     def last_error(self):
         return lib.mscclGetLastError(self.handle).decode(errors="replace")

@@ -70,3 +70,57 @@ def test_nvls_prod_rejected():
     with pytest.raises(runtime.MscclError) as ei:
         gpu_util.run_program(P.nvls_allreduce(R).to_xml(), xs, n, "float32", "prod")
     assert ei.value.code == 4
+
+
+def test_multicast_hardware_path():
+    """The hardware form of the multimem ops: NVLS buffers bound to an NVSwitch multicast
+    object (mscclNvlsAlloc) and multimem.ld_reduce / multimem.st on the multicast address.
+    Every visible GPU joins (one rank per GPU); on a one-GPU box the team has one member, so
+    the reduction is the identity, but the multicast object, its mappings and the multimem
+    instructions all run on the hardware. Outputs are checked against the oracle and the
+    device counter proves the multicast path executed."""
+    import torch
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    ndev = torch.cuda.device_count()
+    if not all(runtime.nvls_supported(d) for d in range(ndev)):
+        pytest.skip("CU_DEVICE_ATTRIBUTE_MULTICAST_SUPPORTED is 0 on this box")
+    R = ndev
+    comms = runtime.Comm.init_all(list(range(R)))
+    try:
+        n = 65536 * R
+        nbytes = 2 * n * 4 * 2   # in + out, fp32, headroom
+        bufs, ptrs = runtime.nvls_alloc(comms, nbytes)
+        try:
+            for dtype, tdt, build, out_mul in (("float32", torch.float32, P.nvls_allreduce, 1),
+                                               ("bfloat16", torch.bfloat16, P.nvls_allreduce, 1),
+                                               ("int32", torch.int32, P.nvls_allgather, R)):
+                w = torch.tensor([], dtype=tdt).element_size()
+                count = n // R if out_mul == R else n
+                xs = synth.inputs(R, count, dtype, "uniform" if dtype != "int32" else "pattern")
+                algo = build(R, 2)
+                want = sim.simulate(irparse.parse(algo.to_xml()), xs, count, dtype, "sum")
+                progs = [c.load(algo.to_xml()) for c in comms]
+                send, recv = [], []
+                for q in range(R):
+                    b = bufs[q]
+                    s = b[:count * w].view(tdt)
+                    r = b[count * w + 4096 - (count * w) % 4096:][:count * out_mul * w].view(tdt)
+                    s.copy_(torch.from_numpy(xs[q].view(np.uint8).copy()).cuda(q).view(tdt))
+                    send.append(s)
+                    recv.append(r)
+                before = [c.stats()["multicast_pieces"] for c in comms]
+                with runtime.group():
+                    for c, p_, s, r in zip(comms, progs, send, recv):
+                        c.run(p_, s, r, count)
+                torch.cuda.synchronize()
+                for q in range(R):
+                    got = recv[q].cpu().view(torch.uint8).numpy()
+                    assert np.array_equal(got, np.ascontiguousarray(want[q]).view(np.uint8)), (dtype, q)
+                    assert comms[q].stats()["multicast_pieces"] > before[q], dtype
+                for c, p_ in zip(comms, progs):
+                    c.unload(p_)
+        finally:
+            runtime.nvls_free(comms, ptrs)
+    finally:
+        for c in comms:
+            c.destroy()
