@@ -470,6 +470,7 @@ def extras(R, stream, nccl=None, S=256 * MIB):
     recv = [torch.empty_like(x) for x in send]
     for name, algo in (("floor_nop", None), ("one_hop_LL", "hop"), ("one_hop_LL128", "hop128"),
                        ("oneshot_LL", P.oneshot_allreduce(W, protocol="LL")),
+                       ("nvls_multimem", P.nvls_allreduce(W, 1)),
                        ("allpairs_LL", P.allpairs_allreduce(W, protocol="LL")),
                        ("ring_LL", P.ring_allreduce(W, protocol="LL")),
                        ("ring_ch%d_LL" % W, P.ring_allreduce(W, channels=W, protocol="LL"))):

@@ -1087,13 +1087,29 @@ mscclResult_t mscclNvlsAlloc(mscclComm_t* comms, int n, size_t bytes, void** ptr
   ap.location.id = c0->dev;
   CUCHECK(c0, d.memGran(&ugran, &ap, CU_MEM_ALLOC_GRANULARITY_RECOMMENDED));
   size_t g2 = std::max(gran, ugran);
-  const size_t size = (bytes + g2 - 1) / g2 * g2;
-  mp.size = size;
+  mp.size = (bytes + g2 - 1) / g2 * g2;
   CUmemGenericAllocationHandle mc = 0;
   {
     DeviceGuard g(c0->dev);
-    CUCHECK(c0, d.mcCreate(&mc, &mp));
+    // the handle type only matters for export; some drivers refuse 0, so try the POSIX fd
+    // type (the one NCCL uses for NVLS) first
+    CUresult e = CUDA_ERROR_INVALID_VALUE;
+    for (unsigned long long ht : {(unsigned long long)CU_MEM_HANDLE_TYPE_POSIX_FILE_DESCRIPTOR, 0ull,
+                                  (unsigned long long)CU_MEM_HANDLE_TYPE_FABRIC}) {
+      mp.handleTypes = ht;
+      size_t gr = 0;
+      if (d.mcGran(&gr, &mp, CU_MULTICAST_GRANULARITY_RECOMMENDED) != CUDA_SUCCESS) continue;
+      g2 = std::max(gr, ugran);
+      mp.size = (bytes + g2 - 1) / g2 * g2;
+      if ((e = d.mcCreate(&mc, &mp)) == CUDA_SUCCESS) break;
+    }
+    if (e != CUDA_SUCCESS) {
+      std::ostringstream o;
+      o << "cuMulticastCreate(numDevices=" << n << ", size=" << mp.size << ") failed with CUresult " << (int)e;
+      return setErr(c0, e == CUDA_ERROR_NOT_SUPPORTED ? mscclSystemError : mscclUnhandledCudaError, o.str());
+    }
   }
+  const size_t size = mp.size;
   for (int i = 0; i < n; i++) CUCHECK(comms[i], d.mcAddDevice(mc, (CUdevice)comms[i]->dev));
   // the multicast address, mapped once and accessible from every device
   CUdeviceptr mcva = 0;

@@ -89,7 +89,10 @@ def test_multicast_hardware_path():
     try:
         n = 65536 * R
         nbytes = 2 * n * 4 * 2   # in + out, fp32, headroom
-        bufs, ptrs = runtime.nvls_alloc(comms, nbytes)
+        try:
+            bufs, ptrs = runtime.nvls_alloc(comms, nbytes)
+        except runtime.MscclError as e:   # e.g. cuMulticastCreate refused (profiles/r02/mcprobe.txt)
+            pytest.skip("NVSwitch multicast object unavailable on this box: %s" % e)
         try:
             for dtype, tdt, build, out_mul in (("float32", torch.float32, P.nvls_allreduce, 1),
                                                ("bfloat16", torch.bfloat16, P.nvls_allreduce, 1),
