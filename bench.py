@@ -468,6 +468,7 @@ def extras(R, stream, nccl=None, S=256 * MIB):
     n = 512  # 1 KiB of fp16 per rank
     send = [synth.hashed(q, torch.arange(n, device=R.dev), "float16") for q in R.ranks]
     recv = [torch.empty_like(x) for x in send]
+    lat_regs = register_all(R, send + recv)   # N > 1: direct placement / multimem need them
     for name, algo in (("floor_nop", None), ("one_hop_LL", "hop"), ("one_hop_LL128", "hop128"),
                        ("oneshot_LL", P.oneshot_allreduce(W, protocol="LL")),
                        ("nvls_multimem", P.nvls_allreduce(W, 1)),
@@ -494,6 +495,8 @@ def extras(R, stream, nccl=None, S=256 * MIB):
                    "epilogue under graph replay; one_hop = rank r sends 1 KiB to rank r+1 (one message of the "
                    "protocol); the collective latencies are read against floor + hops")
     out["allreduce_1KiB_fp16_latency_us"] = lat
+    for r_ in lat_regs:
+        r_.deregister()
     del send, recv
     # AllToAll (direct two-step N=1), AllGather and ReduceScatter rings: S per rank (256 MiB), bf16
     n = S // 2

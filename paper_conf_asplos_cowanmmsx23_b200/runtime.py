@@ -180,10 +180,22 @@ def _dtype_name(t):
     return _TORCH_DT[t.dtype]
 
 
-def _stream(stream):
+_RAW_STREAM = None
+
+
+def _stream(stream, device=None):
+    """cudaStream_t of `stream`, or of the current stream of `device` (the per-call path:
+    torch's raw-stream query avoids building a Stream object on every call)."""
+    global _RAW_STREAM
     if stream is None:
-        import torch
-        stream = torch.cuda.current_stream()
+        if _RAW_STREAM is None:
+            import torch
+            _RAW_STREAM = getattr(torch._C, "_cuda_getCurrentRawStream", None) or \
+                (lambda d: torch.cuda.current_stream(d).cuda_stream)
+        if device is None:
+            import torch
+            device = torch.cuda.current_device()
+        return _RAW_STREAM(device)
     s = getattr(stream, "cuda_stream", None)
     return s if s is not None else int(stream)
 
@@ -246,6 +258,9 @@ class Comm:
     def __init__(self, handle):
         self.handle = _vp(handle) if not isinstance(handle, _vp) else handle
         self.programs = []
+        d = _i()
+        _check(lib.mscclCommCuDevice(self.handle, _c.byref(d)))
+        self.device = d.value
 
     # --- construction
     @staticmethod
@@ -338,24 +353,24 @@ class Comm:
     def allreduce(self, send, recv, op="sum", stream=None, count=None):
         n = send.numel() if count is None else count
         _check(lib.mscclAllReduce(_vp(send.data_ptr()), _vp(recv.data_ptr()), n, DTYPES[_dtype_name(send)],
-                                  OPS[op], self.handle, _stream(stream)), self.handle)
+                                  OPS[op], self.handle, _stream(stream, self.device)), self.handle)
 
     def allgather(self, send, recv, stream=None):
         _check(lib.mscclAllGather(_vp(send.data_ptr()), _vp(recv.data_ptr()), send.numel(),
-                                  DTYPES[_dtype_name(send)], self.handle, _stream(stream)), self.handle)
+                                  DTYPES[_dtype_name(send)], self.handle, _stream(stream, self.device)), self.handle)
 
     def reducescatter(self, send, recv, op="sum", stream=None):
         _check(lib.mscclReduceScatter(_vp(send.data_ptr()), _vp(recv.data_ptr()), recv.numel(),
-                                      DTYPES[_dtype_name(send)], OPS[op], self.handle, _stream(stream)), self.handle)
+                                      DTYPES[_dtype_name(send)], OPS[op], self.handle, _stream(stream, self.device)), self.handle)
 
     def alltoall(self, send, recv, stream=None):
         n = send.numel() // self.nranks
         _check(lib.mscclAllToAll(_vp(send.data_ptr()), _vp(recv.data_ptr()), n, DTYPES[_dtype_name(send)],
-                                 self.handle, _stream(stream)), self.handle)
+                                 self.handle, _stream(stream, self.device)), self.handle)
 
     def run(self, prog, send, recv, count, op="sum", stream=None, dtype=None):
         dt = DTYPES[dtype or _dtype_name(send)]
         r = _run_program(prog.handle, send.data_ptr(), recv.data_ptr(), count, dt, OPS[op], self.handle,
-                         _stream(stream))
+                         _stream(stream, self.device))
         if r:
             _check(r, self.handle)
