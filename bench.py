@@ -587,10 +587,14 @@ def sweep(R, stream, path, max_mib, nccl=None):
     from paper_conf_asplos_cowanmmsx23_b200 import programs as P
     W = R.R
     f = open(path, "w") if path else None
-    impl_sets = {"allreduce": P.tuned_allreduce(W), "alltoall": P.tuned_alltoall(W)}
+    impl_sets = {"allreduce": P.tuned_allreduce(W), "allreduce_multimem": P.tuned_allreduce_multimem(W),
+                 "alltoall": P.tuned_alltoall(W)}
     lines = []
-    for coll in ("allreduce", "alltoall"):
-        sets = [(algo, lo, hi, R.load(algo, lo, hi)) for algo, lo, hi in impl_sets[coll]]
+    for label in ("allreduce", "allreduce_multimem", "alltoall"):
+        coll = "allreduce" if label.startswith("allreduce") else label
+        if label == "allreduce_multimem" and nccl is not None:
+            pass  # NCCL runs once per collective, with the first AllReduce set
+        sets = [(algo, lo, hi, R.load(algo, lo, hi)) for algo, lo, hi in impl_sets[label]]
         size = 1024
         while size <= max_mib * MIB:
             n = size // 2
@@ -600,7 +604,7 @@ def sweep(R, stream, path, max_mib, nccl=None):
             per = (n // W) * 2 if coll == "alltoall" else size   # selection bytes (count * w)
             chosen = next(a for a, lo, hi, _ in sets if lo <= per and (hi == 0 or per < hi))
             impls = [("msccl", lambda: R.coll(coll, send, recv))]
-            if nccl is not None:
+            if nccl is not None and label != "allreduce_multimem":
                 impls.append(("nccl", (lambda: nccl.allreduce(send[0], recv[0], "bfloat16", stream=cur()))
                               if coll == "allreduce" else
                               (lambda: nccl.alltoall(send[0], recv[0], "bfloat16", W, cur()))))
@@ -608,7 +612,7 @@ def sweep(R, stream, path, max_mib, nccl=None):
                 for graph in (False, True):
                     iters = 50 if size <= 256 * MIB else 20
                     t, mode = timed(fn, iters, 20, stream, graph, R)
-                    rec = {"impl": impl, "coll": coll, "program": chosen.name if impl == "msccl" else "nccl",
+                    rec = {"impl": impl, "coll": coll, "set": label, "program": chosen.name if impl == "msccl" else "nccl",
                            "R": W, "dtype": "bf16", "op": "sum", "bytes": size, "count": n,
                            "iters": iters, "warmup": 20, "graph": mode == "cuda-graph", "t_us_max": round(t * 1e6, 3),
                            "algbw": round(size / t / 1e9, 3), "busbw": round(busbw(coll, size, t, W), 3)}
