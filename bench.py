@@ -394,6 +394,15 @@ class Ranks:
         dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         return float(tt.item())
 
+    def per_rank(self, t):
+        """every rank's own time (rank order), via the plumbing group."""
+        if self.world == 1:
+            return [t]
+        import torch.distributed as dist
+        out = [None] * self.world
+        dist.all_gather_object(out, t)
+        return out
+
     def all_ok(self, ok):
         if self.world == 1:
             return bool(ok)
@@ -417,7 +426,7 @@ def cur():
     return torch.cuda.current_stream().cuda_stream
 
 
-def timed(fn, iters, warmup, stream, graph, R):
+def timed(fn, iters, warmup, stream, graph, R, local=None):
     """Mean device time per call of fn() (CUDA events on `stream`, synchronised on both
     sides, max over ranks). fn() must issue its work on the current stream. graph=True
     captures `iters` calls into one CUDA graph and times its replay. Returns (seconds, mode)."""
@@ -451,7 +460,10 @@ def timed(fn, iters, warmup, stream, graph, R):
     run()
     e1.record(stream)
     torch.cuda.synchronize()
-    return R.tmax(e0.elapsed_time(e1) / 1e3 / iters), mode
+    t = e0.elapsed_time(e1) / 1e3 / iters
+    if local is not None:
+        local[0] = t
+    return R.tmax(t), mode
 
 
 # ----------------------------------------------------------------------------- extras
@@ -611,11 +623,20 @@ def sweep(R, stream, path, max_mib, nccl=None):
             for impl, fn in impls:
                 for graph in (False, True):
                     iters = 50 if size <= 256 * MIB else 20
-                    t, mode = timed(fn, iters, 20, stream, graph, R)
+                    t_local = [0.0]
+                    t, mode = timed(fn, iters, 20, stream, graph, R, t_local)
                     rec = {"impl": impl, "coll": coll, "set": label, "program": chosen.name if impl == "msccl" else "nccl",
                            "R": W, "dtype": "bf16", "op": "sum", "bytes": size, "count": n,
                            "iters": iters, "warmup": 20, "graph": mode == "cuda-graph", "t_us_max": round(t * 1e6, 3),
+                           "t_us_per_rank": [round(x * 1e6, 3) for x in R.per_rank(t_local[0])],
                            "algbw": round(size / t / 1e9, 3), "busbw": round(busbw(coll, size, t, W), 3)}
+                    if impl == "msccl":
+                        rec.update({"proto": chosen.proto, "instances": chosen.ninstances,
+                                    "channels": chosen.nchannels, "ctas_per_rank": chosen.max_tbs(),
+                                    "slots": R.rt.get_param("MSCCL_SLOTS"),
+                                    "slot_bytes": R.rt.get_param({"LL": "MSCCL_LL_SLOT_BYTES",
+                                                                  "LL128": "MSCCL_LL128_SLOT_BYTES"}.get(
+                                                                      chosen.proto, "MSCCL_SLOT_BYTES"))})
                     if R.world > 1:
                         rec["frac_nvlink"] = round(rec["busbw"] / NVLINK_NOMINAL, 4)
                     if size <= 64 * 1024 and graph:
