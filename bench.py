@@ -730,7 +730,8 @@ def run_virtual(args):
     res = {"t": t, "coll": coll, "launches": launches, "clocks": clk, "parity_bad": bad, "parity_total": total,
            "algo": algo, "S": S, "R": W, "touches": touches, "direct": direct}
     if not args.no_e2e:
-        res["e2e"] = e2e(R, send, recv, lambda: step(), S, coll, W, args.steps, stream)
+        res["e2e"] = e2e(R, send, recv, lambda sn, rc, st: R.call(progs, sn, rc, count, st), S, coll, W,
+                         args.steps, stream)
     R.unload(progs)
     if not args.quiet_extra:
         del send, recv
@@ -741,37 +742,80 @@ def run_virtual(args):
     return res
 
 
-def e2e(R, send, recv, step, S, coll, W, steps, stream):
-    """The same metric end to end through the public API: every step copies the step's
+def e2e(R, send, recv, call, S, coll, W, steps, stream):
+    """The same metric end to end through the public API: every step copies that step's
     inputs from pinned host memory to the device, runs the collective, and reads the result
-    back (all local ranks); max over ranks."""
-    import torch
-    host_in = [s.cpu().pin_memory() for s in send]
-    host_out = [torch.empty(r.numel(), dtype=r.dtype).pin_memory() for r in recv]
-    k = max(2, min(5, steps))
+    back (every local rank); max over ranks.
 
-    def e2e_step():
-        for s, h in zip(send, host_in):
-            s.copy_(h, non_blocking=True)
-        step()
-        for r, h in zip(recv, host_out):
+    Steps are software-pipelined over two device buffer sets and three streams: the H2D of
+    step k+1 and the D2H of step k-1 overlap the collective of step k. Every step still pays
+    its own copies inside the timed region; only independent work overlaps. PCIe moves data
+    in both directions at once. `serial_ms` is the same loop with each step's three phases
+    run back to back on one stream."""
+    import torch
+    host_in = [s_.cpu().pin_memory() for s_ in send]
+    sets = [(send, recv), ([torch.empty_like(x) for x in send], [torch.empty_like(x) for x in recv])]
+    host_out = [[torch.empty(r.numel(), dtype=r.dtype).pin_memory() for r in recv] for _ in range(2)]
+    k = max(4, min(8, steps))
+    s_in, s_out = torch.cuda.Stream(), torch.cuda.Stream()
+    ev = lambda: torch.cuda.Event()
+    h2d_done = [ev(), ev()]
+    coll_done = [ev(), ev()]
+    d2h_done = [ev(), ev()]
+
+    def pipelined_step(i):
+        b = i % 2
+        snd, rcv = sets[b]
+        with torch.cuda.stream(s_in):
+            s_in.wait_event(coll_done[b])        # step i-2 has finished reading snd
+            for d, h in zip(snd, host_in):
+                d.copy_(h, non_blocking=True)
+            h2d_done[b].record(s_in)
+        stream.wait_event(h2d_done[b])
+        stream.wait_event(d2h_done[b])           # step i-2's result has left rcv
+        call(snd, rcv, stream)
+        coll_done[b].record(stream)
+        with torch.cuda.stream(s_out):
+            s_out.wait_event(coll_done[b])
+            for r, h in zip(rcv, host_out[b]):
+                h.copy_(r, non_blocking=True)
+            d2h_done[b].record(s_out)
+
+    def serial_step():
+        for d, h in zip(send, host_in):
+            d.copy_(h, non_blocking=True)
+        call(send, recv, stream)
+        for r, h in zip(recv, host_out[0]):
             h.copy_(r, non_blocking=True)
 
-    e2e_step()
+    for i in range(2):
+        pipelined_step(i)
     torch.cuda.synchronize()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     R.barrier()
+    torch.cuda.synchronize()
     e0.record(stream)
-    for _ in range(k):
-        e2e_step()
+    for i in range(k):
+        pipelined_step(i)
+    stream.wait_stream(s_out)
     e1.record(stream)
     torch.cuda.synchronize()
     te = R.tmax(e0.elapsed_time(e1) / 1e3 / k)
-    nl = len(send)
+    serial_step()
+    torch.cuda.synchronize()
+    e0.record(stream)
+    for _ in range(2):
+        serial_step()
+    e1.record(stream)
+    torch.cuda.synchronize()
+    ts = R.tmax(e0.elapsed_time(e1) / 1e3 / 2)
+    h2d = sum(x.numel() * x.element_size() for x in send)
+    d2h = sum(x.numel() * x.element_size() for x in recv)
     return {"value": round(busbw(coll, S, te, W), 3), "unit": "GB/s",
-            "h2d_bytes_per_step": S * nl, "d2h_bytes_per_step": S * nl, "ms_per_step": round(te * 1e3, 3),
+            "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h, "ms_per_step": round(te * 1e3, 3),
+            "serial_ms_per_step": round(ts * 1e3, 3),
             "note": "C-ABI call with pinned host buffers: H2D of this process's %d rank input(s) + collective + "
-                    "D2H of the output(s) per step (PCIe-bound)" % nl}
+                    "D2H of the output(s) every step, pipelined over 2 buffer sets (PCIe-bound)" % len(send)}
 
 
 # ----------------------------------------------------------------------------- N > 1
@@ -899,7 +943,8 @@ def run_multi(args, rank, world, local_rank):
         res["nccl"] = {"value": round(busbw(coll, S, tn, world), 3), "ms_per_step": round(tn * 1e3, 4),
                        "note": nccl_note}
     if not args.no_e2e:
-        res["e2e"] = e2e(R, send, recv, step, S, coll, world, args.steps, stream)
+        res["e2e"] = e2e(R, send, recv, lambda sn, rc, st: R.call(progs, sn, rc, count, st), S, coll, world,
+                         args.steps, stream)
     for r_ in regs:
         r_.deregister()
     R.unload(progs)

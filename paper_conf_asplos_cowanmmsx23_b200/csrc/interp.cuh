@@ -913,11 +913,13 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
 // (peer memory over NVLink, or the same HBM for virtual ranks), folded in ascending rank order
 // with fp32 accumulation and one rounding for fp16 / bf16 sums (what the switch's .acc::f32
 // reduction computes), and one store per rank.
-template <int DT, int OP>
-struct MMAcc {  // fold of R 32-byte vectors in ascending rank order
+template <int DT, int OP, int VB>
+struct MMAcc {  // fold of R VB-byte vectors in ascending rank order
+  typedef typename VecT<VB>::T Vec;
   static constexpr bool kHalfSum = (DT == DT_BF16 || DT == DT_F16) && OP == R_SUM;
-  float f[16];
-  V32 v;
+  static constexpr int NH = VB / 2;
+  float f[NH];
+  Vec v;
   static __device__ __forceinline__ float widen(uint16_t x) {
     if constexpr (DT == DT_BF16) return __uint_as_float(((uint32_t)x) << 16);
     else return __half2float(__ushort_as_half(x));
@@ -926,30 +928,30 @@ struct MMAcc {  // fold of R 32-byte vectors in ascending rank order
     if constexpr (DT == DT_BF16) return __bfloat16_as_ushort(__float2bfloat16_rn(x));
     else return __half_as_ushort(__float2half_rn(x));
   }
-  __device__ __forceinline__ void first(const V32& x) {
+  __device__ __forceinline__ void first(const Vec& x) {
     if constexpr (kHalfSum) {
       const uint16_t* h = reinterpret_cast<const uint16_t*>(&x);
 #pragma unroll
-      for (int k = 0; k < 16; k++) f[k] = widen(h[k]);
+      for (int k = 0; k < NH; k++) f[k] = widen(h[k]);
     } else {
       v = x;
     }
   }
-  __device__ __forceinline__ void add(const V32& x) {
+  __device__ __forceinline__ void add(const Vec& x) {
     if constexpr (kHalfSum) {
       const uint16_t* h = reinterpret_cast<const uint16_t*>(&x);
 #pragma unroll
-      for (int k = 0; k < 16; k++) f[k] = f[k] + widen(h[k]);
+      for (int k = 0; k < NH; k++) f[k] = f[k] + widen(h[k]);
     } else {
       v = vop<DT, OP>(v, x);
     }
   }
-  __device__ __forceinline__ V32 result() const {
+  __device__ __forceinline__ Vec result() const {
     if constexpr (kHalfSum) {
-      V32 r;
+      Vec r;
       uint16_t* h = reinterpret_cast<uint16_t*>(&r);
 #pragma unroll
-      for (int k = 0; k < 16; k++) h[k] = narrow(f[k]);
+      for (int k = 0; k < NH; k++) h[k] = narrow(f[k]);
       return r;
     } else {
       return v;
@@ -1011,16 +1013,53 @@ __device__ __forceinline__ bool multicastPiece(const Ctx& c, const DevInstr& in,
   return true;
 }
 
+// nv VB-byte vectors of one multimem piece starting at byte `off`; returns nv
+template <int DT, int OP, int KIND, int VB>
+__device__ __forceinline__ int64_t mmVecLoop(const Ctx& c, const DevInstr& in, int64_t so, int64_t dof, int64_t nv,
+                                             int64_t off) {
+  typedef typename VecT<VB>::T Vec;
+  constexpr bool RALL = KIND != K_MST, WALL = KIND != K_MRD;
+  constexpr int B = MSCCL_MM_BATCH;
+  const RankArgs& ra = *c.ra;
+  const int R = ra.nRanks, me = ra.myRank;
+  const uint64_t pol = policyEvictFirst();
+  so += off;
+  dof += off;
+  for (int64_t i = c.tid; i < nv; i += c.nt) {
+    MMAcc<DT, OP, VB> acc;
+    if constexpr (RALL) {  // B ranks' loads in flight, folded in ascending rank order
+      for (int p0 = 0; p0 < R; p0 += B) {
+        Vec x[B];
+#pragma unroll
+        for (int u = 0; u < B; u++)
+          if (p0 + u < R) ldStream(x[u], c.mmBuf[p0 + u][in.srcBuf] + so + i * VB, pol);
+#pragma unroll
+        for (int u = 0; u < B; u++) {
+          if (p0 + u >= R) break;
+          if (p0 + u == 0) acc.first(x[u]);
+          else acc.add(x[u]);
+        }
+      }
+    } else {
+      Vec x;
+      ldStream(x, c.mmBuf[me][in.srcBuf] + so + i * VB, pol);
+      acc.first(x);
+    }
+    const Vec v = acc.result();
+    for (int p = 0; p < R; p++)
+      if (WALL || p == me) stHint(c.mmBuf[p][in.dstBuf] + dof + i * VB, v, pol);
+  }
+  return nv;
+}
+
 template <int DT, int OP, int KIND>
 __device__ __noinline__ void runMultimem(const Ctx& c, const DevInstr& in, int t) {
   typedef typename DType<DT>::T T;
   const KernelArgs& a = *c.a;
   const RankArgs& ra = *c.ra;
   constexpr bool RALL = KIND != K_MST, WALL = KIND != K_MRD;
-  constexpr int B = MSCCL_MM_BATCH;
   const int R = ra.nRanks, me = ra.myRank;
   const int64_t w = sizeof(T), a0 = (int64_t)t * a.T;
-  const uint64_t pol = policyEvictFirst();
   for (int j = 0; j < in.cnt; j++) {
     int64_t ss, sl, ds, dl;
     chunkSpan(a, in.srcBuf, (int64_t)in.srcOff + j, ss, sl);
@@ -1032,38 +1071,18 @@ __device__ __noinline__ void runMultimem(const Ctx& c, const DevInstr& in, int t
     if (multicastPiece<DT, OP, KIND>(c, in, so, dof, m)) continue;
     uintptr_t al = (uintptr_t)so | (uintptr_t)dof;
     for (int p = 0; p < R; p++) al |= (uintptr_t)c.mmBuf[p][in.srcBuf] | (uintptr_t)c.mmBuf[p][in.dstBuf];
-    const int64_t nvec = (al & 31) ? 0 : m * w / 32;
-    for (int64_t i = c.tid; i < nvec; i += c.nt) {
-      MMAcc<DT, OP> acc;
-      if constexpr (RALL) {  // B ranks' 256-bit loads in flight, folded in ascending rank order
-        for (int p0 = 0; p0 < R; p0 += B) {
-          V32 x[B];
-#pragma unroll
-          for (int u = 0; u < B; u++)
-            if (p0 + u < R) ldStream(x[u], c.mmBuf[p0 + u][in.srcBuf] + so + i * 32, pol);
-#pragma unroll
-          for (int u = 0; u < B; u++) {
-            if (p0 + u >= R) break;
-            if (p0 + u == 0) acc.first(x[u]);
-            else acc.add(x[u]);
-          }
-        }
-      } else {
-        V32 x;
-        ldStream(x, c.mmBuf[me][in.srcBuf] + so + i * 32, pol);
-        acc.first(x);
-      }
-      const V32 v = acc.result();
-      for (int p = 0; p < R; p++)
-        if (WALL || p == me) stHint(c.mmBuf[p][in.dstBuf] + dof + i * 32, v, pol);
-    }
-    for (int64_t e = nvec * 32 / w + c.tid; e < m; e += c.nt) {  // scalar tail (ragged or unaligned)
+    // 32-byte vectors when every rank's span is 32-byte aligned, else 16-byte (chunk starts are
+    // multiples of 16 bytes, reading R1), then a scalar tail
+    int64_t done = 0;
+    if ((al & 31) == 0) done = 32 * mmVecLoop<DT, OP, KIND, 32>(c, in, so, dof, m * w / 32, 0);
+    if ((al & 15) == 0) done += 16 * mmVecLoop<DT, OP, KIND, 16>(c, in, so, dof, (m * w - done) / 16, done);
+    for (int64_t e = done / w + c.tid; e < m; e += c.nt) {  // scalar tail (ragged or unaligned)
       T v;
       if constexpr (RALL) {
-        if constexpr (MMAcc<DT, OP>::kHalfSum) {
-          float f = MMAcc<DT, OP>::widen(*(const T*)(c.mmBuf[0][in.srcBuf] + so + e * w));
-          for (int p = 1; p < R; p++) f = f + MMAcc<DT, OP>::widen(*(const T*)(c.mmBuf[p][in.srcBuf] + so + e * w));
-          v = MMAcc<DT, OP>::narrow(f);
+        if constexpr (MMAcc<DT, OP, 16>::kHalfSum) {
+          float f = MMAcc<DT, OP, 16>::widen(*(const T*)(c.mmBuf[0][in.srcBuf] + so + e * w));
+          for (int p = 1; p < R; p++) f = f + MMAcc<DT, OP, 16>::widen(*(const T*)(c.mmBuf[p][in.srcBuf] + so + e * w));
+          v = MMAcc<DT, OP, 16>::narrow(f);
         } else {
           v = *(const T*)(c.mmBuf[0][in.srcBuf] + so + e * w);
           for (int p = 1; p < R; p++) v = DType<DT>::op(OP, v, *(const T*)(c.mmBuf[p][in.srcBuf] + so + e * w));

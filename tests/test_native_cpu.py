@@ -136,3 +136,17 @@ def test_cpp_v11_multimem_rules(rt):
     for text in (ll, sc):
         with pytest.raises(pv.ValidationError, match="^V11"):
             pv.validate(irparse.parse(text), nranks=4)
+
+
+def test_bench_probe_programs_are_valid(rt):
+    """bench.py's latency probes (the empty program and the one-hop program) pass both
+    validators and the race check."""
+    import bench
+    from oracle import races
+    for R in (2, 8):
+        for text in (bench.nop_ir(R), bench.hop_ir(R), bench.hop_ir(R, "LL128")):
+            ok, msg = rt.validate(text, R)
+            assert ok, msg
+            al = irparse.parse(text)
+            pyval.validate(al, nranks=R, races=True)
+            assert races.find_races(al) == []
