@@ -109,6 +109,8 @@ struct KernelArgs {
   // from the launch arguments, no barrier); 2 cross-launch (group barrier lines publish the
   // ranks' buffer references at the start and completion at the end)
   int32_t mm;
+  int32_t mmVec32;            // multimem: every chunk / tile span is 32-byte aligned (32-byte vectors)
+  int32_t pad1;
   int64_t mmLineOff;          // offset of the group-barrier lines in every region
   uint64_t timeoutNs;         // device watchdog; 0 = disabled
   uint64_t* trace;            // MSCCL_TRACE builds: per-CTA phase times (ns), else null

@@ -1013,53 +1013,18 @@ __device__ __forceinline__ bool multicastPiece(const Ctx& c, const DevInstr& in,
   return true;
 }
 
-// nv VB-byte vectors of one multimem piece starting at byte `off`; returns nv
+// VB = 32 when every span of the launch is 32-byte aligned (host: KernelArgs::mmVec32), else 16
 template <int DT, int OP, int KIND, int VB>
-__device__ __forceinline__ int64_t mmVecLoop(const Ctx& c, const DevInstr& in, int64_t so, int64_t dof, int64_t nv,
-                                             int64_t off) {
-  typedef typename VecT<VB>::T Vec;
-  constexpr bool RALL = KIND != K_MST, WALL = KIND != K_MRD;
-  constexpr int B = MSCCL_MM_BATCH;
-  const RankArgs& ra = *c.ra;
-  const int R = ra.nRanks, me = ra.myRank;
-  const uint64_t pol = policyEvictFirst();
-  so += off;
-  dof += off;
-  for (int64_t i = c.tid; i < nv; i += c.nt) {
-    MMAcc<DT, OP, VB> acc;
-    if constexpr (RALL) {  // B ranks' loads in flight, folded in ascending rank order
-      for (int p0 = 0; p0 < R; p0 += B) {
-        Vec x[B];
-#pragma unroll
-        for (int u = 0; u < B; u++)
-          if (p0 + u < R) ldStream(x[u], c.mmBuf[p0 + u][in.srcBuf] + so + i * VB, pol);
-#pragma unroll
-        for (int u = 0; u < B; u++) {
-          if (p0 + u >= R) break;
-          if (p0 + u == 0) acc.first(x[u]);
-          else acc.add(x[u]);
-        }
-      }
-    } else {
-      Vec x;
-      ldStream(x, c.mmBuf[me][in.srcBuf] + so + i * VB, pol);
-      acc.first(x);
-    }
-    const Vec v = acc.result();
-    for (int p = 0; p < R; p++)
-      if (WALL || p == me) stHint(c.mmBuf[p][in.dstBuf] + dof + i * VB, v, pol);
-  }
-  return nv;
-}
-
-template <int DT, int OP, int KIND>
 __device__ __noinline__ void runMultimem(const Ctx& c, const DevInstr& in, int t) {
   typedef typename DType<DT>::T T;
+  typedef typename VecT<VB>::T Vec;
   const KernelArgs& a = *c.a;
   const RankArgs& ra = *c.ra;
   constexpr bool RALL = KIND != K_MST, WALL = KIND != K_MRD;
+  constexpr int B = MSCCL_MM_BATCH;
   const int R = ra.nRanks, me = ra.myRank;
   const int64_t w = sizeof(T), a0 = (int64_t)t * a.T;
+  const uint64_t pol = policyEvictFirst();
   for (int j = 0; j < in.cnt; j++) {
     int64_t ss, sl, ds, dl;
     chunkSpan(a, in.srcBuf, (int64_t)in.srcOff + j, ss, sl);
@@ -1071,18 +1036,38 @@ __device__ __noinline__ void runMultimem(const Ctx& c, const DevInstr& in, int t
     if (multicastPiece<DT, OP, KIND>(c, in, so, dof, m)) continue;
     uintptr_t al = (uintptr_t)so | (uintptr_t)dof;
     for (int p = 0; p < R; p++) al |= (uintptr_t)c.mmBuf[p][in.srcBuf] | (uintptr_t)c.mmBuf[p][in.dstBuf];
-    // 32-byte vectors when every rank's span is 32-byte aligned, else 16-byte (chunk starts are
-    // multiples of 16 bytes, reading R1), then a scalar tail
-    int64_t done = 0;
-    if ((al & 31) == 0) done = 32 * mmVecLoop<DT, OP, KIND, 32>(c, in, so, dof, m * w / 32, 0);
-    if ((al & 15) == 0) done += 16 * mmVecLoop<DT, OP, KIND, 16>(c, in, so, dof, (m * w - done) / 16, done);
-    for (int64_t e = done / w + c.tid; e < m; e += c.nt) {  // scalar tail (ragged or unaligned)
+    const int64_t nvec = (al & (VB - 1)) ? 0 : m * w / VB;
+    for (int64_t i = c.tid; i < nvec; i += c.nt) {
+      MMAcc<DT, OP, VB> acc;
+      if constexpr (RALL) {  // B ranks' loads in flight, folded in ascending rank order
+        for (int p0 = 0; p0 < R; p0 += B) {
+          Vec x[B];
+#pragma unroll
+          for (int u = 0; u < B; u++)
+            if (p0 + u < R) ldStream(x[u], c.mmBuf[p0 + u][in.srcBuf] + so + i * VB, pol);
+#pragma unroll
+          for (int u = 0; u < B; u++) {
+            if (p0 + u >= R) break;
+            if (p0 + u == 0) acc.first(x[u]);
+            else acc.add(x[u]);
+          }
+        }
+      } else {
+        Vec x;
+        ldStream(x, c.mmBuf[me][in.srcBuf] + so + i * VB, pol);
+        acc.first(x);
+      }
+      const Vec v = acc.result();
+      for (int p = 0; p < R; p++)
+        if (WALL || p == me) stHint(c.mmBuf[p][in.dstBuf] + dof + i * VB, v, pol);
+    }
+    for (int64_t e = nvec * VB / w + c.tid; e < m; e += c.nt) {  // scalar tail (ragged or unaligned)
       T v;
       if constexpr (RALL) {
-        if constexpr (MMAcc<DT, OP, 16>::kHalfSum) {
-          float f = MMAcc<DT, OP, 16>::widen(*(const T*)(c.mmBuf[0][in.srcBuf] + so + e * w));
-          for (int p = 1; p < R; p++) f = f + MMAcc<DT, OP, 16>::widen(*(const T*)(c.mmBuf[p][in.srcBuf] + so + e * w));
-          v = MMAcc<DT, OP, 16>::narrow(f);
+        if constexpr (MMAcc<DT, OP, VB>::kHalfSum) {
+          float f = MMAcc<DT, OP, VB>::widen(*(const T*)(c.mmBuf[0][in.srcBuf] + so + e * w));
+          for (int p = 1; p < R; p++) f = f + MMAcc<DT, OP, VB>::widen(*(const T*)(c.mmBuf[p][in.srcBuf] + so + e * w));
+          v = MMAcc<DT, OP, VB>::narrow(f);
         } else {
           v = *(const T*)(c.mmBuf[0][in.srcBuf] + so + e * w);
           for (int p = 1; p < R; p++) v = DType<DT>::op(OP, v, *(const T*)(c.mmBuf[p][in.srcBuf] + so + e * w));
@@ -1169,13 +1154,18 @@ static __device__ __noinline__ bool mmBarrier(const Ctx& c, const DevTB& tb, uin
   return __syncthreads_and(ok) != 0;
 }
 
+template <int DT, int OP, int VB>
+__device__ __forceinline__ void multimemOpV(const Ctx& c, const DevInstr& in, int t) {
+  if (in.op == K_MST) runMultimem<DT, OP, K_MST, VB>(c, in, t);
+  if constexpr (OP != R_COPY) {
+    if (in.op == K_MRD) runMultimem<DT, OP, K_MRD, VB>(c, in, t);
+    if (in.op == K_MRS) runMultimem<DT, OP, K_MRS, VB>(c, in, t);
+  }
+}
 template <int DT, int OP>
 __device__ __noinline__ void multimemOp(const Ctx& c, const DevInstr& in, int t) {
-  if (in.op == K_MST) runMultimem<DT, OP, K_MST>(c, in, t);
-  if constexpr (OP != R_COPY) {
-    if (in.op == K_MRD) runMultimem<DT, OP, K_MRD>(c, in, t);
-    if (in.op == K_MRS) runMultimem<DT, OP, K_MRS>(c, in, t);
-  }
+  if (c.a->mmVec32) multimemOpV<DT, OP, 32>(c, in, t);  // every span 32-byte aligned (host decides)
+  else multimemOpV<DT, OP, 16>(c, in, t);
 }
 
 // MM: the kernel variant for programs with multimem ops (reading R23). Their code lives only

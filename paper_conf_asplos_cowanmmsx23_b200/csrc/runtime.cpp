@@ -487,6 +487,13 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
     ka.directHints = (int32_t)c0->prm.directHints;
     ka.mm = mm;
     ka.mmLineOff = (int64_t)c0->mmLineOff();
+    {  // multimem vector width: chunk starts (E*w) and tile offsets (T*w) 32-byte aligned
+      const int64_t w = elemBytes(v[0]->dtype);
+      bool a32 = (g.E * w) % 32 == 0 && (g.T * w) % 32 == 0 && ((uint64_t)g.n * w) % 32 == 0;
+      for (auto* cl : v)
+        a32 = a32 && ((uintptr_t)cl->buf[0] % 32 == 0) && ((uintptr_t)cl->buf[1] % 32 == 0);
+      ka.mmVec32 = a32 ? 1 : 0;
+    }
     int cta = 0;
     for (int i = 0; i < (int)v.size(); i++) {
       Call* cl = v[i];
