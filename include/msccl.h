@@ -98,7 +98,8 @@ mscclResult_t mscclCommCount(const mscclComm_t comm, int* count);
  *     destination and stored directly into a peer (device-side count, reading R15b);
  * [1] launches with one-launch direct placement (every rank in the launch, reading R15);
  * [2] launches in which this rank published a reachable destination (cross-launch mode);
- * [3] multimem pieces executed through an NVSwitch multicast address (device-side count). */
+ * [3] multimem pieces executed through an NVSwitch multicast address (device-side count);
+ * [4] V9 re-checks run at a launch's real pipeline depth (one per program and depth I > 2). */
 mscclResult_t mscclCommGetStats(mscclComm_t comm, int64_t* stats, int n);
 mscclResult_t mscclCommUserRank(const mscclComm_t comm, int* rank);
 mscclResult_t mscclCommCuDevice(const mscclComm_t comm, int* device);

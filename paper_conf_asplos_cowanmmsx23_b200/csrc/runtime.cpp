@@ -119,6 +119,7 @@ struct mscclComm {
   std::string lastError;
   int maxCoResident = 0;
   uint64_t launchesDirect1 = 0, launchesDirect2 = 0;  // launches this rank took part in, by direct mode
+  uint64_t depthChecks = 0;            // V9 re-runs at a launch's real pipeline depth (R24)
   uint32_t loadCounter = 0;            // programs loaded so far (multimem group-barrier epochs)
   // NVLS buffers (mscclNvlsAlloc): this rank's unicast range and the multicast address of it
   struct Nvls {
@@ -401,6 +402,7 @@ mscclResult_t checkDepth(mscclComm* c, mscclProgram* p, int I) {
     return setErr(c, mscclInvalidProgram, std::string(e.what()) + " (pipeline depth I=" + std::to_string(I) + ")");
   }
   p->v9Iters.insert(I);
+  c->depthChecks++;
   return mscclSuccess;
 }
 
@@ -1178,8 +1180,9 @@ mscclResult_t mscclCommGetStats(mscclComm_t c, int64_t* stats, int n) {
   DeviceGuard g(c->dev);
   uint64_t dev[2] = {0, 0};
   CUDACHECK(c, cudaMemcpy(dev, c->region + c->statsOff(), sizeof(dev), cudaMemcpyDeviceToHost));
-  const int64_t v[4] = {(int64_t)dev[0], (int64_t)c->launchesDirect1, (int64_t)c->launchesDirect2, (int64_t)dev[1]};
-  for (int i = 0; i < n && i < 4; i++) stats[i] = v[i];
+  const int64_t v[5] = {(int64_t)dev[0], (int64_t)c->launchesDirect1, (int64_t)c->launchesDirect2, (int64_t)dev[1],
+                        (int64_t)c->depthChecks};
+  for (int i = 0; i < n && i < 5; i++) stats[i] = v[i];
   return mscclSuccess;
 }
 

@@ -316,11 +316,11 @@ class Comm:
 
     def stats(self):
         """mscclCommGetStats: {"cross_direct_handshakes", "launches_direct1", "launches_direct2",
-        "multicast_pieces"}."""
-        v = (_i64 * 4)()
-        _check(lib.mscclCommGetStats(self.handle, v, 4), self.handle)
+        "multicast_pieces", "depth_checks"}."""
+        v = (_i64 * 5)()
+        _check(lib.mscclCommGetStats(self.handle, v, 5), self.handle)
         return {"cross_direct_handshakes": v[0], "launches_direct1": v[1], "launches_direct2": v[2],
-                "multicast_pieces": v[3]}
+                "multicast_pieces": v[3], "depth_checks": v[4]}
 
     def last_error(self):
         return lib.mscclGetLastError(self.handle).decode(errors="replace")

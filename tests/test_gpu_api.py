@@ -246,3 +246,34 @@ def test_aliassafe_inplace_call_disables_direct_placement(env):
     finally:
         for c, p in zip(comms, ps):
             c.unload(p)
+
+
+def test_v9_rechecked_once_per_pipeline_depth(env):
+    """Reading R24: the loader verified deadlock freedom over 2
+    pipeline iterations; the first launch with a deeper pipeline re-runs V9 at its real depth
+    I, once per (program, I) -- a second call of the same size is not re-checked, a larger
+    size is. One-launch direct placement counts too (mscclCommGetStats)."""
+    torch, runtime, comms = env
+    algo = P.ring_allreduce(R, instances=2)
+    ps = [c.load(algo.to_xml()) for c in comms]
+    try:
+        slot = runtime.get_param("MSCCL_SLOT_BYTES")
+        def run(n):
+            x = [torch.ones(n, device="cuda") for _ in comms]
+            y = [torch.empty_like(t) for t in x]
+            _call(runtime, comms, lambda q, c: c.allreduce(x[q], y[q]))
+            torch.cuda.synchronize()
+            assert all(bool((t == R).all()) for t in y)
+        s0 = comms[0].stats()
+        n1 = (slot // 4) * R * 2 * 3          # 3 tiles per chunk (fp32)
+        run(n1)
+        s1 = comms[0].stats()
+        assert s1["depth_checks"] == s0["depth_checks"] + 1
+        assert s1["launches_direct1"] == s0["launches_direct1"] + 1
+        run(n1)
+        assert comms[0].stats()["depth_checks"] == s1["depth_checks"]
+        run(n1 * 2)
+        assert comms[0].stats()["depth_checks"] == s1["depth_checks"] + 1
+    finally:
+        for c, p_ in zip(comms, ps):
+            c.unload(p_)
