@@ -87,3 +87,55 @@ def test_inconsistent_handles_rejected(monkeypatch):
     monkeypatch.setitem(sys.modules, "torch.distributed", D)
     with pytest.raises(RuntimeError):
         mdist.exchange_handles(b"x" * 128)
+
+
+class FakeReg:
+    def __init__(self, rank):
+        self.rank = rank
+        self.got = None
+
+    def export(self):
+        return bytes([0x40 + self.rank]) * 128
+
+    def connect(self, descs):
+        self.got = descs
+
+
+class FakeRegComm(FakeComm):
+    def register(self, tensor):
+        self.reg = FakeReg(self.rank)
+        self.reg.tensor = tensor
+        return self.reg
+
+
+def _register_worker(rank, world, port, q):
+    import torch
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_asplos_cowanmmsx23_b200 import dist as mdist
+        c = FakeRegComm(rank)
+        reg = mdist.register(c, torch.zeros(4))
+        q.put((rank, [d[0] - 0x40 for d in reg.got], all(len(d) == 128 for d in reg.got)))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_buffer_registration_exchange_two_ranks():
+    """dist.register (reading R15b): every rank's registration descriptor reaches every rank
+    in rank order (mscclRegConnect's contract), over a real world-size-2 gloo group."""
+    world = 2
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_register_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = [q.get(timeout=120) for _ in range(world)]
+    for p in procs:
+        p.join(timeout=60)
+        assert p.exitcode == 0
+    for rank, order, sizes in res:
+        assert order == [0, 1] and sizes
