@@ -842,7 +842,8 @@ mscclResult_t mscclCommExportHandle(mscclComm_t c, void* handle, size_t* bytes) 
   memcpy(handle, &h, sizeof(h));
   // parameters that both ends of a connection must agree on (region layout, warp partition)
   // parameters both ends of a connection must agree on (region layout, slot geometry)
-  int64_t meta[8] = {(int64_t)c->regionBytes, (int64_t)c->dev,     c->prm.threads,        c->prm.slots,
+  // (MSCCL_DIRECT too: a receiver that publishes its destination expects the sender to store there)
+  int64_t meta[8] = {(int64_t)c->regionBytes, c->prm.direct != 0, c->prm.threads,        c->prm.slots,
                      c->prm.slotBytes,         c->prm.llSlotBytes, c->prm.ll128SlotBytes, c->prm.maxChannels};
   static_assert(sizeof(cudaIpcMemHandle_t) + sizeof(meta) <= MSCCL_HANDLE_BYTES, "handle size");
   memcpy((char*)handle + sizeof(h), meta, sizeof(meta));
@@ -861,12 +862,12 @@ mscclResult_t mscclCommConnect(mscclComm_t c, const void* allHandles) {
     memcpy(&ih, h, sizeof(ih));
     int64_t meta[8];
     memcpy(meta, h + sizeof(ih), sizeof(meta));
-    const int64_t mine[8] = {(int64_t)c->regionBytes, 0,  c->prm.threads,        c->prm.slots,
+    const int64_t mine[8] = {(int64_t)c->regionBytes, c->prm.direct != 0, c->prm.threads,        c->prm.slots,
                              c->prm.slotBytes,         c->prm.llSlotBytes, c->prm.ll128SlotBytes, c->prm.maxChannels};
-    static const char* names[8] = {"region size", "", "MSCCL_THREADS", "MSCCL_SLOTS", "MSCCL_SLOT_BYTES",
+    static const char* names[8] = {"region size", "MSCCL_DIRECT", "MSCCL_THREADS", "MSCCL_SLOTS", "MSCCL_SLOT_BYTES",
                                    "MSCCL_LL_SLOT_BYTES", "MSCCL_LL128_SLOT_BYTES", "MSCCL_MAX_CHANNELS"};
     for (int k = 0; k < 8; k++)
-      if (k != 1 && meta[k] != mine[k]) {
+      if (meta[k] != mine[k]) {
         std::ostringstream o;
         o << "rank " << p << " uses a different " << names[k] << " (" << meta[k] << " vs " << mine[k]
           << "): every rank must use the same MSCCL_* parameters";
