@@ -59,6 +59,8 @@ def _algo(name, W, proto):
         return P.nvls_reducescatter(W, 2)
     if name == "nvls_ag":
         return P.nvls_allgather(W, 2)
+    if name == "ring_mm":
+        return P.ring_rs_multimem_ag_allreduce(W, 2)
     raise KeyError(name)
 
 
@@ -90,6 +92,7 @@ CASES = [
     ("nvls_ar", "Simple", "int32", "max", 7001, True),
     ("nvls_rs", "Simple", "float32", "sum", 9001, True),
     ("nvls_ag", "Simple", "int32", None, 5003, True),
+    ("ring_mm", "Simple", "float32", "sum", 12007, True),
 ]
 
 
@@ -200,7 +203,7 @@ def _run_world(world, cases, timeout):
             handshakes += hs
         # device-side evidence of cross-launch direct placement (reading R15b): senders found
         # a registered destination exactly when the buffers were registered
-        if not reg or proto != "Simple" or name.startswith("nvls"):
+        if not reg or proto != "Simple" or name.startswith("nvls") or name == "ring_mm":
             assert handshakes == 0, (name, proto, handshakes)
         elif name in DIRECT_EXPECTED:
             assert handshakes > 0, (name, proto, handshakes)

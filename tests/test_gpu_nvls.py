@@ -127,3 +127,17 @@ def test_multicast_hardware_path():
     finally:
         for c in comms:
             c.destroy()
+
+
+@pytest.mark.parametrize("R", [2, 4, 8])
+@pytest.mark.parametrize("dtype", ["bfloat16", "float32", "int32"])
+def test_mixed_ring_rs_multimem_ag_bit_exact(R, dtype):
+    """Connection ops and multimem ops in one program (the multimem kernel variant runs the
+    ring part too): bit-exact with the oracle."""
+    n = 50021
+    xs = synth.inputs(R, n, dtype, "uniform" if dtype != "int32" else "int")
+    algo = P.ring_rs_multimem_ag_allreduce(R, 2)
+    want = sim.simulate(irparse.parse(algo.to_xml()), xs, n, dtype, "sum")
+    got = _run(algo, xs, n, dtype, "sum")
+    for g, w in zip(got, want):
+        assert np.array_equal(np.asarray(g).view(np.uint8), np.asarray(w).view(np.uint8))

@@ -204,3 +204,24 @@ def test_sampled_oracle_evaluates_multimem_nodes():
     for q in (0, 5):
         got = sampled.allreduce_at(al, lambda r, i: xs[r][i], n, "bfloat16", "sum", idx, rank=q)
         assert np.array_equal(got, full[q][idx])
+
+
+@pytest.mark.parametrize("R", [2, 4, 8])
+def test_mixed_ring_rs_multimem_ag(R):
+    """A program mixing connection ops and multimem ops (ring ReduceScatter + multimem
+    AllGather): postcondition, rank-identical trees, race free (with the loader's direct
+    marking), brute-force exact on integer-valued inputs."""
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    for r in (1, 2):
+        algo = P.ring_rs_multimem_ag_allreduce(R, r)
+        ir = algo.to_xml()
+        al = irparse.parse(ir)
+        validate.validate(al, nranks=R, races=True)
+        symbolic.check(al)
+        assert races.check_direct(al, {q: runtime.direct_placement(ir, q) for q in range(R)}) == []
+        n = 97 * R + 3
+        xs = synth.inputs(R, n, "bfloat16", "intval")
+        got = sim.simulate(al, xs, n, "bfloat16", "sum")
+        ref = mpi_ref.allreduce(xs, "sum", "bfloat16")[0]
+        for g in got:
+            assert np.array_equal(nm.to_f64(g, "bfloat16"), ref)
