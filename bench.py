@@ -514,6 +514,8 @@ def extras(R, stream, nccl=None, S=256 * MIB):
     n = S // 2
     nb = n // W
     specs = (("nvls_allreduce", P.nvls_allreduce(W, 32 if R.world == 1 else 8), n, n, n),
+             ("nvls_reducescatter", P.nvls_reducescatter(W, 32 if R.world == 1 else 8), n, nb, nb),
+             ("nvls_allgather", P.nvls_allgather(W, 32 if R.world == 1 else 8), nb, n, nb),
              ("alltoall", P.alltoall_twostep(1, W, instances=2 if R.world == 1 else 4), n, n, nb),
              ("allgather", P.ring_allgather(W, 1, 32 if R.world == 1 else 8), nb, n, nb),
              ("reducescatter", P.ring_reducescatter(W, 1, 32 if R.world == 1 else 8), n, nb, nb))
@@ -525,7 +527,7 @@ def extras(R, stream, nccl=None, S=256 * MIB):
         t, mode = timed(lambda: R.call(progs, send, recv, cnt), 5, 2, stream, False, R)
         if coll == "alltoall":
             ok = check_alltoall(R, recv, W, n)
-        elif coll == "allgather":
+        elif coll in ("allgather", "nvls_allgather"):
             ok = check_allgather(R, recv, W, nb)
         elif coll == "nvls_allreduce":
             ranks = [q for q in (0, W - 1) if q in R.ranks]
@@ -535,10 +537,11 @@ def extras(R, stream, nccl=None, S=256 * MIB):
             ranks = [q for q in (0, W - 1) if q in R.ranks]
             bad, _ = sampled_parity(algo, recv, nb, ranks, local=R.ranks)
             ok = bad == 0
-        ent = {"busbw_GBps": round(busbw("allreduce" if coll == "nvls_allreduce" else coll, S, t, W), 2),
+        base_coll = coll.replace("nvls_", "")
+        ent = {"busbw_GBps": round(busbw(base_coll, S, t, W), 2),
                "ms": round(t * 1e3, 3),
                "ctas_per_rank": int(progs[0].info()["thread_blocks"]), "bit_exact": R.all_ok(ok)}
-        if nccl is not None and coll != "nvls_allreduce":
+        if nccl is not None and not coll.startswith("nvls_"):
             fn = {"alltoall": lambda: nccl.alltoall(send[0], recv[0], "bfloat16", W, cur()),
                   "allgather": lambda: nccl.allgather(send[0], recv[0], "bfloat16", cur()),
                   "reducescatter": lambda: nccl.reducescatter(send[0], recv[0], "bfloat16", "sum", cur())}[coll]
