@@ -536,6 +536,9 @@ __device__ __forceinline__ bool pieceLL(int64_t m, int64_t sendUnits, const char
 // read by the same 8 lanes in one warp load and accepted when its flag matches; no fence and
 // no separate head counter are needed. Lines per piece message: ceil(min(T, E - t*T)*w/120)
 // (the sender pads, reading R2).
+#ifndef MSCCL_LL128_BACKOFF
+#define MSCCL_LL128_BACKOFF 8  // empty polls of a batch before the poller sleeps between polls
+#endif
 #ifndef MSCCL_LL128_UNROLL
 #define MSCCL_LL128_UNROLL 4  // lines in flight per 8-lane group of a warp
 #endif
@@ -586,7 +589,7 @@ __device__ __forceinline__ bool ll128Batch(int64_t base, int64_t bytes, int64_t 
         }
       }
       if (__all_sync(0xffffffffu, mine)) break;
-      if (it >= 8) __nanosleep(64);  // back off after a few empty polls (L2 traffic)
+      if (it >= MSCCL_LL128_BACKOFF) __nanosleep(64);  // back off after empty polls (L2 traffic)
       if ((it & 255u) == 255u) {
         uint64_t now = globaltimer();
         if (t0 == 0) t0 = now;
