@@ -893,6 +893,11 @@ mscclResult_t mscclCommDestroy(mscclComm_t c) {
     for (auto* r : std::vector<mscclReg*>(c->regs))
       if (r) releaseReg(c, r);
     c->regs.clear();
+    if (!c->nvls.empty()) {  // NVLS buffers the caller did not free (mscclNvlsFree of each rank)
+      std::vector<void*> mine;
+      for (auto& nv : c->nvls) mine.push_back(nv.uc);
+      for (void* p : mine) mscclNvlsFree(&c, 1, &p);
+    }
     cudaFree(c->dRegMap);
     cudaFree(c->dPeerRegion);
     for (int p = 0; p < c->nranks; p++)
@@ -1120,9 +1125,40 @@ mscclResult_t mscclNvlsAlloc(mscclComm_t* comms, int n, size_t bytes, void** ptr
     }
   }
   const size_t size = mp.size;
-  for (int i = 0; i < n; i++) CUCHECK(comms[i], d.mcAddDevice(mc, (CUdevice)comms[i]->dev));
-  // the multicast address, mapped once and accessible from every device
+  // everything created below is released again if a later step fails
+  struct Made {
+    int dev;
+    CUmemGenericAllocationHandle phys;
+    CUdeviceptr uc;
+    bool bound, mapped;
+  };
+  std::vector<Made> made;
   CUdeviceptr mcva = 0;
+  bool mcMapped = false;
+  auto undo = [&]() {
+    for (auto& m : made) {
+      DeviceGuard g(m.dev);
+      if (m.mapped) d.memUnmap(m.uc, size);
+      if (m.uc) d.addrFree(m.uc, size);
+      if (m.bound) d.mcUnbind(mc, (CUdevice)m.dev, 0, size);
+      if (m.phys) d.memRelease(m.phys);
+    }
+    if (mcMapped) d.memUnmap(mcva, size);
+    if (mcva) d.addrFree(mcva, size);
+    d.memRelease(mc);
+  };
+#define NVTRY(c, call)                                                                        \
+  do {                                                                                        \
+    CUresult e_ = (call);                                                                     \
+    if (e_ != CUDA_SUCCESS) {                                                                 \
+      undo();                                                                                 \
+      std::ostringstream o_;                                                                  \
+      o_ << #call << " failed with CUresult " << (int)e_;                                     \
+      return setErr((c), mscclUnhandledCudaError, o_.str());                                  \
+    }                                                                                         \
+  } while (0)
+  for (int i = 0; i < n; i++) NVTRY(comms[i], d.mcAddDevice(mc, (CUdevice)comms[i]->dev));
+  // the multicast address, mapped once and accessible from every device
   std::vector<CUmemAccessDesc> acc(n);
   for (int i = 0; i < n; i++) {
     acc[i].location.type = CU_MEM_LOCATION_TYPE_DEVICE;
@@ -1133,30 +1169,37 @@ mscclResult_t mscclNvlsAlloc(mscclComm_t* comms, int n, size_t bytes, void** ptr
     DeviceGuard g(comms[i]->dev);
     cudaFree(nullptr);
     ap.location.id = comms[i]->dev;
-    CUmemGenericAllocationHandle phys = 0;
-    CUCHECK(comms[i], d.memCreate(&phys, size, &ap, 0));
-    CUCHECK(comms[i], d.mcBindMem(mc, 0, phys, 0, size, 0));
-    CUdeviceptr uc = 0;
-    CUCHECK(comms[i], d.addrReserve(&uc, size, g2, 0, 0));
-    CUCHECK(comms[i], d.memMap(uc, size, 0, phys, 0));
-    CUCHECK(comms[i], d.setAccess(uc, size, acc.data(), acc.size()));  // peers reach it too (unicast form)
+    made.push_back({comms[i]->dev, 0, 0, false, false});
+    Made& m = made.back();
+    NVTRY(comms[i], d.memCreate(&m.phys, size, &ap, 0));
+    NVTRY(comms[i], d.mcBindMem(mc, 0, m.phys, 0, size, 0));
+    m.bound = true;
+    NVTRY(comms[i], d.addrReserve(&m.uc, size, g2, 0, 0));
+    NVTRY(comms[i], d.memMap(m.uc, size, 0, m.phys, 0));
+    m.mapped = true;
+    NVTRY(comms[i], d.setAccess(m.uc, size, acc.data(), acc.size()));  // peers reach it too (unicast form)
     if (i == 0) {
-      CUCHECK(comms[i], d.addrReserve(&mcva, size, g2, 0, 0));
-      CUCHECK(comms[i], d.memMap(mcva, size, 0, mc, 0));
-      CUCHECK(comms[i], d.setAccess(mcva, size, acc.data(), acc.size()));
+      NVTRY(comms[i], d.addrReserve(&mcva, size, g2, 0, 0));
+      NVTRY(comms[i], d.memMap(mcva, size, 0, mc, 0));
+      mcMapped = true;
+      NVTRY(comms[i], d.setAccess(mcva, size, acc.data(), acc.size()));
     }
-    mscclComm::Nvls nv{(char*)uc, nullptr, size, (unsigned long long)phys, (unsigned long long)mc, i == 0};
-    comms[i]->nvls.push_back(nv);
-    ptrs[i] = (void*)uc;
   }
-  for (int i = 0; i < n; i++) comms[i]->nvls.back().mc = (char*)mcva;
+#undef NVTRY
+  for (int i = 0; i < n; i++) {
+    mscclComm::Nvls nv{(char*)made[i].uc, (char*)mcva, size, (unsigned long long)made[i].phys,
+                       (unsigned long long)mc, i == 0};
+    comms[i]->nvls.push_back(nv);
+    ptrs[i] = (void*)made[i].uc;
+  }
   return mscclSuccess;
 }
 
 mscclResult_t mscclNvlsFree(mscclComm_t* comms, int n, void** ptrs) {
   if (!comms || n < 1 || !ptrs) return mscclInvalidArgument;
   const Drv& d = drv();
-  for (int i = 0; i < n; i++) {
+  std::vector<mscclComm::Nvls> owners;
+  for (int i = 0; i < n; i++) {  // every rank's memory first ...
     mscclComm* c = comms[i];
     DeviceGuard g(c->dev);
     CUDACHECK(c, cudaDeviceSynchronize());
@@ -1166,12 +1209,13 @@ mscclResult_t mscclNvlsFree(mscclComm_t* comms, int n, void** ptrs) {
     d.addrFree((CUdeviceptr)it->uc, it->size);
     d.mcUnbind((CUmemGenericAllocationHandle)it->mcHandle, (CUdevice)c->dev, 0, it->size);
     d.memRelease((CUmemGenericAllocationHandle)it->phys);
-    if (it->owner) {
-      d.memUnmap((CUdeviceptr)it->mc, it->size);
-      d.addrFree((CUdeviceptr)it->mc, it->size);
-      d.memRelease((CUmemGenericAllocationHandle)it->mcHandle);
-    }
+    if (it->owner) owners.push_back(*it);
     c->nvls.erase(it);
+  }
+  for (auto& o : owners) {  // ... then the multicast address and object
+    d.memUnmap((CUdeviceptr)o.mc, o.size);
+    d.addrFree((CUdeviceptr)o.mc, o.size);
+    d.memRelease((CUmemGenericAllocationHandle)o.mcHandle);
   }
   return mscclSuccess;
 }
