@@ -299,3 +299,84 @@ def test_connect_rejects_mismatched_parameters():
     for p in procs:
         p.join(timeout=60)
     assert res[0] == (5, True) and res[1] == (5, True), res
+
+
+SEQUENCE = [("ring", "Simple", "float32", "sum", 30001, True), ("a2a", "Simple", "bfloat16", None, 4003, True),
+            ("ring", "LL", "bfloat16", "sum", 2001, False), ("nvls_ar", "Simple", "bfloat16", "sum", 9001, True),
+            ("allgather", "Simple", "int32", None, 5001, True), ("ring", "LL128", "float16", "sum", 7001, False),
+            ("ring_i2", "Simple", "bfloat16", "sum", 40001, False), ("ring_mm", "Simple", "float32", "sum", 8001, True)]
+
+
+def _sequence_worker(rank, world, port, q):
+    import torch
+    import torch.distributed as dist
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        from paper_conf_asplos_cowanmmsx23_b200 import dist as mdist
+        from paper_conf_asplos_cowanmmsx23_b200 import runtime
+        runtime.set_param("MSCCL_TIMEOUT_S", 120)
+        for k in ("MSCCL_SLOT_BYTES", "MSCCL_LL_SLOT_BYTES", "MSCCL_LL128_SLOT_BYTES"):
+            runtime.set_param(k, 16384)
+        runtime.set_param("MSCCL_MAX_CHANNELS", 8)
+        runtime.set_param("MSCCL_THREADS", 128)
+        comm = mdist.init_from_process_group(0)
+        progs = [comm.load(_algo(name, world, proto).to_xml()) for name, proto, *_ in SEQUENCE]
+        bufs = []
+        for name, proto, dtype, op, n, reg in SEQUENCE:
+            xs, out_elems = _inputs(name, world, n, dtype)
+            x = torch.from_numpy(xs[rank].view(np.uint8).copy()).cuda()
+            y = torch.full((out_elems * xs[0].itemsize,), 0xA5, dtype=torch.uint8, device="cuda")
+            regs = [mdist.register(comm, x), mdist.register(comm, y)] if reg else []
+            bufs.append((x, y, regs))
+        for rep in range(2):   # every program back to back on one stream, no host sync in between
+            for (name, proto, dtype, op, n, reg), p, (x, y, _) in zip(SEQUENCE, progs, bufs):
+                comm.run(p, x, y, n, op=op or "sum", dtype=dtype)
+        torch.cuda.synchronize()
+        out = [y.cpu().numpy().copy() for _, y, _ in bufs]
+        dist.barrier()
+        for _, _, regs in bufs:
+            for r_ in regs:
+                r_.deregister()
+        q.put((rank, out, comm.async_error()))
+        dist.barrier()
+        comm.destroy()
+    except Exception as e:
+        import traceback
+        q.put((rank, "%r\n%s" % (e, traceback.format_exc()), -1))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_mixed_program_sequence_four_processes():
+    """Eight different programs -- Simple with and without registered buffers, LL, LL128,
+    multimem, and a mixed program -- run back to back twice on one stream per process. The
+    per-connection launch ordinals, the ready lines, the multimem epochs and the
+    per-protocol FIFOs must stay consistent across every kind of launch (R15b, R20, R23).
+    Every output is bit-exact with the oracle."""
+    world = 4
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_sequence_worker, args=(r, world, port, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    res = {}
+    try:
+        for _ in range(world):
+            r, out, err = q.get(timeout=900)
+            res[r] = (out, err)
+    finally:
+        for p in procs:
+            p.join(timeout=60)
+            if p.is_alive():
+                p.kill()
+    for r in range(world):
+        assert not isinstance(res[r][0], str), res[r][0]
+        assert res[r][1] == 0
+    for k, (name, proto, dtype, op, n, reg) in enumerate(SEQUENCE):
+        want = _expected(name, world, proto, dtype, op, n)
+        for r in range(world):
+            w = np.ascontiguousarray(want[r]).view(np.uint8)
+            assert np.array_equal(res[r][0][k][:w.size], w), (name, proto, r)
