@@ -1,4 +1,5 @@
-"""Small cases for compute-sanitizer (memcheck): every protocol, direct on/off, ragged sizes."""
+"""Small cases for compute-sanitizer (memcheck / synccheck): every protocol, direct on/off, multimem
+programs, ragged sizes."""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tests"))
@@ -18,7 +19,9 @@ for direct in (1, 0):
                                  ("ring_LL128", P.ring_allreduce(4, protocol="LL128"), 4, 5001, "float16"),
                                  ("allpairs", P.allpairs_allreduce(4, protocol="Simple"), 4, 3003, "float32"),
                                  ("oneshot", P.oneshot_allreduce(4), 4, 777, "int32"),
-                                 ("hier", P.hierarchical_allreduce(2, 2), 4, 999, "float32")]:
+                                 ("hier", P.hierarchical_allreduce(2, 2), 4, 999, "float32"),
+                                 ("nvls", P.nvls_allreduce(4, 2), 4, 4099, "bfloat16"),
+                                 ("ring_mm", P.ring_rs_multimem_ag_allreduce(4, 2), 4, 3001, "float32")]:
         xs = synth.inputs(R, n, dt, "uniform" if dt != "int32" else "int")
         want = sim.simulate(irparse.parse(algo.to_xml()), xs, n, dt)
         got = gpu_util.run_program(algo.to_xml(), xs, n, dt)
