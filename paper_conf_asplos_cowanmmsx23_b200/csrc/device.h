@@ -82,6 +82,10 @@ struct RankArgs {
                               // resolved a direct destination (mscclCommGetStats)
   char* const* peerRegion;    // every rank's shared region in this address space (group barriers)
   int32_t myRank, nRanks;
+  // latency kernels: each thread block's DevTB followed by its instructions, one record per
+  // block at tbRec + tb * tbRecStride (0 = no records: instructions longer than the stage)
+  const char* tbRec;
+  int64_t tbRecStride;
   // NVSwitch multicast addresses of this rank's in / out buffers when they lie inside an
   // NVLS buffer (mscclNvlsAlloc), else null: multimem ops on them use multimem.ld_reduce /
   // multimem.st (the hardware form of reading R23)

@@ -1394,18 +1394,37 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, MSCCL_MIN_BLOCKS) mscclInte
   if (tbi >= ra.nTB) return;
   // Prologue: the thread block's descriptor and instruction list are staged in
   // shared memory by parallel 16-byte loads, so the instruction loop never waits on a global
-  // round trip to decode a step.
+  // round trip to decode a step. Latency kernels load both in ONE round trip from the
+  // program's per-block record (DevTB followed by its instructions); the generation word is
+  // loaded at the same time.
   __shared__ __align__(16) DevTB sTB;
   __shared__ __align__(16) DevInstr sIns[kLat ? MSCCL_SMEM_INSTR : 1];
-  if (kLat && threadIdx.x < sizeof(DevTB) / 16)
-    reinterpret_cast<uint4*>(&sTB)[threadIdx.x] = reinterpret_cast<const uint4*>(&ra.tbs[tbi])[threadIdx.x];
-  if (kLat) __syncthreads();
+  uint64_t genEarly = 0;
+  const DevInstr* ins = nullptr;
+  if constexpr (kLat) {
+    if (ra.tbRecStride) {
+      const uint4* rec = reinterpret_cast<const uint4*>(ra.tbRec + (int64_t)tbi * ra.tbRecStride);
+      const int nw = (int)(ra.tbRecStride / 16), ntb = (int)(sizeof(DevTB) / 16);
+      for (int i = threadIdx.x; i < nw; i += blockDim.x) {
+        const uint4 v = rec[i];
+        if (i < ntb) reinterpret_cast<uint4*>(&sTB)[i] = v;
+        else reinterpret_cast<uint4*>(sIns)[i - ntb] = v;
+      }
+      genEarly = *(volatile uint64_t*)&ra.gen[tbi];
+      ins = sIns;
+    } else if (threadIdx.x < sizeof(DevTB) / 16) {
+      reinterpret_cast<uint4*>(&sTB)[threadIdx.x] = reinterpret_cast<const uint4*>(&ra.tbs[tbi])[threadIdx.x];
+    }
+    __syncthreads();
+  }
   const DevTB& tb = kLat ? sTB : ra.tbs[tbi];
-  const DevInstr* ins = ra.instrs + tb.instrStart;
-  if (kLat && tb.nSteps <= MSCCL_SMEM_INSTR) {
-    for (int i = threadIdx.x; i < tb.nSteps * (int)(sizeof(DevInstr) / 16); i += blockDim.x)
-      reinterpret_cast<uint4*>(sIns)[i] = reinterpret_cast<const uint4*>(ins)[i];
-    ins = sIns;
+  if (!ins) {
+    ins = ra.instrs + tb.instrStart;
+    if (kLat && tb.nSteps <= MSCCL_SMEM_INSTR) {
+      for (int i = threadIdx.x; i < tb.nSteps * (int)(sizeof(DevInstr) / 16); i += blockDim.x)
+        reinterpret_cast<uint4*>(sIns)[i] = reinterpret_cast<const uint4*>(ins)[i];
+      ins = sIns;
+    }
   }
   __shared__ uint64_t sAck;
   __shared__ char* sPeerDst[3];
@@ -1424,7 +1443,7 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, MSCCL_MIN_BLOCKS) mscclInte
   }
   uint64_t sent = tb.sendFifo ? *(volatile uint64_t*)tb.sendCnt : 0;
   uint64_t recvd = tb.recvFifo ? *(volatile uint64_t*)tb.recvCnt : 0;
-  const uint64_t gen = *(volatile uint64_t*)&ra.gen[tbi];
+  const uint64_t gen = (kLat && ra.tbRecStride) ? genEarly : *(volatile uint64_t*)&ra.gen[tbi];
   // Launch ordinals per connection (word 1 of the persistent counter lines) stay in lock-step
   // on both ends in every launch; in cross-launch direct mode the receiving thread block also
   // publishes where its destinations are (reading R15b), released by one fence.

@@ -176,6 +176,8 @@ struct mscclProgram {
   char* dScratch = nullptr;
   size_t scratchBytes = 0;
   std::vector<char*> retiredScratch;  // outgrown scratch buffers: a captured graph may still use them
+  char* dRec = nullptr;    // latency kernels: per-block records (DevTB + instructions), see RankArgs
+  int64_t recStride = 0;
   int maxCnt = 1;
   bool hasReduce = false;
   bool allDirect = true;  // every message of this rank's program is a direct placement (R15)
@@ -257,6 +259,7 @@ void freeProgram(mscclProgram* p) {
   cudaFree(p->dDeps);
   cudaFree(p->dSem);
   cudaFree(p->dScratch);
+  cudaFree(p->dRec);
   for (char* x : p->retiredScratch) cudaFree(x);
   delete p;
 }
@@ -521,6 +524,8 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
       ra.hostAbort = cl->comm->hostAbortDev;
       ra.regMap = cl->comm->dRegMap;
       ra.peerRegion = cl->comm->dPeerRegion;
+      ra.tbRec = p->dRec;
+      ra.tbRecStride = p->dRec ? p->recStride : 0;
       ra.myRank = cl->comm->rank;
       ra.nRanks = cl->comm->nranks;
       if (mm) {  // NVSwitch multicast addresses of in / out (reading R23, hardware form)
@@ -1406,6 +1411,24 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
   if (!deps.empty()) {
     CUDACHECK(c, cudaMalloc(&p->dDeps, deps.size() * sizeof(uint64_t)));
     CUDACHECK(c, cudaMemcpy(p->dDeps, deps.data(), deps.size() * sizeof(uint64_t), cudaMemcpyHostToDevice));
+  }
+  // per-block records for the latency kernels: DevTB followed by its instructions, fixed
+  // stride, so one round trip stages both (only when every list fits the shared stage)
+  {
+    int maxSteps = 0;
+    for (auto& d : tbs) maxSteps = std::max(maxSteps, d.nSteps);
+    if (p->nTB && maxSteps <= 64) {
+      p->recStride = (int64_t)(sizeof(DevTB) + (size_t)maxSteps * sizeof(DevInstr) + 15) / 16 * 16;
+      std::vector<char> host((size_t)p->nTB * p->recStride, 0);
+      for (int t = 0; t < p->nTB; t++) {
+        memcpy(host.data() + (size_t)t * p->recStride, &tbs[t], sizeof(DevTB));
+        if (tbs[t].nSteps)
+          memcpy(host.data() + (size_t)t * p->recStride + sizeof(DevTB), &ins[tbs[t].instrStart],
+                 (size_t)tbs[t].nSteps * sizeof(DevInstr));
+      }
+      CUDACHECK(c, cudaMalloc(&p->dRec, host.size()));
+      CUDACHECK(c, cudaMemcpy(p->dRec, host.data(), host.size(), cudaMemcpyHostToDevice));
+    }
   }
   // scratch pre-sized for the largest call of the size range: every chunk of a
   // call with count*w < maxBytes has E*w <= maxBytes/cb + 16 bytes (reading R1)
