@@ -69,7 +69,7 @@ typedef enum { mscclSum = 0, mscclProd = 1, mscclMax = 2, mscclMin = 3, mscclNum
 
 /* One process drives `ndev` ranks; rank i runs on device devlist[i] (devlist may be NULL:
  * devices 0..ndev-1). Distinct devices are connected by CUDA peer access over NVLink.
- * Repeated device ids are VIRTUAL RANKS: several ranks on one GPU, whose buffers and
+ * Repeated device ids are VIRTUAL RANKS (at most 8 per device): several ranks on one GPU, whose buffers and
  * FIFOs all live in that GPU's HBM (used for correctness work on one GPU). Ranks that
  * share a device must issue their calls inside mscclGroupStart/End so that they run in
  * ONE cooperative launch (all thread blocks co-resident, §6.2).

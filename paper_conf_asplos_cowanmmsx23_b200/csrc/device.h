@@ -8,7 +8,10 @@
 
 namespace msccl {
 
-#define MSCCL_MAX_LOCAL 16   // ranks that one kernel launch may cover (virtual ranks)
+#ifndef MSCCL_MAX_LOCAL
+#define MSCCL_MAX_LOCAL 8    // ranks that one kernel launch may cover (virtual ranks); every RankArgs slot
+                             // is a kernel parameter: 16 -> 8 cut the launch floor by ~0.4 us
+#endif
 #define MSCCL_FLAG_STRIDE 16 // u64 words between connection counters (one 128-byte line each)
 #define MSCCL_REF_REG (1ull << 63)  // destination reference: registered-buffer (index, offset) form
 #define MSCCL_MM_MAX_TB 64   // thread-block ids that may hold multimem ops (group-barrier lines)

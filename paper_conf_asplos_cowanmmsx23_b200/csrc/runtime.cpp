@@ -780,6 +780,15 @@ uint64_t* msccl_debug_trace(void) { return gTraceHost; }
 
 mscclResult_t mscclCommInitAll(mscclComm_t* comms, int ndev, const int* devlist) {
   if (!comms || ndev < 1) return setErr(nullptr, mscclInvalidArgument, "bad arguments to mscclCommInitAll");
+  for (int i = 0; i < ndev; i++) {  // every rank of one device runs in one launch (MSCCL_MAX_LOCAL slots)
+    int same = 0;
+    for (int j = 0; j < ndev; j++) same += (devlist ? devlist[j] : j) == (devlist ? devlist[i] : i);
+    if (same > MSCCL_MAX_LOCAL) {
+      std::ostringstream o;
+      o << "mscclCommInitAll: at most " << MSCCL_MAX_LOCAL << " ranks per device";
+      return setErr(nullptr, mscclInvalidArgument, o.str());
+    }
+  }
   auto clique = std::make_shared<Clique>();
   for (int i = 0; i < ndev; i++) {
     mscclComm* c = new mscclComm();
