@@ -60,6 +60,8 @@ def parse():
     ap.add_argument("--program", default="ring",
                     choices=["ring", "allpairs", "oneshot", "alltoall", "allgather", "reducescatter", "nvls"])
     ap.add_argument("--channels", type=int, default=1)
+    ap.add_argument("--split", action="store_true", help="ring: AllGather half on its own channels (reading R26)")
+    ap.add_argument("--rings", type=int, default=1, help="ring: K interleaved logical rings per thread block (R27)")
     ap.add_argument("--instances", type=int, default=32)
     ap.add_argument("--protocol", default="Simple")
     ap.add_argument("--threads", type=int, default=256)
@@ -168,7 +170,8 @@ def busbw(coll, S, t, R):
 def build_program(args, R):
     from paper_conf_asplos_cowanmmsx23_b200 import programs as P
     if args.program == "ring":
-        return P.ring_allreduce(R, channels=args.channels, instances=args.instances, protocol=args.protocol)
+        return P.ring_allreduce(R, channels=args.channels, instances=args.instances, protocol=args.protocol,
+                                split_phases=args.split, rings=args.rings)
     if args.program == "allpairs":
         return P.allpairs_allreduce(R, instances=args.instances, protocol=args.protocol)
     if args.program == "oneshot":
@@ -323,6 +326,7 @@ def config_dict(args, R, N):
                            int(args.size_mib)),
             "program": args.program, "ranks": R, "bytes_per_rank": int(args.size_mib * MIB),
             "channels": args.channels, "instances": args.instances, "protocol": args.protocol,
+            "split_phases": bool(args.split), "rings": args.rings,
             "threads": args.threads, "slots": args.slots, "slot_bytes": args.slot_kib * 1024,
             "l2": "inputs (%d MiB total) larger than L2 (126 MB); no flush" % int(args.size_mib * (R if N == 1 else 1)),
             "parallelism": "virtual%d" % R if N == 1 else "ranks%d" % N}
@@ -333,7 +337,7 @@ def set_params(rt, args):
     rt.set_param("MSCCL_SLOTS", args.slots)
     rt.set_param("MSCCL_SLOT_BYTES", args.slot_kib * 1024)
     rt.set_param("MSCCL_THREADS", args.threads)
-    rt.set_param("MSCCL_MAX_CHANNELS", max(32, args.channels * args.instances))
+    rt.set_param("MSCCL_MAX_CHANNELS", max(32, args.channels * args.instances * (2 if args.split else 1)))
     rt.set_param("MSCCL_TIMEOUT_S", 60)
 
 
@@ -1023,8 +1027,8 @@ def main():
         achieved = alg_bytes / launch_s / 1e9
         traffic, prof = ncu_traffic()
         l2peak, l2src = l2_peak()
-        is_default = (args.program, args.instances, args.channels, args.slot_kib, args.threads, args.protocol) == \
-            ("ring", 32, 1, 256, 256, "Simple")
+        is_default = (args.program, args.instances, args.channels, args.slot_kib, args.threads, args.protocol,
+                      args.split, args.rings) == ("ring", 32, 1, 256, 256, "Simple", False, 1)
         out["roofline"] = {
             "bound": "hbm", "achieved": round(hbm_achieved, 1), "peak": peak, "unit": "GB/s",
             "frac": round(hbm_achieved / peak, 4), "traffic": traffic if is_default else None,

@@ -232,7 +232,10 @@ const char* mscclGetLastError(mscclComm_t comm); /* comm may be NULL: last globa
  * -- each protocol has its own slots; "MSCCL_MAX_CHANNELS" (32); "MSCCL_THREADS" threads
  * per CTA (64..256, default 256 = 2 CTAs per SM); "MSCCL_TIMEOUT_S" watchdog (default 60,
  * <= 0 disables); "MSCCL_DIRECT" direct placement (1); "MSCCL_DIRECT_TILE" one tile per
- * chunk when every message is direct (1); "MSCCL_MAX_REGISTRATIONS" (64). All ranks must
+ * chunk when every message is direct (1); "MSCCL_DIRECT_HINTS" L2 hints of direct stores, a
+ * bit set (default 9: bit 0 terminal direct sends evict_first, bit 3 forwarded direct sends
+ * evict_normal; bit 1 demote forwarded lines after reading, bit 2 FIFO stores evict_normal:
+ * measured slower, off); "MSCCL_MAX_REGISTRATIONS" (64). All ranks must
  * use the same values (mscclCommConnect checks). Returns mscclInvalidArgument for an
  * unknown key. */
 mscclResult_t mscclSetParam(const char* key, int64_t value);

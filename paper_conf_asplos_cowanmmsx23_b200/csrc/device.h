@@ -111,7 +111,9 @@ struct KernelArgs {
   // direct placement (reading R15): 0 off; 1 every rank is in this launch (rank == slot);
   // 2 cross-launch (ranks in other launches / processes, ready handshake per connection)
   int32_t direct;
-  int32_t directHints;        // bit 0: terminal direct sends store L2 evict_first (cache hint)
+  int32_t directHints;        // L2 hints (interp.cuh HINT_*): bit 0 terminal direct sends evict_first,
+                              // bit 1 demote read forwarded lines, bit 2 FIFO stores / bit 3 direct
+                              // forwards evict_normal (default 9)
   // multimem ops (reading R23): 0 none; 1 every rank in this launch (slot r = rank r, buffers
   // from the launch arguments, no barrier); 2 cross-launch (group barrier lines publish the
   // ranks' buffer references at the start and completion at the end)

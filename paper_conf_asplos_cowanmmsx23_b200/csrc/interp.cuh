@@ -160,6 +160,16 @@ __device__ __forceinline__ uint64_t policyEvictFirst() {
 #endif
   return p;
 }
+__device__ __forceinline__ uint64_t policyEvictNormal() {
+  uint64_t p;
+  asm volatile("createpolicy.fractional.L2::evict_normal.b64 %0, 1.0;" : "=l"(p));
+  return p;
+}
+// drop a line's L2 priority back to normal (a forwarded line that was stored evict_last and
+// has now been read by its forwarder: it is final output, no longer worth protecting)
+__device__ __forceinline__ void demoteL2(const void* p) {
+  asm volatile("applypriority.global.L2::evict_normal [%0], 128;" ::"l"(p) : "memory");
+}
 __device__ __forceinline__ uint64_t policyEvictLast() {
   uint64_t p;
 #if MSCCL_NO_HINTS
@@ -346,7 +356,9 @@ __device__ __forceinline__ void chunkSpan(const KernelArgs& a, int buf, int64_t 
 // Returns the number of VB-byte vectors processed.
 // store hint of one piece: a direct send whose receiver does not forward the data stores it
 // L2 evict_first (reading R15, DI_SEND_TERMINAL)
-enum { HINT_SEND_FIRST = 1 };
+// HINT_SRC_DEMOTE: the src lines were stored evict_last by a direct sender (forwarded data):
+// demote them once read. HINT_SEND_NORMAL: store the outgoing lines evict_normal.
+enum { HINT_SEND_FIRST = 1, HINT_SRC_DEMOTE = 2, HINT_SEND_NORMAL = 4 };
 
 template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST, int VB>
 __device__ __forceinline__ int64_t vecLoop(int64_t nvec, const char* rslot, const char* src, char* dst, char* sslot,
@@ -354,7 +366,7 @@ __device__ __forceinline__ int64_t vecLoop(int64_t nvec, const char* rslot, cons
   typedef typename VecT<VB>::T Vec;
   constexpr int U = ((int)RECV + (int)SRC + (int)REDDST) >= 2 ? MSCCL_UNROLL : MSCCL_UNROLL1;
   const uint64_t pFirst = policyEvictFirst(), pLast0 = policyEvictLast();
-  const uint64_t pLast = (hint & HINT_SEND_FIRST) ? pFirst : pLast0;
+  const uint64_t pLast = (hint & HINT_SEND_FIRST) ? pFirst : (hint & HINT_SEND_NORMAL) ? policyEvictNormal() : pLast0;
   const bool canDiscard = RECV && ((((uintptr_t)rslot) & 127) == 0);
   const int lane = ti & 31, warp = ti >> 5, nw = nt >> 5;
   // Full blocks of U x 32 vectors, one block per warp-iteration (warp-uniform trip count,
@@ -384,6 +396,12 @@ __device__ __forceinline__ int64_t vecLoop(int64_t nvec, const char* rslot, cons
       if (canDiscard && ((lane * VB) & 127) == 0) {
 #pragma unroll
         for (int u = 0; u < U; u++) discardL2(rslot + (base + u * 32) * VB);
+      }
+    }
+    if constexpr (SRC && !RECV && !REDDST) {
+      if ((hint & HINT_SRC_DEMOTE) && ((lane * VB) & 127) == 0) {
+#pragma unroll
+        for (int u = 0; u < U; u++) demoteL2(src + (base + u * 32) * VB);
       }
     }
   }
@@ -755,9 +773,14 @@ __device__ __noinline__ void movePiecesSimple(const Ctx& c, const DevTB& tb, con
       if (rl - a0 < m) m = rl - a0;
     }
     if (m <= 0) continue;
-    const int hint = (sdirect && (in.flags & DI_SEND_TERMINAL)) ? (a.directHints & HINT_SEND_FIRST) : 0;
+    int hint = (sdirect && (in.flags & DI_SEND_TERMINAL)) ? (a.directHints & HINT_SEND_FIRST) : 0;
+    if (SEND && !(hint & HINT_SEND_FIRST)) {  // MSCCL_DIRECT_HINTS bit 2: FIFO stores, bit 3: direct forwards
+      if (sdirect ? (a.directHints & 8) : (a.directHints & 4)) hint |= HINT_SEND_NORMAL;
+    }
     if (rdirect) {  // the data is already in dst (the sender wrote it there)
-      if (SEND) pieceSimple<DT, OP, false, true, true, false, false>(m, nullptr, dst, nullptr, so, c.tid, c.nt, hint);
+      if (SEND)
+        pieceSimple<DT, OP, false, true, true, false, false>(m, nullptr, dst, nullptr, so, c.tid, c.nt,
+                                                             hint | (a.directHints & HINT_SRC_DEMOTE));
       continue;
     }
     pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, RECV ? rslot + j * a.T * w : nullptr, src, dst, so, c.tid, c.nt,

@@ -31,7 +31,7 @@ namespace {
 // threads per CTA (2 CTAs per SM), direct placement on. LL / LL128 have their own FIFO slots.
 struct Params {
   int64_t slots = 4, slotBytes = 262144, llSlotBytes = 65536, ll128SlotBytes = 262144, maxChannels = 32,
-          threads = 256, timeoutS = 60, direct = 1, directTile = 1, directHints = 1, regMax = 64;
+          threads = 256, timeoutS = 60, direct = 1, directTile = 1, directHints = 9, regMax = 64;
 };
 
 std::mutex gMu;

@@ -70,6 +70,8 @@ AR = [
     ("ring", lambda R: P.ring_allreduce(R)),
     ("ring_inplace", lambda R: P.ring_allreduce(R, inplace=True)),
     ("ring_channels_instances", lambda R: P.ring_allreduce(R, channels=R, instances=2)),
+    ("ring_split", lambda R: P.ring_allreduce(R, channels=R, split_phases=True)),
+    ("ring_k2", lambda R: P.ring_allreduce(R, rings=2)),
     ("ring_LL", lambda R: P.ring_allreduce(R, protocol="LL")),
     ("ring_LL128", lambda R: P.ring_allreduce(R, instances=2, protocol="LL128")),
     ("allpairs_LL128", lambda R: P.allpairs_allreduce(R, protocol="LL128")),

@@ -80,6 +80,11 @@ def test_cpp_deadlock_fixtures(rt):
     text = irmutate.outstanding_sends_ir()
     assert not rt.validate(text, 2, slots=2)[0]
     assert rt.validate(text, 2, slots=3)[0]
+    for K in (2, 3):  # K interleaved rings (reading R27) need K+1 slots, as in the oracle
+        k = P.ring_allreduce(8, rings=K).to_xml()
+        ok, msg = rt.validate(k, 8, slots=K)
+        assert not ok and msg.startswith("V9")
+        assert rt.validate(k, 8, slots=K + 1)[0]
 
 
 def test_cpp_thread_block_limit(rt):

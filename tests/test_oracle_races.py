@@ -32,6 +32,8 @@ SHIPPED = {
     "ring": lambda R, r: P.ring_allreduce(R, instances=r),
     "ring_inplace": lambda R, r: P.ring_allreduce(R, instances=r, inplace=True),
     "ring_channels": lambda R, r: P.ring_allreduce(R, channels=R, instances=r),
+    "ring_split": lambda R, r: P.ring_allreduce(R, channels=R, instances=r, split_phases=True),
+    "ring_k2": lambda R, r: P.ring_allreduce(R, instances=r, rings=2),
     "ring_LL128": lambda R, r: P.ring_allreduce(R, instances=r, protocol="LL128"),
     "allpairs": lambda R, r: P.allpairs_allreduce(R, instances=r, protocol="Simple"),
     "oneshot": lambda R, r: P.oneshot_allreduce(R, instances=r, protocol="Simple"),

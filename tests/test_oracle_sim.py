@@ -52,6 +52,8 @@ PROGS_AR = [
     ("ring", lambda R: P.ring_allreduce(R)),
     ("ring_inplace", lambda R: P.ring_allreduce(R, inplace=True)),
     ("ring_channels", lambda R: P.ring_allreduce(R, channels=R, instances=2)),
+    ("ring_split", lambda R: P.ring_allreduce(R, channels=R, split_phases=True)),
+    ("ring_k2", lambda R: P.ring_allreduce(R, rings=2)),
     ("allpairs", lambda R: P.allpairs_allreduce(R)),
     ("oneshot", lambda R: P.oneshot_allreduce(R)),
 ]
@@ -117,13 +119,15 @@ def test_alltonext_definition(N, G):
         assert _eq(out[q], ref[q])
 
 
-def _ring_closed_form(xs, dtype, E):
-    """chunk c = x_c + (x_{c-1} + (... + (x_{c+2} + x_{c+1}))) per element."""
+def _ring_closed_form(xs, dtype, E, K=1):
+    """chunk c = x_c + (x_{c-1} + (... + (x_{c+2} + x_{c+1}))) per element (SURVEY §4.2);
+    with K logical rings over K*R chunks, chunk c starts on rank (c mod R) + 1 (Fig. 3b with
+    offset (c div R)*R)."""
     R = len(xs)
     ts = [_t(x, dtype) for x in xs]
     n = ts[0].numel()
     out = torch.empty_like(ts[0])
-    for c in range(R):
+    for c in range(K * R):
         lo, hi = c * E, min((c + 1) * E, n)
         if lo >= hi:
             continue
@@ -142,8 +146,25 @@ def test_ring_matches_closed_form_bitwise(R, dtype):
     V = 16 // nm.elem_bytes(dtype)
     E = -(-(-(-n // R)) // V) * V
     want = _ring_closed_form(xs, dtype, E)
-    for algo in (P.ring_allreduce(R), P.ring_allreduce(R, inplace=True)):
+    for algo in (P.ring_allreduce(R), P.ring_allreduce(R, inplace=True),
+                 P.ring_allreduce(R, channels=R, split_phases=True)):  # R26: same chunk paths
         out = sim.simulate(_parse(algo), xs, n, dtype, "sum")
+        for o in out:
+            assert _eq(o, want)
+
+
+@pytest.mark.parametrize("R", [2, 4, 8])
+@pytest.mark.parametrize("K", [2, 3])
+def test_k_rings_match_closed_form_bitwise(R, K):
+    """R27: K logical rings over K*R chunks; chunk geometry per reading R1 with K*R chunks."""
+    n = 4096 + 40
+    dtype = "bfloat16"
+    xs = synth.inputs(R, n, dtype, "uniform")
+    V = 16 // nm.elem_bytes(dtype)
+    E = -(-(-(-n // (K * R))) // V) * V
+    want = _ring_closed_form(xs, dtype, E, K)
+    for algo in (P.ring_allreduce(R, rings=K), P.ring_allreduce(R, rings=K, inplace=True)):
+        out = sim.simulate(_parse(algo), xs, n, dtype, "sum", slots=8)
         for o in out:
             assert _eq(o, want)
 
