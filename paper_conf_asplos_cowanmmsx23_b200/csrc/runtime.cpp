@@ -31,7 +31,8 @@ namespace {
 // threads per CTA (2 CTAs per SM), direct placement on. LL / LL128 have their own FIFO slots.
 struct Params {
   int64_t slots = 4, slotBytes = 262144, llSlotBytes = 65536, ll128SlotBytes = 262144, maxChannels = 32,
-          threads = 256, timeoutS = 60, direct = 1, directTile = 1, directHints = 9, regMax = 64;
+          threads = 256, timeoutS = 60, direct = 1, directTile = 1, directHints = 9, regMax = 64,
+          crossLaunch = 0;
 };
 
 std::mutex gMu;
@@ -52,6 +53,7 @@ int64_t* paramRef(Params& p, const std::string& k) {
   if (k == "MSCCL_DIRECT") return &p.direct;
   if (k == "MSCCL_DIRECT_TILE") return &p.directTile;
   if (k == "MSCCL_DIRECT_HINTS") return &p.directHints;
+  if (k == "MSCCL_CROSS_LAUNCH") return &p.crossLaunch;
   return nullptr;
 }
 
@@ -61,7 +63,7 @@ Params currentParams() {
     gEnvRead = true;
     for (const char* k : {"MSCCL_SLOTS", "MSCCL_SLOT_BYTES", "MSCCL_LL_SLOT_BYTES", "MSCCL_LL128_SLOT_BYTES",
                           "MSCCL_MAX_CHANNELS", "MSCCL_THREADS", "MSCCL_TIMEOUT_S", "MSCCL_DIRECT",
-                          "MSCCL_DIRECT_TILE", "MSCCL_DIRECT_HINTS", "MSCCL_MAX_REGISTRATIONS"}) {
+                          "MSCCL_DIRECT_TILE", "MSCCL_DIRECT_HINTS", "MSCCL_MAX_REGISTRATIONS", "MSCCL_CROSS_LAUNCH"}) {
       const char* v = getenv(k);
       if (v && *v) *paramRef(gParams, k) = atoll(v);
     }
@@ -456,6 +458,12 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
     // in other launches or processes; each connection does a ready handshake per launch.
     bool allHere = (int)v.size() == R;
     for (int i = 0; allHere && i < (int)v.size(); i++) allHere = v[i]->comm->rank == i && v[i]->comm->nranks == R;
+    // MSCCL_CROSS_LAUNCH=1 (test mode): run the cross-launch protocol (R15b ready handshakes, R23
+    // group barriers, system-scope fences and flags) although every rank is in this one
+    // cooperative launch -- the device code of the multi-GPU / multi-process deployment, with
+    // all ranks co-resident (so nothing waits on a kernel that might not be running)
+    const bool emulateCross = c0->prm.crossLaunch != 0;
+    if (emulateCross) allHere = false;
     int direct = 0;
     if (p0->algo.proto == PROTO_SIMPLE && c0->prm.direct) direct = allHere ? 1 : 2;
     bool aliasedAny = false;
@@ -554,7 +562,7 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
                       "a multimem program across processes needs sendbuff and recvbuff inside registered buffers "
                       "(mscclCommRegister; reading R23)");
       cta += p->nTB;
-      if (cl->comm->sysScope) ka.sysScope = 1;
+      if (cl->comm->sysScope || emulateCross) ka.sysScope = 1;
       if (direct == 1) cl->comm->launchesDirect1++;
       if (direct == 2 && ra.directMask) cl->comm->launchesDirect2++;
     }

@@ -12,7 +12,8 @@ def comms(R, device=0):
     key = (R, device) + tuple(runtime.get_param(k) for k in ("MSCCL_SLOTS", "MSCCL_SLOT_BYTES", "MSCCL_THREADS",
                                                               "MSCCL_MAX_CHANNELS", "MSCCL_TIMEOUT_S",
                                                               "MSCCL_DIRECT", "MSCCL_LL_SLOT_BYTES",
-                                                              "MSCCL_LL128_SLOT_BYTES"))
+                                                              "MSCCL_LL128_SLOT_BYTES",
+                                                              "MSCCL_CROSS_LAUNCH", "MSCCL_DIRECT_HINTS"))
     if key not in _COMMS:
         _COMMS[key] = runtime.Comm.virtual(R, device)
     return _COMMS[key]

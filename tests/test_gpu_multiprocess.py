@@ -18,7 +18,16 @@ import numpy as np
 import pytest
 import torch.multiprocessing as mp
 
-pytestmark = pytest.mark.gpu
+# Ranks that wait on one another, run as separate processes time-slicing one GPU, can raise
+# Xid 109 (context-switch timeout) on this driver (B200_PROFILING.md). They ran green in
+# this round's explicit runs (profiles/r02/gpu_tests_final.log); the default GPU suite covers
+# the same cross-launch device code with every rank co-resident in one launch instead
+# (tests/test_gpu_cross_launch.py). Set MSCCL_MULTIPROC_GPU=1 to run these on a GPU box
+# where that is safe (one GPU per process, or a single-GPU box you accept the risk on).
+pytestmark = [pytest.mark.gpu,
+              pytest.mark.skipif(os.environ.get("MSCCL_MULTIPROC_GPU") != "1",
+                                 reason="separate processes spinning on one GPU (Xid 109 risk); "
+                                        "set MSCCL_MULTIPROC_GPU=1; covered by test_gpu_cross_launch.py")]
 
 
 def _free_port():
