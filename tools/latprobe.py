@@ -70,6 +70,7 @@ def main():
     ap.add_argument("--proto", default="LL")
     ap.add_argument("--iters", type=int, default=200)
     ap.add_argument("--ranks", type=int, default=8)
+    ap.add_argument("--n", type=int, default=512, help="fp16 elements per rank (512 = 1 KiB)")
     args = ap.parse_args()
     import torch
     import bench
@@ -81,7 +82,7 @@ def main():
     comms = rt.Comm.virtual(W, 0)
     R = bench.Ranks(rt, comms, list(range(W)), W, 1, dev)
     stream = torch.cuda.current_stream()
-    n = 512
+    n = args.n
     send = [synth.hashed(q, torch.arange(n, device=dev), "float16") for q in range(W)]
     recv = [torch.empty_like(x) for x in send]
     probes = [("nop", bench.nop_ir(W)), ("hop", bench.hop_ir(W, args.proto)),
