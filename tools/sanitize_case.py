@@ -1,5 +1,6 @@
-"""Small cases for compute-sanitizer (memcheck / synccheck): every protocol, direct on/off, multimem
-programs, ragged sizes."""
+"""Small cases for compute-sanitizer (memcheck / synccheck): every protocol, direct on/off, the
+cross-launch protocol in one launch (MSCCL_CROSS_LAUNCH, reading R28), multimem programs, the
+split-phase and K-ring schedules, ragged sizes."""
 import os, sys
 sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 sys.path.insert(0, os.path.join(os.path.dirname(os.path.dirname(os.path.abspath(__file__))), "tests"))
@@ -12,10 +13,14 @@ runtime.set_param("MSCCL_SLOT_BYTES", 16384)
 runtime.set_param("MSCCL_THREADS", 128)
 import gpu_util
 bad = 0
-for direct in (1, 0):
+for cross, direct in ((0, 1), (0, 0), (1, 1)):
     runtime.set_param("MSCCL_DIRECT", direct)
+    runtime.set_param("MSCCL_CROSS_LAUNCH", cross)
+    direct = "%d%s" % (direct, "x" if cross else "")
     for name, algo, R, n, dt in [("ring", P.ring_allreduce(4, instances=2), 4, 20011, "bfloat16"),
                                  ("ring_LL", P.ring_allreduce(4, protocol="LL"), 4, 5001, "float32"),
+                                 ("ring_split", P.ring_allreduce(4, channels=4, split_phases=True), 4, 9001, "bfloat16"),
+                                 ("ring_k2", P.ring_allreduce(4, rings=2), 4, 9001, "float16"),
                                  ("ring_LL128", P.ring_allreduce(4, protocol="LL128"), 4, 5001, "float16"),
                                  ("allpairs", P.allpairs_allreduce(4, protocol="Simple"), 4, 3003, "float32"),
                                  ("oneshot", P.oneshot_allreduce(4), 4, 777, "int32"),
