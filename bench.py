@@ -58,7 +58,8 @@ def parse():
     ap.add_argument("--ranks", type=int, default=8, help="virtual ranks when N=1")
     ap.add_argument("--size-mib", type=float, default=256.0, help="bytes per rank (MiB)")
     ap.add_argument("--program", default="ring",
-                    choices=["ring", "allpairs", "oneshot", "alltoall", "allgather", "reducescatter", "nvls"])
+                    choices=["ring", "allpairs", "oneshot", "alltoall", "allgather", "allgather_direct", "reducescatter",
+                             "nvls"])
     ap.add_argument("--channels", type=int, default=1)
     ap.add_argument("--split", action="store_true", help="ring: AllGather half on its own channels (reading R26)")
     ap.add_argument("--rings", type=int, default=1, help="ring: K interleaved logical rings per thread block (R27)")
@@ -180,13 +181,16 @@ def build_program(args, R):
         return P.nvls_allreduce(R, args.instances)
     if args.program == "allgather":
         return P.ring_allgather(R, args.channels, args.instances, protocol=args.protocol)
+    if args.program == "allgather_direct":
+        return P.allpairs_allgather(R, args.instances, protocol=args.protocol)
     if args.program == "reducescatter":
         return P.ring_reducescatter(R, args.channels, args.instances, protocol=args.protocol)
     return P.alltoall_twostep(1, R, instances=args.instances, protocol=args.protocol)
 
 
 def coll_of(program):
-    return {"alltoall": "alltoall", "allgather": "allgather", "reducescatter": "reducescatter"}.get(program,
+    return {"alltoall": "alltoall", "allgather": "allgather", "allgather_direct": "allgather",
+            "reducescatter": "reducescatter"}.get(program,
                                                                                                   "allreduce")
 
 
@@ -311,6 +315,7 @@ def config_dict(args, R, N):
                 "oneshot": "BASELINE configs[2] shape (one-shot AllReduce)",
                 "alltoall": "BASELINE configs[3] shape (AllToAll)",
                 "allgather": "BASELINE configs[4] shape (ring AllGather)",
+                "allgather_direct": "BASELINE configs[4] shape (all-pairs AllGather)",
                 "nvls": "BASELINE configs[1] shape with the multimem (NVLS) AllReduce program",
                 "reducescatter": "BASELINE configs[4] shape (ring ReduceScatter)"}[args.program]
         mode = "%d virtual ranks on 1 B200 (HBM-bound)" % R
@@ -318,7 +323,8 @@ def config_dict(args, R, N):
         base = {"ring": "BASELINE configs[1]: ring AllReduce, bf16", "allpairs": "all-pairs AllReduce",
                 "oneshot": "one-shot AllReduce", "alltoall": "BASELINE configs[3]: AllToAll",
                 "nvls": "multimem (NVLS) AllReduce",
-                "allgather": "BASELINE configs[4]: ring AllGather", "reducescatter": "BASELINE configs[4]: ring "
+                "allgather": "BASELINE configs[4]: ring AllGather",
+                "allgather_direct": "BASELINE configs[4]: all-pairs AllGather", "reducescatter": "BASELINE configs[4]: ring "
                 "ReduceScatter"}[args.program]
         mode = "%d B200, 1 process per GPU, CUDA IPC over NVLink" % N
     return {"workload": "%s -- MSCCL-IR %s, %d channel(s) x %d instance(s), %s protocol, %s, %d MiB per rank"

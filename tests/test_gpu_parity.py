@@ -115,6 +115,10 @@ def test_allgather_reducescatter(R, r):
     got = _gpu().run_program(P.ring_allgather(R, 2, r).to_xml(), xs, n, "int32", out_elems=R * n)
     for g, e in zip(got, mpi_ref.allgather(xs)):
         assert _bits_equal(g, e)
+    if R * 2 * (R - 1) * r <= 296:  # all-pairs: 2(R-1) thread blocks per rank and instance, co-resident
+        got = _gpu().run_program(P.allpairs_allgather(R, r).to_xml(), xs, n, "int32", out_elems=R * n)
+        for g, e in zip(got, mpi_ref.allgather(xs)):
+            assert _bits_equal(g, e)
     xs = synth.inputs(R, R * n, "bfloat16", "uniform")
     ir = P.ring_reducescatter(R, 2, r).to_xml()
     want = sim.simulate(irparse.parse(ir), xs, n, "bfloat16", "sum")

@@ -38,6 +38,7 @@ SHIPPED = {
     "allpairs": lambda R, r: P.allpairs_allreduce(R, instances=r, protocol="Simple"),
     "oneshot": lambda R, r: P.oneshot_allreduce(R, instances=r, protocol="Simple"),
     "allgather": lambda R, r: P.ring_allgather(R, 1, r),
+    "allgather_allpairs": lambda R, r: P.allpairs_allgather(R, r),
     "reducescatter": lambda R, r: P.ring_reducescatter(R, 1, r),
     "alltoall": lambda R, r: P.alltoall_twostep(1, R, r),
 }

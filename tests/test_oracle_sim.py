@@ -91,6 +91,8 @@ def test_allgather_reducescatter_equal_brute_force(R, r):
     xs = synth.inputs(R, n, "int32", "pattern")
     out = sim.simulate(_parse(P.ring_allgather(R, 2, r)), xs, n, "int32")
     assert all(_eq(o, e) for o, e in zip(out, mpi_ref.allgather(xs)))
+    out = sim.simulate(_parse(P.allpairs_allgather(R, r)), xs, n, "int32")
+    assert all(_eq(o, e) for o, e in zip(out, mpi_ref.allgather(xs)))
     xs = _exact_inputs(R, R * n, "bfloat16", "sum")
     out = sim.simulate(_parse(P.ring_reducescatter(R, 2, r)), xs, n, "bfloat16", "sum")
     ref = mpi_ref.reducescatter(xs, n, "sum", "bfloat16")
