@@ -287,7 +287,7 @@ def run_reference(args):
     t = (time.perf_counter() - t0) / args.steps
     v = busbw("allreduce", sample, t, R)
     cfg = config_dict(args, R, args.gpus)
-    out = {"impl": "reference", "metric": metric_name(), "value": round(v, 4), "unit": "GB/s",
+    out = {"impl": "reference", "metric": metric_name(coll_of(args.program), args.program), "value": round(v, 4), "unit": "GB/s",
            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 3),
            "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16", "data": "synthetic",
            "config": cfg,
@@ -300,12 +300,15 @@ def run_reference(args):
     print(json.dumps(out), flush=True)
 
 
-def metric_name(coll="allreduce"):
+def metric_name(coll="allreduce", program="ring"):
+    form = {"ring": "ring", "allpairs": "all-pairs", "oneshot": "one-shot", "nvls": "multimem (NVLS)",
+            "allgather": "ring", "allgather_direct": "all-pairs", "reducescatter": "ring"}.get(program, program)
     if coll == "alltoall":
         return "AllToAll busBW (GB/s), direct MSCCL-IR (two-step N=1), bf16"
     if coll in ("allgather", "reducescatter"):
-        return "%s busBW (GB/s), ring MSCCL-IR, bf16" % {"allgather": "AllGather", "reducescatter": "ReduceScatter"}[coll]
-    return "AllReduce busBW (GB/s), ring MSCCL-IR, bf16"
+        return "%s busBW (GB/s), %s MSCCL-IR, bf16" % ({"allgather": "AllGather", "reducescatter": "ReduceScatter"}[coll],
+                                                      form)
+    return "AllReduce busBW (GB/s), %s MSCCL-IR, bf16" % form
 
 
 def config_dict(args, R, N):
@@ -998,7 +1001,7 @@ def main():
     value = busbw(coll, S, t, R)
     launches_per_step = max(1, res["launches"] // args.steps)
     out = {
-        "metric": metric_name(coll), "value": round(value, 3), "unit": "GB/s", "n_gpus": N,
+        "metric": metric_name(coll, args.program), "value": round(value, 3), "unit": "GB/s", "n_gpus": N,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(t * 1e3, 4),
         "higher_is_better": True, "scaling": "weak", "vs_baseline": None, "dtype": "bf16",
         "data": "synthetic (counter-based uniform[-1,1) bf16, seed 20230325+rank)",
