@@ -330,7 +330,11 @@ __device__ __forceinline__ void chunkSpan(const KernelArgs& a, int buf, int64_t 
     len = a.E;
     return;
   }
-  int64_t b = k / a.cb, j = k - b * a.cb;
+  // chunk indices and chunks-per-block fit in 32 bits: a 32-bit division (a few instructions)
+  // instead of the 64-bit division subroutine (hundreds of cycles on the latency path)
+  const uint32_t kk = (uint32_t)k, cb = (uint32_t)a.cb;
+  const uint32_t bq = kk / cb;
+  int64_t b = (int64_t)bq, j = (int64_t)(kk - bq * cb);
   start = b * a.n + j * a.E;
   int64_t rem = a.n - j * a.E;
   len = rem < 0 ? 0 : (rem < a.E ? rem : a.E);
@@ -823,6 +827,12 @@ __device__ __noinline__ bool movePiecesLL128(const Ctx& c, const DevInstr& in, i
   return ok;
 }
 
+// FIFO slot of message number x (monotone 64-bit counter): a mask for power-of-two slot counts
+// (the default 4), the 64-bit remainder otherwise
+__device__ __forceinline__ uint32_t slotOf(uint64_t x, uint32_t s) {
+  return (s & (s - 1)) == 0 ? (uint32_t)x & (s - 1) : (uint32_t)(x % s);
+}
+
 // ------------------------------------------------------------------ one instruction, one tile
 template <int DT, int OP, int PROTO, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
 __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr& in, int t, uint64_t& sent,
@@ -874,8 +884,8 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
 #if MSCCL_TRACE
   if (c.tid == 0) tr2 = globaltimer();
 #endif
-  const char* rslot = RECV ? tb.recvFifo + (int64_t)(recvd % (uint64_t)a.slots) * a.slotBytes : nullptr;
-  char* sslot = SEND ? tb.sendFifo + (int64_t)(sent % (uint64_t)a.slots) * a.slotBytes : nullptr;
+  const char* rslot = RECV ? tb.recvFifo + (int64_t)slotOf(recvd, (uint32_t)a.slots) * a.slotBytes : nullptr;
+  char* sslot = SEND ? tb.sendFifo + (int64_t)slotOf(sent, (uint32_t)a.slots) * a.slotBytes : nullptr;
   // each protocol's data path is its own non-inlined function (separate register allocation)
   if constexpr (!ll || (!RECV && !SEND)) {
     movePiecesSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(c, tb, in, t, rslot, sslot);
@@ -1256,6 +1266,9 @@ __device__ __noinline__ void chainExec(const Ctx& c, const DevInstr* mem, int L,
   const int64_t w = sizeof(T);
   const int64_t a0 = (int64_t)t * a.T;
   const bool headCopy = mem[0].op == K_COPY;
+#if MSCCL_TRACE
+  uint64_t ct0 = c.tid == 0 ? globaltimer() : 0, ct1 = 0, ct2 = 0;
+#endif
   for (int j = 0; j < mem[0].cnt; j++) {
     if (c.tid < L) {
       const int k = c.tid;
@@ -1271,6 +1284,9 @@ __device__ __noinline__ void chainExec(const Ctx& c, const DevInstr* mem, int L,
       }
     }
     __syncthreads();
+#if MSCCL_TRACE
+    if (c.tid == 0) ct1 = globaltimer();
+#endif
     const int64_t m = cs.m[0];
     bool same = true;
     uintptr_t al = (uintptr_t)cs.dst;
@@ -1318,8 +1334,21 @@ __device__ __noinline__ void chainExec(const Ctx& c, const DevInstr* mem, int L,
         *(T*)(dst + e * w) = acc;
       }
     }
+#if MSCCL_TRACE
+    if (c.tid == 0) ct2 = globaltimer();
+#endif
     __syncthreads();  // the operand table is rewritten for the next piece
   }
+#if MSCCL_TRACE
+  if (c.tid == 0 && a.trace) {  // chain phases: operand table, data (thread 0), barrier
+    uint64_t* tr = a.trace + (size_t)blockIdx.x * 8;
+    const uint64_t ct3 = globaltimer();
+    tr[0] += ct1 - ct0;
+    tr[1] += ct2 - ct1;
+    tr[2] += ct3 - ct2;
+    tr[7] += 1;
+  }
+#endif
 }
 
 // Simple-protocol kernels: the chain pass of reading R16 with its operand table in registers

@@ -156,3 +156,20 @@ def test_repeated_launches_keep_counters_consistent():
     for _ in range(3):
         got = _gpu().run_program(ir, xs, n, "float32")
         assert all(_bits_equal(g, w) for g, w in zip(got, want))
+
+
+@pytest.mark.parametrize("slots", [2, 3, 5, 8])
+@pytest.mark.parametrize("proto", ["Simple", "LL", "LL128"])
+def test_slot_counts(slots, proto):
+    """FIFO slot index of message k is k mod s (§6.1): power-of-two slot counts
+    take a mask, others the remainder; every protocol, many tiles (wrap-around many times)."""
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    runtime.set_param("MSCCL_SLOTS", slots)
+    try:
+        n = 3 * 8192 * 4 + 37
+        _check_allreduce(P.ring_allreduce(4, protocol=proto).to_xml(), 4, n, "bfloat16", "sum")
+        if slots >= 3:  # two interleaved rings need s >= 3 (reading R27, V9)
+            _check_allreduce(P.ring_allreduce(4, instances=2, rings=2, protocol=proto).to_xml(), 4, n, "float32",
+                             "sum")
+    finally:
+        runtime.set_param("MSCCL_SLOTS", 4)

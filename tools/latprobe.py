@@ -50,16 +50,21 @@ def scatter_ir(R, proto, with_dep):
     return _algo("scatter", R, proto, gpus)
 
 
-def fold_ir(R, proto, members=None):
+def fold_ir(R, proto, members=None, repeat=1):
     """one block per rank: cpy in -> out, then `members`-1 reduces of scratch chunks into out
-    (a fused chain, reading R16); members = R is the one-shot fold"""
+    (a fused chain, reading R16); members = R is the one-shot fold; `repeat` runs the same
+    chain again in the same block (warm instruction cache, same data)"""
     members = R if members is None else members
     gpus = []
     for q in range(R):
-        steps = [_step(0, "cpy", "i", 0, "o", 0)]
-        for p in range(R):
-            if p != q and len(steps) < members:
-                steps.append(_step(len(steps), "re", "s", p, "o", 0))
+        steps = []
+        for _ in range(repeat):
+            steps.append(_step(len(steps), "cpy", "i", 0, "o", 0))
+            k = 1
+            for p in range(R):
+                if p != q and k < members:
+                    steps.append(_step(len(steps), "re", "s", p, "o", 0))
+                    k += 1
         gpus.append('<gpu id="%d" i_chunks="1" o_chunks="1" s_chunks="%d"><tb id="0" send="-1" recv="-1" chan="0">'
                     '%s</tb></gpu>' % (q, R, "".join(steps)))
     return _algo("fold", R, proto, gpus)
@@ -89,6 +94,8 @@ def main():
               ("scatter", scatter_ir(W, args.proto, False)), ("scatter+d", scatter_ir(W, args.proto, True)),
               ("copy", fold_ir(W, args.proto, 1)), ("fold2", fold_ir(W, args.proto, 2)),
               ("fold4", fold_ir(W, args.proto, 4)), ("fold", fold_ir(W, args.proto)),
+              ("copy_x2", fold_ir(W, args.proto, 1, 2)), ("fold_x2", fold_ir(W, args.proto, None, 2)),
+              ("fold_x4", fold_ir(W, args.proto, None, 4)),
               ("oneshot", P.oneshot_allreduce(W, protocol=args.proto).to_xml()),
               ("nvls", P.nvls_allreduce(W, 1).to_xml())]
     out = {"proto": args.proto, "ranks": W, "bytes": 2 * n, "mode": None}
