@@ -49,7 +49,7 @@ struct DevTB {
   uint64_t* sendHead;         // peer: messages posted by me
   uint64_t* sendAck;          // mine: messages the peer consumed (written by the peer)
   uint64_t* sendCnt;          // mine: [0] messages I posted, [1] launches on this connection
-  uint64_t* sendReady;        // mine: [0] receiver's launch ordinal, [1..3] its in/out/sc refs
+  uint64_t* sendReady;        // mine: [0] receiver's launch ordinal, [1..3] its in/out/sc refs, [4] its tile T
   // receive connection (peer = sender)
   char* recvFifo;             // my FIFO base for (peer -> me, chan)
   uint64_t* recvHead;         // mine: messages the peer posted (written by the peer)
@@ -119,7 +119,7 @@ struct KernelArgs {
   // ranks' buffer references at the start and completion at the end)
   int32_t mm;
   int32_t mmVec32;            // multimem: every chunk / tile span is 32-byte aligned (32-byte vectors)
-  int32_t pad1;
+  int32_t tileIsChunk;        // reading R19: T = E, every message a direct placement (no FIFO slot)
   int64_t mmLineOff;          // offset of the group-barrier lines in every region
   uint64_t timeoutNs;         // device watchdog; 0 = disabled
   uint64_t* trace;            // MSCCL_TRACE builds: per-CTA phase times (ns), else null

@@ -736,6 +736,10 @@ __device__ __forceinline__ char* resolveRef(const RankArgs& ra, int peer, uint64
 __device__ __forceinline__ bool waitReady(const Ctx& c, const DevTB& tb) {
   uint64_t seen;
   if (!waitGE(tb.sendReady, c.sendL, c.a->sysScope != 0, c, seen)) return false;
+  if (*(volatile const uint64_t*)(tb.sendReady + 4) != (uint64_t)c.a->T) {  // ranks chose different tiles
+    raiseAbort(*c.a);                                                        // (asymmetric registration, R19)
+    return false;
+  }
   bool any = false;
 #pragma unroll
   for (int b = 0; b < 3; b++) {
@@ -1507,7 +1511,8 @@ __global__ void __launch_bounds__(MSCCL_MAX_THREADS, MSCCL_MIN_BLOCKS) mscclInte
     const uint64_t L = *(volatile uint64_t*)(tb.recvCnt + 1) + 1;
     *(volatile uint64_t*)(tb.recvCnt + 1) = L;
     if (a.direct == 2) {
-      for (int b = 0; b < 3; b++) postFlag(tb.recvReady + 1 + b, ra.bufRef[b], a.sysScope != 0);
+      for (int b = 0; b < 4; b++)  // in / out / scratch refs, then the tile size (R19 check)
+        postFlag(tb.recvReady + 1 + b, b < 3 ? ra.bufRef[b] : (uint64_t)a.T, a.sysScope != 0);
       if (a.sysScope) fenceSys();
       else fenceGpu();
       postFlag(tb.recvReady, L, a.sysScope != 0);

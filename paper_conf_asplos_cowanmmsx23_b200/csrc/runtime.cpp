@@ -478,8 +478,24 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
     // what it receives (ring AllGather: rcs reads the chunk its predecessor just stored): then
     // the slot-sized tile bounds the data in flight so the forwarded tile is still in L2 when
     // it is read (measured: ring AllGather 337 -> 389 GB/s busBW on 8 virtual ranks)
-    bool noFifo = direct == 1 && c0->prm.directTile;
+    bool noFifo = (direct == 1 || direct == 2) && c0->prm.directTile;
     for (auto* cl : v) noFifo = noFifo && cl->prog->allDirect && !cl->prog->forwards;
+    // Cross-launch (R15b): whether a message is direct is settled per connection at the ready
+    // handshake, so one tile per chunk also needs every destination of this rank reachable by
+    // its senders (user buffers inside registrations, or raw pointers in one process; the
+    // library's scratch only in one process). Ranks decide from their own buffers; the
+    // receiver publishes its tile size on the ready line and a sender whose tile differs (a rank
+    // registered differently) raises the watchdog abort instead of storing past a FIFO slot.
+    if (noFifo && direct == 2) {
+      for (auto* cl : v) {
+        const int Rr = cl->comm->nranks, w = elemBytes(cl->dtype);
+        const size_t inB = (size_t)cl->n * blocksOf(cl->prog->algo.coll, BUF_IN, Rr) * w;
+        const size_t outB = (size_t)cl->n * blocksOf(cl->prog->algo.coll, BUF_OUT, Rr) * w;
+        const bool sc = cl->prog->algo.gpus[cl->comm->rank].sChunks > 0;
+        noFifo = noFifo && !cl->aliased && bufferRef(cl->comm, cl->buf[0], inB) && bufferRef(cl->comm, cl->buf[1], outB) &&
+                 (!sc || cl->comm->clique);
+      }
+    }
     Geometry g{};
     mscclResult_t r = geometry(c0, p0, v[0]->dtype, v[0]->n, g, noFifo);
     if (r != mscclSuccess) return r;
@@ -497,6 +513,7 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
     ka.timeoutNs = c0->prm.timeoutS > 0 ? (uint64_t)c0->prm.timeoutS * 1000000000ull : 0;  // <= 0: no watchdog
     ka.trace = traceBuffer();
     ka.direct = direct;
+    ka.tileIsChunk = noFifo ? 1 : 0;
     ka.directHints = (int32_t)c0->prm.directHints;
     ka.mm = mm;
     ka.mmLineOff = (int64_t)c0->mmLineOff();
