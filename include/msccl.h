@@ -122,7 +122,12 @@ mscclResult_t mscclCommGetAsyncError(mscclComm_t comm, mscclResult_t* asyncError
  *                                               maps every peer's range; all ranks must
  *                                               return from it before any uses the buffer
  * A call whose recvbuff (or sendbuff, for in-place programs) is not inside a connected
- * registration simply uses the FIFO for messages to this rank. Registration allocates and
+ * registration simply uses the FIFO for messages to this rank. Exception (reading R19b): a
+ * program whose every message is a direct placement and that forwards nothing (e.g. the
+ * direct AllToAll) moves each chunk as ONE message when this rank's sendbuff and recvbuff are
+ * both registered; every rank must then have registered its buffers for the call, otherwise
+ * the ranks disagree on the message size and the launch ends in mscclRemoteError (checked on
+ * the per-launch ready line), never in a store past a FIFO slot. Registration allocates and
  * synchronises (not capturable). mscclCommDeregister unmaps (collective, after the stream
  * work that used the buffer has completed). Errors: InvalidArgument (null, size 0, range
  * not inside one device allocation, more than MSCCL_MAX_REGISTRATIONS), UnhandledCudaError. */
