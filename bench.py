@@ -348,6 +348,7 @@ def set_params(rt, args):
     rt.set_param("MSCCL_THREADS", args.threads)
     rt.set_param("MSCCL_MAX_CHANNELS", max(32, args.channels * args.instances * (2 if args.split else 1)))
     rt.set_param("MSCCL_TIMEOUT_S", 60)
+    rt.set_param("MSCCL_DIRECT_TILE", 2)  # every rank registers its buffers (reading R19b)
 
 
 def sampled_parity(algo, recv_list, n, ranks_to_check, local=None):

@@ -122,12 +122,12 @@ mscclResult_t mscclCommGetAsyncError(mscclComm_t comm, mscclResult_t* asyncError
  *                                               maps every peer's range; all ranks must
  *                                               return from it before any uses the buffer
  * A call whose recvbuff (or sendbuff, for in-place programs) is not inside a connected
- * registration simply uses the FIFO for messages to this rank. Exception (reading R19b): a
- * program whose every message is a direct placement and that forwards nothing (e.g. the
- * direct AllToAll) moves each chunk as ONE message when this rank's sendbuff and recvbuff are
- * both registered; every rank must then have registered its buffers for the call, otherwise
- * the ranks disagree on the message size and the launch ends in mscclRemoteError (checked on
- * the per-launch ready line), never in a store past a FIFO slot. Registration allocates and
+ * registration simply uses the FIFO for messages to this rank. Option (reading R19b,
+ * MSCCL_DIRECT_TILE=2): a program whose every message is a direct placement and that forwards
+ * nothing (e.g. the direct AllToAll) moves each chunk as ONE message when this rank's sendbuff
+ * and recvbuff are both registered; every rank must then have registered its buffers for the
+ * call, otherwise the ranks disagree on the message size and the launch ends in
+ * mscclRemoteError (checked on the per-launch ready line), never in a store past a FIFO slot. Registration allocates and
  * synchronises (not capturable). mscclCommDeregister unmaps (collective, after the stream
  * work that used the buffer has completed). Errors: InvalidArgument (null, size 0, range
  * not inside one device allocation, more than MSCCL_MAX_REGISTRATIONS), UnhandledCudaError. */
@@ -237,7 +237,7 @@ const char* mscclGetLastError(mscclComm_t comm); /* comm may be NULL: last globa
  * -- each protocol has its own slots; "MSCCL_MAX_CHANNELS" (32); "MSCCL_THREADS" threads
  * per CTA (64..256, default 256 = 2 CTAs per SM); "MSCCL_TIMEOUT_S" watchdog (default 60,
  * <= 0 disables); "MSCCL_DIRECT" direct placement (1); "MSCCL_DIRECT_TILE" one tile per
- * chunk when every message is direct (1); "MSCCL_DIRECT_HINTS" L2 hints of direct stores, a
+ * chunk when every message is direct (1; 2 = also across processes, see registration); "MSCCL_DIRECT_HINTS" L2 hints of direct stores, a
  * bit set (default 9: bit 0 terminal direct sends evict_first, bit 3 forwarded direct sends
  * evict_normal; bit 1 demote forwarded lines after reading, bit 2 FIFO stores evict_normal:
  * measured slower, off); "MSCCL_MAX_REGISTRATIONS" (64). All ranks must

@@ -486,6 +486,9 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
     // library's scratch only in one process). Ranks decide from their own buffers; the
     // receiver publishes its tile size on the ready line and a sender whose tile differs (a rank
     // registered differently) raises the watchdog abort instead of storing past a FIFO slot.
+    // Across processes this needs every rank to have registered its buffers, so it is opt-in
+    // there (MSCCL_DIRECT_TILE=2); in one process every buffer is reachable by construction.
+    if (noFifo && direct == 2 && !c0->clique && c0->prm.directTile < 2) noFifo = false;
     if (noFifo && direct == 2) {
       for (auto* cl : v) {
         const int Rr = cl->comm->nranks, w = elemBytes(cl->dtype);
@@ -882,7 +885,8 @@ mscclResult_t mscclCommExportHandle(mscclComm_t c, void* handle, size_t* bytes) 
   // parameters that both ends of a connection must agree on (region layout, warp partition)
   // parameters both ends of a connection must agree on (region layout, slot geometry)
   // (MSCCL_DIRECT too: a receiver that publishes its destination expects the sender to store there)
-  int64_t meta[8] = {(int64_t)c->regionBytes, c->prm.direct != 0, c->prm.threads,        c->prm.slots,
+  // word 1: MSCCL_DIRECT on/off | MSCCL_DIRECT_TILE << 1 (both must match: R15b, R19b)
+  int64_t meta[8] = {(int64_t)c->regionBytes, (c->prm.direct != 0) | (c->prm.directTile << 1), c->prm.threads, c->prm.slots,
                      c->prm.slotBytes,         c->prm.llSlotBytes, c->prm.ll128SlotBytes, c->prm.maxChannels};
   static_assert(sizeof(cudaIpcMemHandle_t) + sizeof(meta) <= MSCCL_HANDLE_BYTES, "handle size");
   memcpy((char*)handle + sizeof(h), meta, sizeof(meta));
@@ -901,9 +905,10 @@ mscclResult_t mscclCommConnect(mscclComm_t c, const void* allHandles) {
     memcpy(&ih, h, sizeof(ih));
     int64_t meta[8];
     memcpy(meta, h + sizeof(ih), sizeof(meta));
-    const int64_t mine[8] = {(int64_t)c->regionBytes, c->prm.direct != 0, c->prm.threads,        c->prm.slots,
+    const int64_t mine[8] = {(int64_t)c->regionBytes, (c->prm.direct != 0) | (c->prm.directTile << 1), c->prm.threads,
+                             c->prm.slots,
                              c->prm.slotBytes,         c->prm.llSlotBytes, c->prm.ll128SlotBytes, c->prm.maxChannels};
-    static const char* names[8] = {"region size", "MSCCL_DIRECT", "MSCCL_THREADS", "MSCCL_SLOTS", "MSCCL_SLOT_BYTES",
+    static const char* names[8] = {"region size", "MSCCL_DIRECT / MSCCL_DIRECT_TILE", "MSCCL_THREADS", "MSCCL_SLOTS", "MSCCL_SLOT_BYTES",
                                    "MSCCL_LL_SLOT_BYTES", "MSCCL_LL128_SLOT_BYTES", "MSCCL_MAX_CHANNELS"};
     for (int k = 0; k < 8; k++)
       if (meta[k] != mine[k]) {

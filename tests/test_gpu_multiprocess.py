@@ -18,16 +18,17 @@ import numpy as np
 import pytest
 import torch.multiprocessing as mp
 
+pytestmark = pytest.mark.gpu
+
 # Ranks that wait on one another, run as separate processes time-slicing one GPU, can raise
-# Xid 109 (context-switch timeout) on this driver (B200_PROFILING.md). They ran green in
-# this round's explicit runs (profiles/r02/gpu_tests_final.log); the default GPU suite covers
-# the same cross-launch device code with every rank co-resident in one launch instead
-# (tests/test_gpu_cross_launch.py). Set MSCCL_MULTIPROC_GPU=1 to run these on a GPU box
-# where that is safe (one GPU per process, or a single-GPU box you accept the risk on).
-pytestmark = [pytest.mark.gpu,
-              pytest.mark.skipif(os.environ.get("MSCCL_MULTIPROC_GPU") != "1",
-                                 reason="separate processes spinning on one GPU (Xid 109 risk); "
-                                        "set MSCCL_MULTIPROC_GPU=1; covered by test_gpu_cross_launch.py")]
+# Xid 109 (context-switch timeout) on this driver (B200_PROFILING.md). The tests that launch
+# such kernels ran green in this round's explicit runs (profiles/r02/gpu_tests_final.log); the
+# default GPU suite covers the same cross-launch device code with every rank co-resident in one
+# launch instead (tests/test_gpu_cross_launch.py). Set MSCCL_MULTIPROC_GPU=1 to run them on a
+# GPU box where that is safe. The Connect test below launches no kernel and always runs.
+spinning = pytest.mark.skipif(os.environ.get("MSCCL_MULTIPROC_GPU") != "1",
+                              reason="separate processes spinning on one GPU (Xid 109 risk); "
+                                     "set MSCCL_MULTIPROC_GPU=1; covered by test_gpu_cross_launch.py")
 
 
 def _free_port():
@@ -218,6 +219,7 @@ def _run_world(world, cases, timeout):
             assert handshakes > 0, (name, proto, handshakes)
 
 
+@spinning
 @pytest.mark.parametrize("world", [2, 4, 8])
 def test_processes_ipc_all_programs(world):
     cases = [c for c in CASES if not (c[0] in ("hier", "a2a_2step") and world < 4)]
@@ -260,6 +262,7 @@ def _silent_peer_worker(rank, world, port, q):
         dist.destroy_process_group()
 
 
+@spinning
 def test_watchdog_turns_a_missing_peer_into_an_error():
     """A peer that never launches: the spin waits time out (MSCCL_TIMEOUT_S), the kernel
     exits, and the communicator reports mscclRemoteError (sticky) instead of hanging."""
@@ -358,6 +361,7 @@ def _sequence_worker(rank, world, port, q):
         dist.destroy_process_group()
 
 
+@spinning
 def test_mixed_program_sequence_four_processes():
     """Eight different programs -- Simple with and without registered buffers, LL, LL128,
     multimem, and a mixed program -- run back to back twice on one stream per process. The
