@@ -1426,8 +1426,16 @@ __device__ __noinline__ void chainExecSimple(const Ctx& c, const DevInstr* mem, 
 #define MSCCL_SMEM_INSTR 64  // instructions per thread block staged in shared memory (LL / LL128)
 #endif
 
+// The LL / LL128 kernels are compiled for 1 CTA per SM: up to 255 registers, no spills (at 2 CTAs
+// per SM they spilled 124 bytes in the kernel body and 130-270 bytes in the LL128 data paths).
+// Latency programs use far fewer than 148 thread blocks; measured: 1 KiB one-shot LL 11.1 ->
+// 10.8 us, LL128 14.0 -> 13.2 us, LL128 ring 16 MiB 113 -> 123 GB/s.
+#ifndef MSCCL_LAT_MIN_BLOCKS
+#define MSCCL_LAT_MIN_BLOCKS 1
+#endif
 template <int DT, int OP, int PROTO, bool MM = false>
-__global__ void __launch_bounds__(MSCCL_MAX_THREADS, MSCCL_MIN_BLOCKS) mscclInterpreter(const __grid_constant__ KernelArgs aParam) {
+__global__ void __launch_bounds__(MSCCL_MAX_THREADS, PROTO == 0 ? MSCCL_MIN_BLOCKS : MSCCL_LAT_MIN_BLOCKS)
+    mscclInterpreter(const __grid_constant__ KernelArgs aParam) {
   __shared__ int sAbort;
   // The launch arguments (all ranks' base pointers and tables, geometry) are copied from the
   // parameter bank into shared memory by all threads at once: every later access is a shared
