@@ -277,3 +277,72 @@ def test_v9_rechecked_once_per_pipeline_depth(env):
     finally:
         for c, p_ in zip(comms, ps):
             c.unload(p_)
+
+
+def _range_sizes(lo, hi, w, cap=8 << 20):
+    """byte sizes that probe one [lo, hi) range: its start, a ragged size inside, its end"""
+    out = []
+    if lo > 0:
+        out.append(lo)
+    out.append(min(lo + 6 * w + 2 * w, cap) if hi == 0 else min(lo + (hi - lo) // 3 + 2 * w, cap))
+    if hi:
+        out.append(min(hi - 2 * w, cap))
+    return sorted({(b // w) * w for b in out if b >= w})
+
+
+@pytest.mark.parametrize("which", ["tuned_allreduce", "tuned_allreduce_multimem"])
+def test_tuned_allreduce_sets_through_the_public_api(which):
+    """The size-range program sets (§6) as a user runs them: every program loaded
+    with its range, mscclAllReduce at each range's start, inside and end (8 ranks, bf16); the
+    result equals, bit for bit, the oracle running the program the range selects."""
+    import torch
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    W = 8
+    sets = getattr(P, which)(W)
+    comms = runtime.Comm.virtual(W, 0)
+    try:
+        for c in comms:
+            for algo, lo, hi in sets:
+                c.load(algo.to_xml(), lo, hi)
+        for algo, lo, hi in sets:
+            for nbytes in _range_sizes(lo, hi, 2):
+                n = nbytes // 2
+                xs = synth.inputs(W, n, "bfloat16", "uniform", seed=nbytes)
+                want = sim.simulate(irparse.parse(algo.to_xml()), xs, n, "bfloat16", "sum")
+                send = [torch.from_numpy(x.view(np.int16).copy()).cuda().view(torch.bfloat16) for x in xs]
+                recv = [torch.empty_like(s) for s in send]
+                _call(runtime, comms, lambda q, c: c.allreduce(send[q], recv[q]))
+                torch.cuda.synchronize()
+                for q in range(W):
+                    got = recv[q].view(torch.int16).cpu().numpy().view(np.uint16)
+                    assert np.array_equal(got, want[q].view(np.uint16)), (which, algo.name, nbytes, q)
+    finally:
+        for c in comms:
+            c.destroy()
+
+
+def test_tuned_alltoall_set_through_the_public_api():
+    """mscclAllToAll with the AllToAll size-range set (selection bytes = per-peer count * w):
+    exact permutation at each range's start, inside and end."""
+    import torch
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    W = 8
+    sets = P.tuned_alltoall(W)
+    comms = runtime.Comm.virtual(W, 0)
+    try:
+        for c in comms:
+            for algo, lo, hi in sets:
+                c.load(algo.to_xml(), lo, hi)
+        for algo, lo, hi in sets:
+            for nbytes in _range_sizes(lo, hi, 4, cap=1 << 20):
+                n = nbytes // 4   # per-peer count
+                xs = synth.inputs(W, W * n, "int32", "pattern")
+                send = [torch.from_numpy(x.copy()).cuda() for x in xs]
+                recv = [torch.empty_like(s) for s in send]
+                _call(runtime, comms, lambda q, c: c.alltoall(send[q], recv[q]))
+                torch.cuda.synchronize()
+                for q, e in enumerate(mpi_ref.alltoall(xs, n)):
+                    assert np.array_equal(recv[q].cpu().numpy(), e), (algo.name, nbytes, q)
+    finally:
+        for c in comms:
+            c.destroy()
