@@ -235,7 +235,8 @@ const char* mscclGetLastError(mscclComm_t comm); /* comm may be NULL: last globa
  * "MSCCL_SLOTS" FIFO slots per connection (1..16, default 4); "MSCCL_SLOT_BYTES" Simple
  * slot (default 262144), "MSCCL_LL_SLOT_BYTES" (65536), "MSCCL_LL128_SLOT_BYTES" (262144)
  * -- each protocol has its own slots; "MSCCL_MAX_CHANNELS" (32); "MSCCL_THREADS" threads
- * per CTA (64..256, default 256 = 2 CTAs per SM); "MSCCL_TIMEOUT_S" watchdog (default 60,
+ * per CTA (64..256, default 256: 2 CTAs per SM for Simple programs, 1 for LL / LL128, so a
+ * launch holds at most 296 / 148 thread blocks); "MSCCL_TIMEOUT_S" watchdog (default 60,
  * <= 0 disables); "MSCCL_DIRECT" direct placement (1); "MSCCL_DIRECT_TILE" one tile per
  * chunk when every message is direct (1; 2 = also across processes, see registration); "MSCCL_DIRECT_HINTS" L2 hints of direct stores, a
  * bit set (default 9: bit 0 terminal direct sends evict_first, bit 3 forwarded direct sends
