@@ -130,7 +130,9 @@ def random_bases():
             (P.ring_allgather(4, 1, 2).to_xml(), 4), (P.ring_reducescatter(4, 1, 1).to_xml(), 4),
             (P.alltoall_twostep(2, 2).to_xml(), 4), (P.hierarchical_allreduce(2, 2).to_xml(), 4),
             (P.ring_allreduce(4, inplace=True).to_xml(), 4), (P.oneshot_allreduce(4).to_xml(), 4),
-            (P.nvls_allreduce(4, 2).to_xml(), 4), (P.nvls_allgather(4).to_xml(), 4)]
+            (P.nvls_allreduce(4, 2).to_xml(), 4), (P.nvls_allgather(4).to_xml(), 4),
+            (P.ring_allreduce(4, channels=4, split_phases=True).to_xml(), 4),
+            (P.ring_allreduce(4, rings=2).to_xml(), 4), (P.allpairs_allgather(4).to_xml(), 4)]
 
 
 def mutate(text, rng):
