@@ -23,7 +23,8 @@ per rank from the max over ranks of the CUDA-event time; roofline = NVLink per d
 (measured peer copy, nominal 900 GB/s); NCCL 2.28.9 runs in the same loop as the
 comparison arm. MSCCL_FORCE_DEVICE=<d> puts every rank on GPU d, which exercises the
 multi-process plumbing on a one-GPU box (NCCL is then skipped: it refuses two ranks on one
-GPU).
+GPU; processes whose kernels spin on each other while time-slicing one GPU can raise Xid 109
+on this driver, B200_PROFILING.md -- a plumbing check, not a measurement).
 
 --sweep PATH : per-size JSON lines (1 KiB..1 GiB, x2) for AllReduce and AllToAll, eager and
   CUDA graph, the paper's protocol (20 warm-up + 50 timed ops) plus a
