@@ -215,7 +215,7 @@ def parallelize(k):
 # ----------------------------------------------------------------------------- instructions
 class _Ins:
     __slots__ = ("rank", "op", "src", "dst", "cnt", "sp", "rp", "ch", "seq", "deps", "raw", "succ",
-                 "send_to", "recv_from", "dead", "tb", "step", "hasdep", "depth", "rdepth")
+                 "send_to", "recv_from", "dead", "tb", "step", "hasdep", "depth", "rdepth", "opi")
 
     def __init__(self, rank, op, src, dst, cnt, sp=-1, rp=-1, ch=None, seq=0):
         self.rank, self.op, self.src, self.dst, self.cnt = rank, op, src, dst, cnt
@@ -229,6 +229,20 @@ class _Ins:
         self.tb = None
         self.step = None
         self.hasdep = False
+        self.opi = -1          # index of the traced op this instruction comes from
+
+
+class _FifoConflict(Exception):
+    """The scheduler cannot keep a connection FIFO-ordered: the receive at the head of the
+    connection's queue waits (through processing edges) on a receive queued behind it."""
+
+    def __init__(self, opi):
+        super().__init__(opi)
+        self.opi = opi
+
+
+class _ChainConflict(Exception):
+    """A free fused chain fits no channel (it needs two connections on one thread block)."""
 
 
 class Program:
@@ -337,31 +351,59 @@ class Program:
 
     # ------------------------------------------------------------------ lowering
     def lower(self, check_fusion=True):
-        """Lower the traced program to an :class:`ir.Algo`."""
-        ins = self._expand()
-        self._fuse(ins)
-        ins = [x for x in ins if not x.dead]
-        nch = self._assign_channels(ins)
-        ins, nch = self._replicate(ins, nch)
-        tbs = self._build_tbs(ins)
-        self._schedule(ins, tbs)
-        return self._emit(ins, tbs, nch)
+        """Lower the traced program to an :class:`ir.Algo`.
+
+        A connection is a FIFO (the k-th receive takes the k-th message), so the order in
+        which the scheduler issues sends on a connection also orders their receives. When
+        that order conflicts with the receiving rank's processing edges (the receive at the
+        head of the queue waits on a receive behind it), the message at the head moves to a
+        channel of its own and lowering restarts -- two connections, no FIFO relation
+        (channels, §5.2). Shipped programs never need it."""
+        forced = {}
+        self._nch_seen = 1
+        fuse = True
+        for _ in range(4 * len(self._ops) + 8):
+            try:
+                ins = self._expand(forced)
+                if fuse:
+                    self._fuse(ins)
+                ins = [x for x in ins if not x.dead]
+                nch = self._assign_channels(ins)
+                ins, nch = self._replicate(ins, nch)
+                tbs = self._build_tbs(ins)
+                self._schedule(ins, tbs)
+                return self._emit(ins, tbs, nch)
+            except _FifoConflict as e:
+                used = {op.ch for op in self._ops if op.ch is not None} | set(forced.values())
+                forced[e.opi] = max(used | {self._nch_seen - 1}) + 1
+            except _ChainConflict:
+                # a fused chain (rcs / rrcs, §4.3) that passes one rank twice with different
+                # peers needs two connections on its single channel: lower without fusion
+                if not fuse:
+                    raise DSLError("no channel satisfies the one-connection-per-thread-block rule")
+                fuse = False
+        raise DSLError("instruction DAG has a cycle")
 
     def ir(self):
         return self.lower().to_xml()
 
     # step 2: instruction generation (§4.2)
-    def _expand(self):
+    def _expand(self, forced=None):
         ins = []
         seq = [0]
+        cur = [0]
 
         def new(*a, **kw):
+            if forced and cur[0] in forced and kw.get("ch") is None:
+                kw["ch"] = forced[cur[0]]
             x = _Ins(*a, seq=seq[0], **kw)
+            x.opi = cur[0]
             seq[0] += 1
             ins.append(x)
             return x
 
-        for op in self._ops:
+        for opi, op in enumerate(self._ops):
+            cur[0] = opi
             s_r, s_b, s_i = op.src
             d_r, d_b, d_i = op.dst
             if op.kind in ir.MULTIMEM_OPS:  # one instruction on the issuing rank (reading R23)
@@ -377,6 +419,12 @@ class Program:
             else:
                 a_r, a_b, a_i = op.acc
                 if s_r == a_r:
+                    if (s_b, s_i) == (d_b, d_i) and (a_b, a_i) != (d_b, d_i):
+                        # the destination IS the second operand c2: dst <- dst (+) c1 (copying c1
+                        # into dst first would overwrite c2 before it is read); (+) is
+                        # commutative bit for bit (IEEE add / multiply, max / min up to NaN payloads)
+                        new(a_r, "re", (a_b, a_i), (d_b, d_i), op.count, ch=op.ch)
+                        continue
                     if (a_b, a_i) != (d_b, d_i):
                         new(a_r, "cpy", (a_b, a_i), (d_b, d_i), op.count, ch=op.ch)
                     new(a_r, "re", (s_b, s_i), (d_b, d_i), op.count, ch=op.ch)
@@ -506,12 +554,16 @@ class Program:
                         m.ch = c
                     break
             else:
+                if ch is None:
+                    raise _ChainConflict()
                 raise DSLError("no channel satisfies the one-connection-per-thread-block rule "
                                "(explicit ch=%s conflicts)" % ch)
         for x in ins:
             if x.ch is None:
                 x.ch = 0
-        return 1 + max([x.ch for x in ins if x.sp >= 0 or x.rp >= 0 or x.op in ir.MULTIMEM_OPS] + [0])
+        nch = 1 + max([x.ch for x in ins if x.sp >= 0 or x.rp >= 0 or x.op in ir.MULTIMEM_OPS] + [0])
+        self._nch_seen = max(getattr(self, "_nch_seen", 1), nch)
+        return nch
 
     # step 5: whole-program instances (reading R5: interleaved sub-chunks)
     def _replicate(self, ins, nch):
@@ -530,6 +582,7 @@ class Program:
                     m = lambda loc: None if loc is None else (loc[0], (loc[1] + j) * r + i)
                     y = _Ins(x.rank, x.op, m(x.src), m(x.dst), 1, x.sp, x.rp, x.ch + i * nch,
                              seq=(x.seq * r + i) * maxc + j)
+                    y.opi = x.opi
                     pieces.append(y)
                     out.append(y)
                 clones[(x, i)] = pieces
@@ -639,6 +692,9 @@ class Program:
                 if indeg[s] == 0:
                     heapq.heappush(heap, (s.depth, -s.rdepth, s.seq, s))
         if pos != len(ins):
+            for key, ds in deferred.items():
+                if ds and queue.get(key):
+                    raise _FifoConflict(queue[key][0].opi)
             raise DSLError("instruction DAG has a cycle")
         for x in ins:
             for d in x.deps:

@@ -1,0 +1,75 @@
+"""Seeded random MSCCLang programs (test infrastructure).
+
+Each program is a random sequence of the DSL's chunk operations (Table 1) on a
+custom collective: `copy` of a chunk to any rank's out / scratch chunk, and `reduce` of two
+chunks into an out / scratch chunk on the first one's rank (c1.reduce(c2, buffer=, index=),
+reading R11), always through the latest reference of each chunk (§3.3). Beside
+the program the generator returns its sequential meaning: the value of every written chunk
+as a set of (rank, input chunk) contributions, evaluated op by op in program order. The
+tests lower the program (tracing, fusion, channels, thread blocks, dependencies: §4-§5) and
+check that the IR computes exactly that meaning -- in the oracle simulator, and on the GPU.
+int32 sums make the value of a chunk independent of the reduction order, so the check is
+about the dataflow the lowering produces.
+"""
+import random
+
+from paper_conf_asplos_cowanmmsx23_b200.dsl import Collective, DSLError, Program, chunk
+
+
+def random_program(seed, protocol="Simple", instances=None):
+    """(algo, R, C, meaning) or None when the DSL refuses the random program. meaning maps
+    (rank, 'o', index) -> sorted tuple of (rank, in index) contributions (with repeats)."""
+    rng = random.Random(seed)
+    R = rng.choice([2, 3, 4])
+    C = rng.choice([1, 2, 3, 4])
+    S = rng.choice([0, 1, 2, 3])
+    n_ops = rng.randint(3, 16)
+    inst = instances if instances is not None else rng.choice([1, 1, 2])
+    meaning = {}
+    for r in range(R):
+        for k in range(C):
+            meaning[(r, "i", k)] = ((r, k),)
+    try:
+        with Program("fuzz_%d" % seed, Collective(R, C, C), protocol=protocol, instances=inst) as p:
+            for _ in range(n_ops):
+                have = sorted(meaning)
+                dst_bufs = ["o"] + (["s"] if S else [])
+                b = rng.choice(dst_bufs)
+                if rng.random() < 0.5 or len(have) < 2:   # copy
+                    src = rng.choice(have)
+                    dr = rng.randrange(R)
+                    di = rng.randrange(C if b == "o" else S)
+                    if (dr, b, di) == src:
+                        continue
+                    chunk(src[0], _name(src[1]), src[2]).copy(dr, _name(b), di)
+                    meaning[(dr, b, di)] = meaning[src]
+                else:                                       # reduce c1 (+) c2 -> (c1.rank, b, di)
+                    c1, c2 = rng.sample(have, 2)
+                    di = rng.randrange(C if b == "o" else S)
+                    chunk(c1[0], _name(c1[1]), c1[2]).reduce(chunk(c2[0], _name(c2[1]), c2[2]),
+                                                               buffer=_name(b), index=di)
+                    meaning[(c1[0], b, di)] = tuple(sorted(meaning[c1] + meaning[c2]))
+        algo = p.lower()
+    except DSLError:
+        return None
+    return algo, R, C, {k: v for k, v in meaning.items() if k[1] == "o"}
+
+
+def _name(b):
+    return {"i": "in", "o": "out", "s": "sc"}[b]
+
+
+def expected_out(meaning, xs, C, n):
+    """Per written out chunk (rank, index): (lo, hi, the int32 sum of its contributions).
+    n must be a multiple of 4 C, so every chunk (reading R1) has the same E = n / C elements
+    (a ragged chunk would only be partly overwritten by a copy from a longer one, reading R2)."""
+    import numpy as np
+    assert n % (4 * C) == 0
+    E = n // C
+    out = {}
+    for (r, _, k), contrib in meaning.items():
+        acc = np.zeros(E, dtype=np.int64)
+        for (q, j) in contrib:
+            acc += xs[q][j * E:(j + 1) * E].astype(np.int64)
+        out[(r, k)] = (k * E, (k + 1) * E, (acc & 0xFFFFFFFF).astype(np.uint32).view(np.int32))
+    return out
