@@ -1,0 +1,56 @@
+"""The interpreter on seeded random MSCCLang programs (tests/progfuzz.py): every written
+output chunk bit-exact with the oracle simulator executing the same IR, under the Simple, LL
+and LL128 protocols, with direct placement on and off (the loader's direct-placement analysis,
+reading R15, meets programs nobody wrote by hand) and with the cross-launch protocol of the
+multi-GPU deployment run in one launch (reading R28), for int32, bf16 and fp32 sums."""
+import numpy as np
+import pytest
+
+import progfuzz
+import synth
+from oracle import irparse, sim
+
+pytestmark = pytest.mark.gpu
+
+PROTOS = ["Simple", "LL", "LL128"]
+DTYPES = ["int32", "bfloat16", "float32"]
+
+
+@pytest.fixture(scope="module")
+def small_slots():
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    keys = ("MSCCL_SLOT_BYTES", "MSCCL_LL_SLOT_BYTES", "MSCCL_LL128_SLOT_BYTES", "MSCCL_TIMEOUT_S", "MSCCL_DIRECT",
+            "MSCCL_CROSS_LAUNCH")
+    old = {k: runtime.get_param(k) for k in keys}
+    for k in keys[:3]:
+        runtime.set_param(k, 4096)     # several tiles per chunk at these sizes
+    runtime.set_param("MSCCL_TIMEOUT_S", 20)
+    yield runtime
+    for k, v in old.items():
+        runtime.set_param(k, v)
+
+
+@pytest.mark.parametrize("mode", ["direct", "fifo", "cross"])
+@pytest.mark.parametrize("block", range(6))
+def test_random_programs_bit_exact_vs_oracle(small_slots, mode, block):
+    import gpu_util
+    runtime = small_slots
+    runtime.set_param("MSCCL_DIRECT", 0 if mode == "fifo" else 1)
+    runtime.set_param("MSCCL_CROSS_LAUNCH", 1 if mode == "cross" else 0)
+    direct = mode
+    for seed in range(block * 50, (block + 1) * 50):
+        proto = PROTOS[seed % 3]
+        dtype = DTYPES[(seed // 3) % 3]
+        prog = progfuzz.random_program(seed, protocol=proto)
+        assert prog is not None
+        algo, R, C, meaning = prog
+        text = algo.to_xml()
+        n = 16 * C * 37 * 2   # every (sub-)chunk a whole number of 16-byte vectors (reading R1)
+        xs = synth.inputs(R, n, dtype, "int" if dtype == "int32" else "uniform", seed=seed)
+        want = sim.simulate(irparse.parse(text), xs, n, dtype, "sum")
+        got = gpu_util.run_program(text, xs, n, dtype, "sum", out_elems=n)
+        E = n // C
+        for (r, _, k) in meaning:
+            a = got[r][k * E:(k + 1) * E].view(np.uint8)
+            b = want[r][k * E:(k + 1) * E].view(np.uint8)
+            assert np.array_equal(a, b), (seed, proto, dtype, direct, r, k)
