@@ -236,9 +236,14 @@ class _FifoConflict(Exception):
     """The scheduler cannot keep a connection FIFO-ordered: the receive at the head of the
     connection's queue waits (through processing edges) on a receive queued behind it."""
 
-    def __init__(self, opi):
-        super().__init__(opi)
-        self.opi = opi
+    def __init__(self, opis, conns):
+        super().__init__(opis)
+        self.opis = opis    # op indices of the messages involved, the queue head first
+        self.conns = conns  # the connections whose queues are stuck
+
+
+def _ch_ok(a, b):
+    return a is None or b is None or a == b
 
 
 class _ChainConflict(Exception):
@@ -336,6 +341,18 @@ class Program:
             raise DSLError("chunks [%d,%d) out of range for buffer %s" % (index, index + count, b))
 
     def _record(self, kind, src, acc, dst, count, ch):
+        # an op reads its whole source before it writes (gather, then scatter: the oracle's and
+        # the paper's chunk semantics) but the interpreter moves a count-c op chunk by chunk, so a
+        # destination on the same rank and buffer that PARTLY overlaps an operand is ambiguous
+        for opnd in (src, acc):
+            if opnd is None or dst is None or opnd[0] != dst[0] or opnd[1] != dst[1]:
+                continue
+            lo = max(opnd[2], dst[2])
+            hi = min(opnd[2], dst[2]) + count
+            if lo < hi and opnd[2] != dst[2]:
+                raise DSLError("%s: destination %s[%d:%d] partly overlaps an operand %s[%d:%d] on rank %d"
+                               % (kind, dst[1], dst[2], dst[2] + count, opnd[1], opnd[2], opnd[2] + count,
+                                  dst[0]))
         par = 1
         for k in self._par:
             par *= k
@@ -361,6 +378,8 @@ class Program:
         (channels, §5.2). Shipped programs never need it."""
         forced = {}
         self._nch_seen = 1
+        self._trace_conns = set()
+        self._trace_all = False
         fuse = True
         for _ in range(4 * len(self._ops) + 8):
             try:
@@ -374,8 +393,23 @@ class Program:
                 self._schedule(ins, tbs)
                 return self._emit(ins, tbs, nch)
             except _FifoConflict as e:
-                used = {op.ch for op in self._ops if op.ch is not None} | set(forced.values())
-                forced[e.opi] = max(used | {self._nch_seen - 1}) + 1
+                # move a message the program left free (no explicit ch=) and not moved before
+                movable = [i for i in e.opis if i >= 0 and self._ops[i].ch is None and i not in forced]
+                if movable:
+                    used = {op.ch for op in self._ops if op.ch is not None} | set(forced.values())
+                    forced[movable[0]] = max(used | {self._nch_seen - 1}) + 1
+                    continue
+                # the program named these channels: keep its connections but send on them in
+                # program (trace) order, which the sequential program itself proves schedulable
+                new_conns = set(e.conns) - self._trace_conns
+                if new_conns:
+                    self._trace_conns |= new_conns
+                elif not self._trace_all:
+                    self._trace_all = True   # every connection in program order
+                elif fuse:
+                    fuse = False             # program order holds for the unfused instructions
+                else:
+                    raise DSLError("instruction DAG has a cycle")
             except _ChainConflict:
                 # a fused chain (rcs / rrcs, §4.3) that passes one rank twice with different
                 # peers needs two connections on its single channel: lower without fusion
@@ -477,9 +511,12 @@ class Program:
         for x in ins:
             if x.dead or x.op not in ("r", "rrc"):
                 continue
+            # the fused instruction sits on one channel: the incoming connection's (x or its
+            # sender named it) and the outgoing one's (s or its receiver) must not differ
+            xch = x.ch if x.ch is not None else (x.recv_from.ch if x.recv_from is not None else None)
             cands = [s for s in x.succ if not s.dead and s.op == "s" and s.src == x.dst and s.cnt == x.cnt
                      and x in s.raw and s.deps == {x}
-                     and (s.ch is None or x.ch is None or s.ch == x.ch)]
+                     and _ch_ok(xch, s.ch if s.ch is not None else s.send_to.ch)]
             if not cands:
                 continue
             s = max(cands, key=lambda c: (longest[c], -c.seq))
@@ -554,8 +591,8 @@ class Program:
                         m.ch = c
                     break
             else:
-                if ch is None:
-                    raise _ChainConflict()
+                if ch is None or any(x.op in ("rcs", "rrcs", "rrs") for x in members):
+                    raise _ChainConflict()   # retried without fusion (see lower)
                 raise DSLError("no channel satisfies the one-connection-per-thread-block rule "
                                "(explicit ch=%s conflicts)" % ch)
         for x in ins:
@@ -655,8 +692,19 @@ class Program:
         def conn(x):
             return (x.recv_from.rank, x.rank, x.ch)
 
+        # connections that must carry their messages in program order (see lower)
+        pend, held = {}, {}
+        for x in sorted(ins, key=lambda x: x.seq):
+            if x.send_to is not None and (getattr(self, "_trace_all", False)
+                                          or conn(x.send_to) in getattr(self, "_trace_conns", ())):
+                pend.setdefault(conn(x.send_to), []).append(x)
+
         while heap:
             _, _, _, x = heapq.heappop(heap)
+            if x.send_to is not None and conn(x.send_to) in pend:
+                if pend[conn(x.send_to)][0] is not x:
+                    held.setdefault(conn(x.send_to), set()).add(x)
+                    continue
             if x.recv_from is not None:
                 q = queue[conn(x)]
                 if q[0] is not x:
@@ -668,6 +716,12 @@ class Program:
                     heapq.heappush(heap, (q[0].depth, -q[0].rdepth, q[0].seq, q[0]))
             if x.send_to is not None:
                 queue.setdefault(conn(x.send_to), []).append(x.send_to)
+                pq = pend.get(conn(x.send_to))
+                if pq:
+                    pq.pop(0)
+                    if pq and pq[0] in held.get(conn(x.send_to), ()):
+                        held[conn(x.send_to)].discard(pq[0])
+                        heapq.heappush(heap, (pq[0].depth, -pq[0].rdepth, pq[0].seq, pq[0]))
             cands = [tb for tb in tbs[x.rank] if _fits(tb, x)]
             if not cands:
                 raise DSLError("rank %d: no thread block for %s" % (x.rank, x.op))
@@ -692,9 +746,15 @@ class Program:
                 if indeg[s] == 0:
                     heapq.heappush(heap, (s.depth, -s.rdepth, s.seq, s))
         if pos != len(ins):
-            for key, ds in deferred.items():
-                if ds and queue.get(key):
-                    raise _FifoConflict(queue[key][0].opi)
+            stuck = [key for key, ds in deferred.items() if ds and queue.get(key)]
+            stuck += [key for key, hs in held.items() if hs]
+            if stuck:
+                opis = []
+                for key in stuck:
+                    if queue.get(key):
+                        opis.append(queue[key][0].opi)
+                    opis += sorted(d.opi for d in deferred.get(key, ()))
+                raise _FifoConflict(opis, stuck)
             raise DSLError("instruction DAG has a cycle")
         for x in ins:
             for d in x.deps:

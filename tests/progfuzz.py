@@ -18,7 +18,10 @@ from paper_conf_asplos_cowanmmsx23_b200.dsl import Collective, DSLError, Program
 
 def random_program(seed, protocol="Simple", instances=None):
     """(algo, R, C, meaning) or None when the DSL refuses the random program. meaning maps
-    (rank, 'o', index) -> sorted tuple of (rank, in index) contributions (with repeats)."""
+    (rank, 'o', index) -> sorted tuple of (rank, in index) contributions (with repeats).
+    Ops move 1 or 2 consecutive chunks (count > 1: strided tiles, reading R3) and sometimes
+    name a channel (ch=, §5.2); a destination that partly overlaps an operand on the same
+    rank is avoided (the DSL refuses it)."""
     rng = random.Random(seed)
     R = rng.choice([2, 3, 4])
     C = rng.choice([1, 2, 3, 4])
@@ -29,26 +32,44 @@ def random_program(seed, protocol="Simple", instances=None):
     for r in range(R):
         for k in range(C):
             meaning[(r, "i", k)] = ((r, k),)
+
+    def span(loc, cnt):
+        return [(loc[0], loc[1], loc[2] + j) for j in range(cnt)]
+
+    def overlaps(a, b, cnt):
+        return a[0] == b[0] and a[1] == b[1] and a[2] != b[2] and abs(a[2] - b[2]) < cnt
+
     try:
         with Program("fuzz_%d" % seed, Collective(R, C, C), protocol=protocol, instances=inst) as p:
             for _ in range(n_ops):
-                have = sorted(meaning)
-                dst_bufs = ["o"] + (["s"] if S else [])
-                b = rng.choice(dst_bufs)
+                cnt = 2 if rng.random() < 0.3 else 1
+                have = sorted(l for l in meaning if all(x in meaning for x in span(l, cnt)))
+                if not have:
+                    continue
+                b = rng.choice(["o"] + (["s"] if S >= cnt else []))
+                size = C if b == "o" else S
+                if size < cnt:
+                    continue
+                ch = rng.choice([None, None, None, 0, 1, 2])
                 if rng.random() < 0.5 or len(have) < 2:   # copy
                     src = rng.choice(have)
-                    dr = rng.randrange(R)
-                    di = rng.randrange(C if b == "o" else S)
-                    if (dr, b, di) == src:
+                    dst = (rng.randrange(R), b, rng.randrange(size - cnt + 1))
+                    if dst == src or overlaps(src, dst, cnt):
                         continue
-                    chunk(src[0], _name(src[1]), src[2]).copy(dr, _name(b), di)
-                    meaning[(dr, b, di)] = meaning[src]
+                    chunk(src[0], _name(src[1]), src[2], cnt).copy(dst[0], _name(b), dst[2], ch=ch)
+                    vals = [meaning[x] for x in span(src, cnt)]
+                    for x, v in zip(span(dst, cnt), vals):
+                        meaning[x] = v
                 else:                                       # reduce c1 (+) c2 -> (c1.rank, b, di)
                     c1, c2 = rng.sample(have, 2)
-                    di = rng.randrange(C if b == "o" else S)
-                    chunk(c1[0], _name(c1[1]), c1[2]).reduce(chunk(c2[0], _name(c2[1]), c2[2]),
-                                                               buffer=_name(b), index=di)
-                    meaning[(c1[0], b, di)] = tuple(sorted(meaning[c1] + meaning[c2]))
+                    dst = (c1[0], b, rng.randrange(size - cnt + 1))
+                    if overlaps(c1, dst, cnt) or overlaps(c2, dst, cnt) or overlaps(c1, c2, cnt):
+                        continue
+                    chunk(c1[0], _name(c1[1]), c1[2], cnt).reduce(chunk(c2[0], _name(c2[1]), c2[2], cnt),
+                                                                    buffer=_name(b), index=dst[2], ch=ch)
+                    vals = [tuple(sorted(meaning[x] + meaning[y])) for x, y in zip(span(c1, cnt), span(c2, cnt))]
+                    for x, v in zip(span(dst, cnt), vals):
+                        meaning[x] = v
         algo = p.lower()
     except DSLError:
         return None

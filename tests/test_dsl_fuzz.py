@@ -81,3 +81,23 @@ def test_shipped_programs_unchanged_by_conflict_handling():
     assert P.ring_allreduce(8).nchannels == 1
     assert P.ring_allreduce(8, channels=8).nchannels == 8
     assert P.allpairs_allreduce(8).nchannels == 1
+
+
+def test_explicit_channels_against_the_receivers_order_lower_in_program_order():
+    """Messages the program pinned to one channel (ch=) whose receives depend on each other
+    against the scheduler's send order (fuzzer seeds 478 / 829): the connection keeps the
+    program order instead of failing."""
+    for seed in (478, 829, 1020, 1651):
+        prog = progfuzz.random_program(seed)
+        assert prog is not None, seed
+        _check(*prog, seed)
+
+
+def test_partly_overlapping_local_op_is_refused():
+    """A count-2 copy on one rank from out[0:2] to out[1:3] reads a chunk the same op writes:
+    the gather-then-scatter meaning of an op and the interpreter's chunk-by-chunk execution
+    would differ, so the DSL refuses it."""
+    with pytest.raises(dsl.DSLError, match="partly overlaps"):
+        with Program("ovl", Collective(1, 3, 3)):
+            chunk(0, "in", 0, 2).copy(0, "out", 0)
+            chunk(0, "out", 0, 2).copy(0, "out", 1)
