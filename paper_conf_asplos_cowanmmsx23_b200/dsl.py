@@ -328,6 +328,13 @@ class Program:
 
     def _mm_final(self, b, index, count, rank):
         self._check_bounds(b, index, count)
+        # a store into another rank's chunk is ordered only against the other multimem ops (the
+        # group barrier, reading R23): that chunk must not have been written there before
+        for r in range(self.R):
+            if r != rank and any(v is not None for v in self._versions(r, b, index, count)):
+                raise DSLError("multimem store to %s[%d:%d] of rank %d, which the program already wrote "
+                               "(reading R23: multimem stores go to chunks other ranks have not touched)"
+                               % (b, index, index + count, r))
         for r in range(self.R):
             for k in range(index, index + count):
                 self._ver[self._key(r, b, k)] = FINAL
@@ -574,6 +581,8 @@ class Program:
         for g in glist:
             chs = {c for e in g for c in (e.ch, e.send_to.ch) if c is not None}
             if len(chs) > 1:
+                if any(x.op in ("rcs", "rrcs", "rrs") for x in g):
+                    raise _ChainConflict()   # fusion joined connections the program put on different channels
                 raise DSLError("a fused chain mixes channels %s" % sorted(chs))
             (fixed if chs else free).append((g, chs.pop() if chs else None))
         self._tbstate = [_TBState() for _ in range(self.R)]
@@ -643,6 +652,11 @@ class Program:
                 if not states[x.rank].add(x.sp, x.rp, x.ch):
                     raise DSLError("rank %d: (send %d, recv %d, ch %d) conflicts with an existing "
                                    "thread block" % (x.rank, x.sp, x.rp, x.ch))
+        per_rank = [sorted({x.ch for x in ins if x.rank == r and x.op in ir.MULTIMEM_OPS}) for r in range(self.R)]
+        mm_channels = per_rank[0] if per_rank else []
+        if any(m != mm_channels for m in per_rank):
+            raise DSLError("multimem ops must be issued on every rank on the same channels (their thread "
+                           "blocks pair up across ranks, reading R23 / V11): %s" % per_rank)
         tbs = []
         for r in range(self.R):
             tuples = states[r].final()
@@ -657,10 +671,11 @@ class Program:
                         merged.append(t)
                 tuples = merged + list(recv_only.values())
             lst = [_TB(t[0], t[1], t[2]) for t in tuples]
-            # multimem ops run on their own thread block per channel (its group barrier pairs
-            # it with the same block on every rank, reading R23)
-            for ch in sorted({x.ch for x in ins if x.rank == r and x.op in ir.MULTIMEM_OPS}):
-                lst.append(_TB(-1, -1, ch))
+            # multimem ops run on their own thread block per channel, and that block must have
+            # the same id on every rank (its group barrier pairs it with block b of every rank,
+            # reading R23, rule V11): they come first, in channel order
+            mm = [_TB(-1, -1, ch) for ch in mm_channels]
+            lst = mm + lst
             if not lst and any(x.rank == r for x in ins):
                 lst.append(_TB(-1, -1, 0))
             for i, tb in enumerate(lst):

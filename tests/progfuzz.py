@@ -39,11 +39,40 @@ def random_program(seed, protocol="Simple", instances=None):
     def overlaps(a, b, cnt):
         return a[0] == b[0] and a[1] == b[1] and a[2] != b[2] and abs(a[2] - b[2]) < cnt
 
+    final = set()   # chunks a multimem store wrote on every rank: final (reading R23)
     try:
         with Program("fuzz_%d" % seed, Collective(R, C, C), protocol=protocol, instances=inst) as p:
             for _ in range(n_ops):
                 cnt = 2 if rng.random() < 0.3 else 1
-                have = sorted(l for l in meaning if all(x in meaning for x in span(l, cnt)))
+                if protocol == "Simple" and rng.random() < 0.12:   # a multimem (NVLS) round, Simple only
+                    # every rank issues one (their thread blocks pair up, reading R23 / V11):
+                    # mrd on the same chunk everywhere, or mrs on a distinct chunk per rank
+                    if C < cnt:
+                        continue
+                    if C >= R and rng.random() < 0.5:
+                        base = rng.randrange(C)
+                        ks = [(base + r) % C for r in range(R)]
+                        # stores go to chunks no other rank wrote before (reading R23)
+                        if cnt > 1 or any((q, "o", k) in meaning for r, k in enumerate(ks) for q in range(R)
+                                          if q != r):
+                            continue
+                        for r, k in enumerate(ks):
+                            chunk(r, "in", k).multimem_reduce("out", k, store_all=True)
+                            v = tuple(sorted((q, k) for q in range(R)))
+                            for q in range(R):
+                                meaning[(q, "o", k)] = v
+                                final.add((q, "o", k))
+                    else:
+                        k = rng.randrange(C - cnt + 1)
+                        if any((q, "o", k + j) in final for q in range(R) for j in range(cnt)):
+                            continue
+                        for r in range(R):
+                            chunk(r, "in", k, cnt).multimem_reduce("out", k, store_all=False)
+                            for j in range(cnt):
+                                meaning[(r, "o", k + j)] = tuple(sorted((q, k + j) for q in range(R)))
+                    continue
+                have = sorted(l for l in meaning if l not in final and
+                              all(x in meaning and x not in final for x in span(l, cnt)))
                 if not have:
                     continue
                 b = rng.choice(["o"] + (["s"] if S >= cnt else []))
@@ -54,7 +83,7 @@ def random_program(seed, protocol="Simple", instances=None):
                 if rng.random() < 0.5 or len(have) < 2:   # copy
                     src = rng.choice(have)
                     dst = (rng.randrange(R), b, rng.randrange(size - cnt + 1))
-                    if dst == src or overlaps(src, dst, cnt):
+                    if dst == src or overlaps(src, dst, cnt) or any(x in final for x in span(dst, cnt)):
                         continue
                     chunk(src[0], _name(src[1]), src[2], cnt).copy(dst[0], _name(b), dst[2], ch=ch)
                     vals = [meaning[x] for x in span(src, cnt)]
@@ -63,7 +92,8 @@ def random_program(seed, protocol="Simple", instances=None):
                 else:                                       # reduce c1 (+) c2 -> (c1.rank, b, di)
                     c1, c2 = rng.sample(have, 2)
                     dst = (c1[0], b, rng.randrange(size - cnt + 1))
-                    if overlaps(c1, dst, cnt) or overlaps(c2, dst, cnt) or overlaps(c1, c2, cnt):
+                    if overlaps(c1, dst, cnt) or overlaps(c2, dst, cnt) or overlaps(c1, c2, cnt) or \
+                            any(x in final for x in span(dst, cnt)):
                         continue
                     chunk(c1[0], _name(c1[1]), c1[2], cnt).reduce(chunk(c2[0], _name(c2[1]), c2[2], cnt),
                                                                     buffer=_name(b), index=dst[2], ch=ch)
