@@ -16,12 +16,15 @@ import random
 from paper_conf_asplos_cowanmmsx23_b200.dsl import Collective, DSLError, Program, chunk
 
 
-def random_program(seed, protocol="Simple", instances=None):
+def random_program(seed, protocol="Simple", instances=None, inplace=None):
     """(algo, R, C, meaning) or None when the DSL refuses the random program. meaning maps
     (rank, 'o', index) -> sorted tuple of (rank, in index) contributions (with repeats).
     Ops move 1 or 2 consecutive chunks (count > 1: strided tiles, reading R3) and sometimes
     name a channel (ch=, §5.2); a destination that partly overlaps an operand on the same
     rank is avoided (the DSL refuses it)."""
+    if inplace is None:   # a quarter of the programs are in place: 'out' is 'in' (reading R8)
+        inplace = random.Random(seed ^ 0x5EED).random() < 0.25
+    ib = "i" if inplace else "o"   # the buffer results land in
     rng = random.Random(seed)
     R = rng.choice([2, 3, 4])
     C = rng.choice([1, 2, 3, 4])
@@ -41,10 +44,11 @@ def random_program(seed, protocol="Simple", instances=None):
 
     final = set()   # chunks a multimem store wrote on every rank: final (reading R23)
     try:
-        with Program("fuzz_%d" % seed, Collective(R, C, C), protocol=protocol, instances=inst) as p:
+        with Program("fuzz_%d" % seed, Collective(R, C, C, inplace=inplace), protocol=protocol,
+                     instances=inst) as p:
             for _ in range(n_ops):
                 cnt = 2 if rng.random() < 0.3 else 1
-                if protocol == "Simple" and rng.random() < 0.12:   # a multimem (NVLS) round, Simple only
+                if protocol == "Simple" and not inplace and rng.random() < 0.12:   # multimem round (Simple)
                     # every rank issues one (their thread blocks pair up, reading R23 / V11):
                     # mrd on the same chunk everywhere, or mrs on a distinct chunk per rank
                     if C < cnt:
@@ -75,8 +79,8 @@ def random_program(seed, protocol="Simple", instances=None):
                               all(x in meaning and x not in final for x in span(l, cnt)))
                 if not have:
                     continue
-                b = rng.choice(["o"] + (["s"] if S >= cnt else []))
-                size = C if b == "o" else S
+                b = rng.choice([ib] + (["s"] if S >= cnt else []))
+                size = C if b in ("o", "i") else S
                 if size < cnt:
                     continue
                 ch = rng.choice([None, None, None, 0, 1, 2])
@@ -103,7 +107,7 @@ def random_program(seed, protocol="Simple", instances=None):
         algo = p.lower()
     except DSLError:
         return None
-    return algo, R, C, {k: v for k, v in meaning.items() if k[1] == "o"}
+    return algo, R, C, {(k[0], "o", k[2]): v for k, v in meaning.items() if k[1] == ib}
 
 
 def _name(b):

@@ -17,7 +17,7 @@ from paper_conf_asplos_cowanmmsx23_b200.dsl import Collective, Program, chunk
 
 def _check(algo, R, C, meaning, seed, rt=None):
     text = algo.to_xml()
-    al = irparse.parse(text)
+    al = irparse.parse(text)   # in-place programs: the simulator's out aliases in (reading R8)
     validate.validate(al, nranks=R, slots=8)
     if rt is not None:
         ok, msg = rt.validate(text, R, slots=8)
@@ -68,7 +68,7 @@ def test_fifo_order_conflict_splits_the_connection():
     """Two messages on one connection whose receives depend on each other in the order
     opposite to the one the priority scheduler sends them (seed 3 of the fuzzer): lowering
     moves one message to another channel instead of failing."""
-    prog = progfuzz.random_program(3, instances=1)
+    prog = progfuzz.random_program(3, instances=1, inplace=False)
     assert prog is not None
     _check(*prog, 3)
     assert prog[0].nchannels >= 2
@@ -88,7 +88,7 @@ def test_explicit_channels_against_the_receivers_order_lower_in_program_order():
     against the scheduler's send order (fuzzer seeds 478 / 829): the connection keeps the
     program order instead of failing."""
     for seed in (478, 829, 1020, 1651):
-        prog = progfuzz.random_program(seed)
+        prog = progfuzz.random_program(seed, inplace=False)
         assert prog is not None, seed
         _check(*prog, seed)
 

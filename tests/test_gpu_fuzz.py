@@ -48,7 +48,8 @@ def test_random_programs_bit_exact_vs_oracle(small_slots, mode, block):
         n = 16 * C * 37 * 2   # every (sub-)chunk a whole number of 16-byte vectors (reading R1)
         xs = synth.inputs(R, n, dtype, "int" if dtype == "int32" else "uniform", seed=seed)
         want = sim.simulate(irparse.parse(text), xs, n, dtype, "sum")
-        got = gpu_util.run_program(text, xs, n, dtype, "sum", out_elems=n)
+        # in-place programs run both in place and out of place (pre-copy, reading R8)
+        got = gpu_util.run_program(text, xs, n, dtype, "sum", out_elems=n, inplace=algo.inplace and seed % 2 == 0)
         E = n // C
         for (r, _, k) in meaning:
             a = got[r][k * E:(k + 1) * E].view(np.uint8)
