@@ -19,7 +19,7 @@ def comms(R, device=0):
     return _COMMS[key]
 
 
-def run_program(ir_text, inputs, count, dtype, op="sum", out_elems=None, inplace=False, device=0):
+def run_program(ir_text, inputs, count, dtype, op="sum", out_elems=None, inplace=False, device=0, fill=0xA5):
     """Load `ir_text` on R virtual ranks, run it once on `inputs` (numpy, storage dtype),
     return the per-rank outputs as numpy arrays (storage dtype)."""
     R = len(inputs)
@@ -32,7 +32,7 @@ def run_program(ir_text, inputs, count, dtype, op="sum", out_elems=None, inplace
             recv = send
         else:
             ob = (out_elems if out_elems is not None else raw[0].size) * raw[0].itemsize
-            recv = [torch.full((ob,), 0xA5, dtype=torch.uint8, device=f"cuda:{device}") for _ in range(R)]
+            recv = [torch.full((ob,), fill, dtype=torch.uint8, device=f"cuda:{device}") for _ in range(R)]
         with runtime.group():
             for c, p, s, r in zip(cs, progs, send, recv):
                 c.run(p, s, r, count, op=op, dtype=dtype)
