@@ -57,6 +57,35 @@ def test_random_programs_bit_exact_vs_oracle(small_slots, mode, block):
             assert np.array_equal(a, b), (seed, proto, dtype, direct, r, k)
 
 
+@pytest.mark.parametrize("op", ["max", "min", "prod"])
+def test_random_programs_other_reductions(small_slots, op):
+    """max / min / prod (reading R6; multimem has no product, so prod programs use LL / LL128
+    or Simple without multimem rounds): written chunks bit-exact with the simulator."""
+    import gpu_util
+    runtime = small_slots
+    runtime.set_param("MSCCL_DIRECT", 1)
+    runtime.set_param("MSCCL_CROSS_LAUNCH", 0)
+    for seed in range(2000, 2060):
+        proto = PROTOS[seed % 3]
+        dtype = DTYPES[(seed // 3) % 3]
+        prog = progfuzz.random_program(seed, protocol=proto)
+        assert prog is not None
+        algo, R, C, meaning = prog
+        text = algo.to_xml()
+        if op == "prod" and ('type="mr' in text or 'type="ms' in text):
+            continue
+        n = 16 * C * 37 * 2
+        dist = "int" if dtype == "int32" else "uniform"
+        xs = synth.inputs(R, n, dtype, dist, seed=seed)
+        want = sim.simulate(irparse.parse(text), xs, n, dtype, op)
+        got = gpu_util.run_program(text, xs, n, dtype, op, out_elems=n, inplace=algo.inplace)
+        E = n // C
+        for (r, _, k) in meaning:
+            a = got[r][k * E:(k + 1) * E].view(np.uint8)
+            b = want[r][k * E:(k + 1) * E].view(np.uint8)
+            assert np.array_equal(a, b), (seed, proto, dtype, op, r, k)
+
+
 @pytest.mark.parametrize("mode", ["direct", "fifo"])
 def test_random_programs_ragged_sizes_whole_buffers(small_slots, mode):
     """Ragged counts (chunks of unequal length, reading R1 / R2; LL / LL128 partial lines): every
