@@ -2,7 +2,7 @@
 
 For every program: it lowers (§4-§5: instruction generation, fusion, channels, instances,
 thread blocks, dependencies), both validators accept the IR (V1-V9), the happens-before race
-detector finds nothing (V10), and the oracle simulator computes exactly the program's
+detector finds nothing (V10) -- also under the C++ loader's direct-placement marking -- and the oracle simulator computes exactly the program's
 sequential meaning -- each written out chunk equals the int32 sum of the chunks the program's
 copies and reduces combined into it, in program order (§3.1-3.3)."""
 import numpy as np
@@ -22,6 +22,9 @@ def _check(algo, R, C, meaning, seed, rt=None):
     if rt is not None:
         ok, msg = rt.validate(text, R, slots=8)
         assert ok, msg
+        # the C++ loader's direct-placement marking (reading R15) is race free too (V10)
+        marking = {q: rt.direct_placement(text, q) for q in range(R)}
+        assert races.check_direct(al, marking, alias=algo.inplace) == [], seed
     assert races.find_races(al) == []
     n = 8 * C * 37
     xs = synth.inputs(R, n, "int32", "int", seed=seed)
