@@ -104,3 +104,23 @@ def test_partly_overlapping_local_op_is_refused():
         with Program("ovl", Collective(1, 3, 3)):
             chunk(0, "in", 0, 2).copy(0, "out", 0)
             chunk(0, "out", 0, 2).copy(0, "out", 1)
+
+
+def test_validators_agree_on_deadlock_with_one_and_two_slots(rt):
+    """V9 on random programs with 1 and 2 FIFO slots: the C++
+    loader and the oracle's validator return the same verdict."""
+    verdicts = set()
+    for seed in range(400):
+        algo, R, C, _ = progfuzz.random_program(seed)
+        text = algo.to_xml()
+        al = irparse.parse(text)
+        for s in (1, 2):
+            try:
+                validate.validate(al, nranks=R, slots=s, iters=2)
+                py = None
+            except validate.ValidationError as e:
+                py = str(e)[:2]
+            ok, msg = rt.validate(text, R, slots=s)
+            assert py == (None if ok else msg[:2]), (seed, s, py, msg)
+            verdicts.add(py)
+    assert None in verdicts and "V9" in verdicts   # both outcomes occur
