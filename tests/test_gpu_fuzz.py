@@ -139,3 +139,39 @@ def _simulate_other_poison(text, xs, n, dtype):
         return sim.simulate(irparse.parse(text), xs, n, dtype, "sum")
     finally:
         nm.poison = orig
+
+
+def test_random_programs_with_one_fifo_slot(small_slots):
+    """MSCCL_SLOTS=1: the programs V9 accepts with one slot (the loader re-checks at the launch's
+    pipeline depth, reading R24) run to completion on the GPU -- the abstract machine's
+    deadlock freedom holds for the interpreter -- and match the simulator; the ones it refuses
+    are refused before anything is launched."""
+    import gpu_util
+    runtime = small_slots
+    runtime.set_param("MSCCL_DIRECT", 1)
+    runtime.set_param("MSCCL_CROSS_LAUNCH", 0)
+    old = runtime.get_param("MSCCL_SLOTS")
+    runtime.set_param("MSCCL_SLOTS", 1)
+    ran = refused = 0
+    try:
+        for seed in range(3000, 3080):
+            proto = PROTOS[seed % 3]
+            prog = progfuzz.random_program(seed, protocol=proto)
+            algo, R, C, meaning = prog
+            text = algo.to_xml()
+            n = 16 * C * 37 * 2
+            xs = synth.inputs(R, n, "int32", "int", seed=seed)
+            try:
+                got = gpu_util.run_program(text, xs, n, "int32", "sum", out_elems=n, inplace=algo.inplace)
+            except runtime.MscclError as e:
+                assert e.code == 8 and "V9" in str(e), str(e)   # mscclInvalidProgram, deadlock
+                refused += 1
+                continue
+            want = sim.simulate(irparse.parse(text), xs, n, "int32", "sum", slots=1)
+            E = n // C
+            for (r, _, k) in meaning:
+                assert np.array_equal(got[r][k * E:(k + 1) * E], want[r][k * E:(k + 1) * E]), (seed, proto, r, k)
+            ran += 1
+    finally:
+        runtime.set_param("MSCCL_SLOTS", old)
+    assert ran > 0
