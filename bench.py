@@ -352,9 +352,9 @@ def set_params(rt, args):
     rt.set_param("MSCCL_DIRECT_TILE", 2)  # every rank registers its buffers (reading R19b)
 
 
-def sampled_parity(algo, recv_list, n, ranks_to_check, local=None):
-    """Bit-exact check of sampled outputs against the oracle's reduction trees.
-    recv_list[i] is the output of rank (local[i] if local else i)."""
+def sampled_parity(algo, recv_list, n, ranks_to_check, local=None, dtype="bfloat16"):
+    """Bit-exact check of sampled outputs against the oracle's reduction trees (2-byte float
+    dtypes). recv_list[i] is the output of rank (local[i] if local else i)."""
     import numpy as np
     import torch
     import synth
@@ -364,11 +364,11 @@ def sampled_parity(algo, recv_list, n, ranks_to_check, local=None):
     idx = np.unique(np.concatenate([g.integers(0, n, SEED_SAMPLES), [0, n - 1, n // 2]]))
     bad = 0
     for i, q in enumerate(ranks_to_check):
-        want = sampled.reduction_at(al, lambda r, ii: synth.hashed_numpy(r, ii, "bfloat16"), n, "bfloat16", "sum",
+        want = sampled.reduction_at(al, lambda r, ii: synth.hashed_numpy(r, ii, dtype), n, dtype, "sum",
                                     idx, rank=q)
         out = recv_list[q if local is None else local.index(q)]
         got = out[torch.from_numpy(idx).to(out.device)].view(torch.int16).cpu().numpy().view(np.uint16)
-        bad += int(np.count_nonzero(got != want))
+        bad += int(np.count_nonzero(got != np.asarray(want).view(np.uint16)))   # bit patterns
     return bad, idx.size * len(ranks_to_check)
 
 

@@ -1436,9 +1436,9 @@ __device__ __noinline__ void chainExecSimple(const Ctx& c, const DevInstr* mem, 
 #ifndef MSCCL_MM_MIN_BLOCKS
 #define MSCCL_MM_MIN_BLOCKS MSCCL_MIN_BLOCKS  // multimem kernels (reading R23)
 #endif
-template <int DT, int OP, int PROTO, bool MM = false>
+template <int DT, int OP, int PROTO, bool MM = false, int MINB = 0>  // MINB: CTAs per SM (0 = by protocol)
 __global__ void __launch_bounds__(MSCCL_MAX_THREADS,
-                                  MM ? MSCCL_MM_MIN_BLOCKS : (PROTO == 0 ? MSCCL_MIN_BLOCKS : MSCCL_LAT_MIN_BLOCKS))
+                                  MINB ? MINB : (MM ? MSCCL_MM_MIN_BLOCKS : (PROTO == 0 ? MSCCL_MIN_BLOCKS : MSCCL_LAT_MIN_BLOCKS)))
     mscclInterpreter(const __grid_constant__ KernelArgs aParam) {
   __shared__ int sAbort;
   // The launch arguments (all ranks' base pointers and tables, geometry) are copied from the

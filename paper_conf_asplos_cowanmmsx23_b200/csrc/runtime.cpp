@@ -587,13 +587,23 @@ mscclResult_t launchCalls(std::vector<Call>& calls) {
       if (direct == 2 && ra.directMask) cl->comm->launchesDirect2++;
     }
     if (cta == 0) continue;
-    const void* fn = p0->hasMultimem ? (p0->hasReduce ? interpreterKernelMM(v[0]->dtype, v[0]->op)
-                                                      : copyKernelMM(elemBytes(v[0]->dtype)))
-                     : p0->hasReduce ? interpreterKernel(v[0]->dtype, v[0]->op, ka.proto)
-                                     : copyKernel(elemBytes(v[0]->dtype), ka.proto);
+    auto pick = [&](bool wide) {
+      return p0->hasMultimem ? (p0->hasReduce ? interpreterKernelMM(v[0]->dtype, v[0]->op)
+                                              : copyKernelMM(elemBytes(v[0]->dtype)))
+             : p0->hasReduce ? interpreterKernel(v[0]->dtype, v[0]->op, ka.proto, wide)
+                             : copyKernel(elemBytes(v[0]->dtype), ka.proto, wide);
+    };
+    const void* fn = pick(false);
     int maxCta = 0;
     r = coResident(c0, fn, (int)c0->prm.threads, 0, maxCta);
     if (r != mscclSuccess) return r;
+    if (cta > maxCta && ka.proto != 0 && !p0->hasMultimem) {
+      // the LL / LL128 kernels run 1 CTA per SM (no spills); a larger launch takes their
+      // 2-CTA/SM build instead
+      fn = pick(true);
+      r = coResident(c0, fn, (int)c0->prm.threads, 0, maxCta);
+      if (r != mscclSuccess) return r;
+    }
     if (cta > maxCta) {
       std::ostringstream o;
       o << "program needs " << cta << " co-resident CTAs on device " << c0->dev << " but at most " << maxCta
