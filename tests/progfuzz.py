@@ -13,7 +13,9 @@ about the dataflow the lowering produces.
 """
 import random
 
-from paper_conf_asplos_cowanmmsx23_b200.dsl import Collective, DSLError, Program, chunk
+import contextlib
+
+from paper_conf_asplos_cowanmmsx23_b200.dsl import Collective, DSLError, Program, chunk, parallelize
 
 
 def random_program(seed, protocol="Simple", instances=None, inplace=None):
@@ -84,12 +86,16 @@ def random_program(seed, protocol="Simple", instances=None, inplace=None):
                 if size < cnt:
                     continue
                 ch = rng.choice([None, None, None, 0, 1, 2])
+                # parallelize(2) splits a 2-chunk op into two 1-chunk ops on
+                # channels ch, ch+1
+                par = parallelize(2) if cnt == 2 and rng.random() < 0.4 else contextlib.nullcontext()
                 if rng.random() < 0.5 or len(have) < 2:   # copy
                     src = rng.choice(have)
                     dst = (rng.randrange(R), b, rng.randrange(size - cnt + 1))
                     if dst == src or overlaps(src, dst, cnt) or any(x in final for x in span(dst, cnt)):
                         continue
-                    chunk(src[0], _name(src[1]), src[2], cnt).copy(dst[0], _name(b), dst[2], ch=ch)
+                    with par:
+                        chunk(src[0], _name(src[1]), src[2], cnt).copy(dst[0], _name(b), dst[2], ch=ch)
                     vals = [meaning[x] for x in span(src, cnt)]
                     for x, v in zip(span(dst, cnt), vals):
                         meaning[x] = v
@@ -99,8 +105,9 @@ def random_program(seed, protocol="Simple", instances=None, inplace=None):
                     if overlaps(c1, dst, cnt) or overlaps(c2, dst, cnt) or overlaps(c1, c2, cnt) or \
                             any(x in final for x in span(dst, cnt)):
                         continue
-                    chunk(c1[0], _name(c1[1]), c1[2], cnt).reduce(chunk(c2[0], _name(c2[1]), c2[2], cnt),
-                                                                    buffer=_name(b), index=dst[2], ch=ch)
+                    with par:
+                        chunk(c1[0], _name(c1[1]), c1[2], cnt).reduce(chunk(c2[0], _name(c2[1]), c2[2], cnt),
+                                                                        buffer=_name(b), index=dst[2], ch=ch)
                     vals = [tuple(sorted(meaning[x] + meaning[y])) for x, y in zip(span(c1, cnt), span(c2, cnt))]
                     for x, v in zip(span(dst, cnt), vals):
                         meaning[x] = v
