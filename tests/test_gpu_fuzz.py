@@ -175,3 +175,32 @@ def test_random_programs_with_one_fifo_slot(small_slots):
     finally:
         runtime.set_param("MSCCL_SLOTS", old)
     assert ran > 0
+
+
+@pytest.mark.parametrize("slot", [12544, 65536])
+def test_random_programs_other_slot_sizes(small_slots, slot):
+    """Other FIFO slot sizes (tile T and depth I follow, reading R3): written chunks bit-exact."""
+    import gpu_util
+    runtime = small_slots
+    runtime.set_param("MSCCL_DIRECT", 1)
+    runtime.set_param("MSCCL_CROSS_LAUNCH", 0)
+    keys = ("MSCCL_SLOT_BYTES", "MSCCL_LL_SLOT_BYTES", "MSCCL_LL128_SLOT_BYTES")
+    for k in keys:
+        runtime.set_param(k, slot)
+    try:
+        for seed in range(4000, 4060):
+            proto = PROTOS[seed % 3]
+            dtype = DTYPES[(seed // 3) % 3]
+            algo, R, C, meaning = progfuzz.random_program(seed, protocol=proto)
+            text = algo.to_xml()
+            n = 16 * C * 37 * 8
+            xs = synth.inputs(R, n, dtype, "int" if dtype == "int32" else "uniform", seed=seed)
+            want = sim.simulate(irparse.parse(text), xs, n, dtype, "sum")
+            got = gpu_util.run_program(text, xs, n, dtype, "sum", out_elems=n, inplace=algo.inplace)
+            E = n // C
+            for (r, _, k) in meaning:
+                assert np.array_equal(got[r][k * E:(k + 1) * E].view(np.uint8), want[r][k * E:(k + 1) * E].view(np.uint8)), \
+                    (seed, proto, dtype, slot, r, k)
+    finally:
+        for k in keys:
+            runtime.set_param(k, 4096)
