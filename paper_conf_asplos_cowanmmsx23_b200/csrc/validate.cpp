@@ -200,11 +200,49 @@ void validateIR(Algo& a, int nranks, int slots, int maxTbs, int maxChannels, int
 
 namespace {
 
+// the instruction whose message receive step (tb, s) of rank g takes: the k-th send of the peer's
+// thread block on this connection for the k-th receive of this one
+const Instr* matchingSend(const Algo& a, int g, int tb, int s) {
+  const ThreadBlock& rt = a.gpus[g].tbs[tb];
+  if (rt.recv < 0) return nullptr;
+  int k = 0;
+  for (int i = 0; i < s; i++)
+    if (opRole(rt.steps[i].op).recv) k++;
+  for (auto& st : a.gpus[rt.recv].tbs) {
+    if (st.send != g || st.chan != rt.chan) continue;
+    int j = 0;
+    for (auto& x : st.steps)
+      if (opRole(x.op).send) {
+        if (j == k) return &x;
+        j++;
+      }
+  }
+  return nullptr;
+}
+
+// Chunk k of a buffer has the length of chunk (k mod chunks-per-block) of every block (reading
+// R1); scratch chunks are never short. A direct store of piece j of an instruction that also
+// writes its own destination (rcs / rrcs) is cut to the receiver's chunk length, so that chunk
+// must be as long as the sender's for every count: same position in its block, or scratch.
+bool lengthsCompatible(const Algo& a, const Instr& snd, const Instr& rcv) {
+  if (!opRole(snd.op).dst) return true;  // nothing local to shorten
+  const int cb = a.gpus[0].iChunks / blocksOf(a.coll, BUF_IN, a.ngpus);
+  if (cb <= 0) return false;
+  for (int j = 0; j < rcv.cnt; j++) {
+    if (rcv.dstBuf == BUF_SC) continue;
+    if (snd.dstBuf == BUF_SC) return false;
+    if ((snd.dstOff + j) % cb != (rcv.dstOff + j) % cb) return false;
+  }
+  return true;
+}
+
 // may receive step (tb, s) of rank g write its destination before its turn?
 bool recvCanBeDirect(const Algo& a, int g, int tb, int s) {
   const GpuProgram& gp = a.gpus[g];
   const Instr& q = gp.tbs[tb].steps[s];
   if (q.op != OP_RECV && q.op != OP_RCS) return false;  // data must land unchanged
+  const Instr* snd = matchingSend(a, g, tb, s);
+  if (snd && !lengthsCompatible(a, *snd, q)) return false;
   auto canon = [&](int buf) { return (a.inplace && buf == BUF_OUT) ? BUF_IN : buf; };
   const int qb = canon(q.dstBuf);
   auto overlaps = [&](int buf, int off, int cnt) {

@@ -132,7 +132,7 @@ def _simulate_other_poison(text, xs, n, dtype):
             return np.full(m, 0x4049, dtype=np.uint16)
         if dt in ("float16", "float32", "float64"):
             return np.full(m, 3.25, dtype=nm.storage(dt))
-        return np.full(m, 0x15A5A5A5, dtype=nm.storage(dt))
+        return np.full(m, -0x15A5A5A5, dtype=nm.storage(dt))   # negative: min against int max
 
     nm.poison = other
     try:
@@ -204,3 +204,28 @@ def test_random_programs_other_slot_sizes(small_slots, slot):
     finally:
         for k in keys:
             runtime.set_param(k, 4096)
+
+
+def test_rrcs_direct_target_shorter_than_local_chunk(small_slots):
+    """Fuzzer seed 10013 (Simple, bf16, 8206 elements: the last chunk is 38 elements): an rrcs
+    whose matching receive lands in the ragged last chunk of the peer must not be a direct
+    placement -- the direct store is cut to the receiver's chunk, which used to cut this rank's
+    own stored result short as well. The loader now places such messages through the FIFO."""
+    import gpu_util
+    runtime = small_slots
+    runtime.set_param("MSCCL_DIRECT", 1)
+    runtime.set_param("MSCCL_CROSS_LAUNCH", 0)
+    runtime.set_param("MSCCL_SLOT_BYTES", 8192)
+    try:
+        algo, R, C, meaning = progfuzz.random_program(10013, protocol="Simple")
+        text = algo.to_xml()
+        n = 8206
+        xs = synth.inputs(R, n, "bfloat16", "uniform", seed=10013)
+        got = gpu_util.run_program(text, xs, n, "bfloat16", "sum", out_elems=n, inplace=algo.inplace, fill=0)
+        want = sim.simulate(irparse.parse(text), xs, n, "bfloat16", "sum")
+        want2 = _simulate_other_poison(text, xs, n, "bfloat16")
+        for r in range(R):
+            a, b, g = (x.view(np.uint16) for x in (want[r], want2[r], got[r]))
+            assert np.array_equal(g[a == b], a[a == b]), r
+    finally:
+        runtime.set_param("MSCCL_SLOT_BYTES", 4096)

@@ -155,3 +155,24 @@ def test_bench_probe_programs_are_valid(rt):
             al = irparse.parse(text)
             pyval.validate(al, nranks=R, races=True)
             assert races.find_races(al) == []
+
+
+def test_direct_placement_needs_equal_chunk_lengths(rt):
+    """A receive is placed directly only if the matching send's own destination chunk is as long
+    as the receiver's for every count (same position in its block, or a scratch target), since a
+    direct store stops at the receiver's chunk (reading R15; found by the random-program fuzzer).
+    Here rank 0's rrcs writes its chunk 0 and forwards to rank 1's chunk 1 (the ragged one for
+    counts that are not a multiple of the chunking): not direct; to rank 1's chunk 0: direct."""
+    def prog(peer_off):
+        return ('<algo name="len" coll="custom" ngpus="2" proto="Simple" inplace="0" nchannels="2" ninstances="1">'
+                '<gpu id="0" i_chunks="2" o_chunks="2" s_chunks="0">'
+                '<tb id="0" send="1" recv="1" chan="0"><step s="0" type="rrcs" srcbuf="i" srcoff="0" dstbuf="o" '
+                'dstoff="0" cnt="1" depid="-1" deps="-1" hasdep="0"/></tb></gpu>'
+                '<gpu id="1" i_chunks="2" o_chunks="2" s_chunks="0">'
+                '<tb id="0" send="0" recv="-1" chan="0"><step s="0" type="s" srcbuf="i" srcoff="0" dstbuf="-" '
+                'dstoff="-1" cnt="1" depid="-1" deps="-1" hasdep="0"/></tb>'
+                '<tb id="1" send="-1" recv="0" chan="0"><step s="0" type="r" srcbuf="-" srcoff="-1" dstbuf="o" '
+                'dstoff="%d" cnt="1" depid="-1" deps="-1" hasdep="0"/></tb></gpu></algo>' % peer_off)
+    assert rt.validate(prog(1), 2)[0] and rt.validate(prog(0), 2)[0]
+    assert rt.direct_placement(prog(1), 0)[0][0] == 0      # rank 0's rrcs: FIFO
+    assert rt.direct_placement(prog(0), 0)[0][0] == 1      # same chunk position: direct
