@@ -18,7 +18,7 @@ import contextlib
 from paper_conf_asplos_cowanmmsx23_b200.dsl import Collective, DSLError, Program, chunk, parallelize
 
 
-def random_program(seed, protocol="Simple", instances=None, inplace=None):
+def random_program(seed, protocol="Simple", instances=None, inplace=None, max_ranks=4):
     """(algo, R, C, meaning) or None when the DSL refuses the random program. meaning maps
     (rank, 'o', index) -> sorted tuple of (rank, in index) contributions (with repeats).
     Ops move 1 or 2 consecutive chunks (count > 1: strided tiles, reading R3) and sometimes
@@ -28,7 +28,7 @@ def random_program(seed, protocol="Simple", instances=None, inplace=None):
         inplace = random.Random(seed ^ 0x5EED).random() < 0.25
     ib = "i" if inplace else "o"   # the buffer results land in
     rng = random.Random(seed)
-    R = rng.choice([2, 3, 4])
+    R = rng.choice([2, 3, 4]) if max_ranks == 4 else rng.randint(2, max_ranks)
     C = rng.choice([1, 2, 3, 4])
     S = rng.choice([0, 1, 2, 3])
     n_ops = rng.randint(3, 16)

@@ -47,7 +47,7 @@ def main():
         mode = g.choice(["direct", "fifo", "cross"])
         slot = g.choice([4096, 8192, 16384, 65536])
         slots = g.choice([2, 4, 4, 8])
-        prog = progfuzz.random_program(seed, protocol=proto)
+        prog = progfuzz.random_program(seed, protocol=proto, max_ranks=8)
         if prog is None:
             fails.append((seed, "dsl refused"))
             continue
