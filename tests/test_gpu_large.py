@@ -156,3 +156,65 @@ def test_bench_size_reducescatter_sampled_parity():
     finally:
         for c, p in zip(cs, progs):
             c.unload(p)
+
+
+def test_more_than_2_pow_31_elements():
+    """Maximum sizes: an int8 ring AllReduce of 2^31 + 12345 elements per rank (2 virtual
+    ranks, 8 instances) -- element offsets beyond 32 bits in the chunk geometry (reading R1) and
+    the data loops. int8 sums wrap, so every element is x0 + x1 mod 256 whatever the order; a
+    million sampled elements and the whole ragged tail are checked."""
+    import torch
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    n = (1 << 31) + 12345
+    if torch.cuda.get_device_properties(0).total_memory < 6 * n:
+        pytest.skip("needs 4 buffers of 2 GiB")
+    g = torch.Generator(device="cuda").manual_seed(20230325)
+    send = [torch.randint(-128, 128, (n,), dtype=torch.int8, device="cuda", generator=g) for _ in range(2)]
+    recv = [torch.empty_like(s) for s in send]
+    comms = runtime.Comm.virtual(2, 0)
+    try:
+        algo = P.ring_allreduce(2, instances=8)
+        progs = [c.load(algo.to_xml()) for c in comms]
+        with runtime.group():
+            for c, p, s, r in zip(comms, progs, send, recv):
+                c.run(p, s, r, n, dtype="int8")
+        torch.cuda.synchronize()
+        idx = torch.cat([torch.randint(0, n, (1 << 20,), device="cuda", generator=g),
+                         torch.arange(n - 70000, n, device="cuda")])
+        want = (send[0][idx].to(torch.int32) + send[1][idx].to(torch.int32)).to(torch.uint8).to(torch.int8)
+        for r in recv:
+            assert torch.equal(r[idx], want)
+        for c, p in zip(comms, progs):
+            c.unload(p)
+    finally:
+        for c in comms:
+            c.destroy()
+
+
+def test_allgather_output_beyond_4g_elements():
+    """Maximum sizes: an AllGather of 2^31 + 777 uint8 elements per rank into a 2^32 + 1554
+    element output (2 virtual ranks): block offsets b * n beyond 32 bits (reading R1); exact."""
+    import torch
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    n = (1 << 31) + 777
+    if torch.cuda.get_device_properties(0).total_memory < 8 * n:
+        pytest.skip("needs 12 GiB")
+    g = torch.Generator(device="cuda").manual_seed(7)
+    send = [torch.randint(0, 256, (n,), dtype=torch.uint8, device="cuda", generator=g) for _ in range(2)]
+    recv = [torch.empty(2 * n, dtype=torch.uint8, device="cuda") for _ in range(2)]
+    comms = runtime.Comm.virtual(2, 0)
+    try:
+        algo = P.ring_allgather(2, 1, 4)
+        progs = [c.load(algo.to_xml()) for c in comms]
+        with runtime.group():
+            for c, p, s, r in zip(comms, progs, send, recv):
+                c.run(p, s, r, n, dtype="uint8")
+        torch.cuda.synchronize()
+        for r in recv:
+            for q in range(2):
+                assert torch.equal(r[q * n:(q + 1) * n], send[q])
+        for c, p in zip(comms, progs):
+            c.unload(p)
+    finally:
+        for c in comms:
+            c.destroy()
