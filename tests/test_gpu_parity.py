@@ -173,3 +173,17 @@ def test_slot_counts(slots, proto):
                              "sum")
     finally:
         runtime.set_param("MSCCL_SLOTS", 4)
+
+
+@pytest.mark.parametrize("name", ["ring", "ring_inplace", "allpairs", "oneshot", "allgather", "reducescatter",
+                                  "alltoall", "nvls"])
+def test_one_rank_programs(name):
+    """Degenerate case R = 1 on a one-rank communicator: output = input, bit for bit."""
+    build = {"ring": lambda: P.ring_allreduce(1), "ring_inplace": lambda: P.ring_allreduce(1, inplace=True),
+             "allpairs": lambda: P.allpairs_allreduce(1, protocol="Simple"), "oneshot": lambda: P.oneshot_allreduce(1),
+             "allgather": lambda: P.ring_allgather(1, 2, 2), "reducescatter": lambda: P.ring_reducescatter(1, 2, 2),
+             "alltoall": lambda: P.alltoall_twostep(1, 1), "nvls": lambda: P.nvls_allreduce(1)}[name]
+    n = 4099
+    xs = synth.inputs(1, n, "float32", "uniform")
+    got = _gpu().run_program(build().to_xml(), xs, n, "float32", "sum")
+    assert _bits_equal(got[0][:n], xs[0][:n])

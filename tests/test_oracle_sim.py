@@ -219,3 +219,29 @@ def test_scratch_tail_garbage_never_reaches_output():
     out = sim.simulate(_parse(P.allpairs_allreduce(R)), xs, n, "float32")
     ref = mpi_ref.allreduce(xs, "sum", "float32")
     assert all(_eq(o, r.astype(np.float32)) for o, r in zip(out, ref))
+
+
+ONE_RANK = [
+    ("ring", lambda: P.ring_allreduce(1), "allreduce"),
+    ("ring_inplace", lambda: P.ring_allreduce(1, inplace=True), "allreduce"),
+    ("ring_instances", lambda: P.ring_allreduce(1, instances=2), "allreduce"),
+    ("ring_k2", lambda: P.ring_allreduce(1, rings=2), "allreduce"),
+    ("allpairs", lambda: P.allpairs_allreduce(1), "allreduce"),
+    ("oneshot", lambda: P.oneshot_allreduce(1), "allreduce"),
+    ("allgather", lambda: P.ring_allgather(1, 2, 2), "allgather"),
+    ("reducescatter", lambda: P.ring_reducescatter(1, 2, 2), "reducescatter"),
+    ("alltoall", lambda: P.alltoall_twostep(1, 1), "alltoall"),
+    ("nvls", lambda: P.nvls_allreduce(1), "allreduce"),
+]
+
+
+@pytest.mark.parametrize("name,build,coll", ONE_RANK, ids=[x[0] for x in ONE_RANK])
+def test_one_rank_programs_copy_their_input(name, build, coll):
+    """Degenerate case R = 1: every collective's output is the input (the MPI definitions with
+    one rank); the ring builders used to leave the output unwritten (DSL refused the ring
+    AllReduce, the ReduceScatter was empty)."""
+    algo = _parse(build())
+    n = 1000
+    xs = synth.inputs(1, n, "int32", "int")
+    out = sim.simulate(algo, xs, n, "int32", "sum")
+    assert np.array_equal(out[0][:n], xs[0][:n])
