@@ -187,6 +187,11 @@ mscclResult_t mscclProgramTouches(mscclProgram_t program, int directPlacement, i
 mscclResult_t mscclDebugDirectPlacement(const char* ir, size_t irBytes, int rank, int32_t* flags,
                                         int32_t* rdst, int maxInstr, int* nInstr);
 
+/* Test hook: set the launch generation of every thread block of `program` (the counter the
+ * dependency semaphores carry, reading R4), so tests can cross the 2^24-launch wrap of the
+ * semaphores' generation field without 16 M launches. Synchronises the device. */
+mscclResult_t mscclDebugSetGeneration(mscclProgram_t program, uint64_t generation);
+
 /* Comm-free structural validation (rules V1..V9 of DESIGN.md) — needs no GPU.
  * slots = FIFO slots per connection used by the deadlock check (0 = library default),
  * maxThreadBlocks = co-residency limit per rank (0 = 148). err (may be NULL) receives a

@@ -316,11 +316,31 @@ __device__ __forceinline__ bool waitGE(const uint64_t* p, uint64_t target, bool 
 }
 
 // Cross-thread-block dependency (Fig. 5 lines 15-16): wait until thread block dtb of this
-// rank has finished step dstep of tile t in this launch (monotone semaphore, reading R4).
+// rank has finished step dstep of tile t in this launch (reading R4). A semaphore holds
+// (launch generation mod 2^24) << 40 | (steps done in this launch); it can only hold this
+// launch's value or the previous launch's, so the wait asks for the same generation field and
+// at least the step -- a plain >= on the whole word broke after 2^24 launches, when the
+// generation field wrapped below the previous launch's.
 __device__ __forceinline__ bool waitDep(const RankArgs& ra, uint64_t dep, uint64_t gen, int t, const Ctx& c) {
   const int dtb = (int)(dep >> 48), dstep = (int)((dep >> 32) & 0xffff);
   const uint64_t dn = (uint32_t)dep;  // steps of thread block dtb
-  return waitGE(&ra.sem[dtb], (gen << 40) | ((uint64_t)t * dn + (uint64_t)dstep + 1), false, c);
+  const uint64_t want = (uint64_t)t * dn + (uint64_t)dstep + 1, g = gen << 40;
+  const uint64_t* p = &ra.sem[dtb];
+  constexpr uint64_t kLow = (1ull << 40) - 1;
+  uint64_t v = ldAcquireGpu(p);
+  if ((v & ~kLow) == g && (v & kLow) >= want) return true;
+  const uint64_t t0 = globaltimer();
+  for (uint32_t it = 1;; it++) {
+    v = ldAcquireGpu(p);
+    if ((v & ~kLow) == g && (v & kLow) >= want) return true;
+    if ((it & 1023u) == 0) {
+      if (*(volatile uint32_t*)c.ra->abortFlag) return false;
+      if (c.a->timeoutNs && globaltimer() - t0 > c.a->timeoutNs) {
+        raiseAbort(*c.a);
+        return false;
+      }
+    }
+  }
 }
 
 // ------------------------------------------------------------------ chunk geometry (reading R1)

@@ -1514,6 +1514,16 @@ mscclResult_t mscclProgramInfo(mscclProgram_t p, int* nTB, int* nInstr, int* inp
   return mscclSuccess;
 }
 
+mscclResult_t mscclDebugSetGeneration(mscclProgram_t p, uint64_t generation) {
+  if (!p) return mscclInvalidArgument;
+  if (!p->nTB) return mscclSuccess;
+  DeviceGuard dg(p->comm->dev);
+  std::vector<uint64_t> g(p->nTB, generation);
+  CUDACHECK(p->comm, cudaDeviceSynchronize());
+  CUDACHECK(p->comm, cudaMemcpy(p->dSem + p->nTB, g.data(), g.size() * sizeof(uint64_t), cudaMemcpyHostToDevice));
+  return mscclSuccess;
+}
+
 mscclResult_t mscclProgramTouches(mscclProgram_t p, int direct, int64_t* touches) {
   if (!p || !touches) return mscclInvalidArgument;
   static const int cost[OP_COUNT] = {0, 2, 2, 2, 3, 3, 3, 4, 3};

@@ -64,6 +64,7 @@ SIGNATURES = {
     "mscclRegExport": (_i, [_vp, _vp]),
     "mscclRegConnect": (_i, [_vp, _vp]),
     "mscclCommDeregister": (_i, [_vp, _vp]),
+    "mscclDebugSetGeneration": (_i, [_vp, _c.c_uint64]),
     "mscclDebugDirectPlacement": (_i, [_c.c_char_p, _sz, _i, _c.POINTER(_c.c_int32), _c.POINTER(_c.c_int32), _i,
                                        _c.POINTER(_i)]),
 }
@@ -223,6 +224,10 @@ class Program:
         a, b, c = _i(), _i(), _i()
         _check(lib.mscclProgramInfo(self.handle, _c.byref(a), _c.byref(b), _c.byref(c)), self.comm.handle)
         return {"thread_blocks": a.value, "instructions": b.value, "inplace": bool(c.value)}
+
+    def set_generation(self, gen):
+        """mscclDebugSetGeneration (test hook): the launch generation of every thread block."""
+        _check(lib.mscclDebugSetGeneration(self.handle, gen), self.comm.handle)
 
     def touches(self, direct=True):
         """Algorithmic chunk-sized memory touches of this rank's program (mscclProgramTouches)."""

@@ -346,3 +346,35 @@ def test_tuned_alltoall_set_through_the_public_api():
     finally:
         for c in comms:
             c.destroy()
+
+
+@pytest.mark.parametrize("make", ["allpairs", "oneshot", "hier"])
+def test_semaphores_across_the_generation_wrap(make):
+    """Programs with cross-thread-block dependencies launched across 2^24 launches of their
+    thread blocks (the generation field of a semaphore wraps, reading R4): every launch
+    bit-exact. With a plain >= on the semaphore word the launch right after the wrap saw the
+    previous launch's (larger) value as done and read its inputs too early."""
+    import torch
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    W = 4
+    algo = {"allpairs": lambda: P.allpairs_allreduce(W, protocol="Simple"),
+            "oneshot": lambda: P.oneshot_allreduce(W, protocol="Simple"),
+            "hier": lambda: P.hierarchical_allreduce(2, 2)}[make]()
+    comms = runtime.Comm.virtual(W, 0)
+    try:
+        progs = [c.load(algo.to_xml()) for c in comms]
+        for p in progs:
+            p.set_generation((1 << 24) - 3)
+        for it in range(6):
+            n = 200003 + it
+            xs = synth.inputs(W, n, "float32", "uniform", seed=it)
+            want = sim.simulate(irparse.parse(algo.to_xml()), xs, n, "float32")
+            send = [torch.from_numpy(x).cuda() for x in xs]
+            recv = [torch.empty_like(s) for s in send]
+            _call(runtime, comms, lambda q, c: c.run(progs[q], send[q], recv[q], n))
+            torch.cuda.synchronize()
+            for q in range(W):
+                assert np.array_equal(recv[q].cpu().numpy().view(np.uint32), want[q].view(np.uint32)), (it, q)
+    finally:
+        for c in comms:
+            c.destroy()
