@@ -3,7 +3,7 @@ a protocol / dtype / placement mode / slot size / count drawn from the seed, com
 oracle simulator on every element that does not depend on stale data (the simulator run with two
 poisons, as in tests/test_gpu_fuzz.py). Prints one summary line and the failing seeds.
 
-Usage: python tools/fuzz_campaign.py LO HI   (needs a GPU)
+Usage: python tools/fuzz_campaign.py LO HI [MAX_N]   (needs a GPU; MAX_N = largest count, default 20000)
 """
 import json
 import os
@@ -26,6 +26,7 @@ def main():
     from paper_conf_asplos_cowanmmsx23_b200 import runtime
 
     lo, hi = int(sys.argv[1]), int(sys.argv[2])
+    max_n = int(sys.argv[3]) if len(sys.argv) > 3 else 20000
     runtime.set_param("MSCCL_TIMEOUT_S", 20)
     orig_poison = nm.poison
 
@@ -53,7 +54,7 @@ def main():
             continue
         algo, R, C, meaning = prog
         text = algo.to_xml()
-        n = g.randint(1, 20000)
+        n = g.randint(1, max_n)
         for k in ("MSCCL_SLOT_BYTES", "MSCCL_LL_SLOT_BYTES", "MSCCL_LL128_SLOT_BYTES"):
             runtime.set_param(k, slot)
         runtime.set_param("MSCCL_SLOTS", slots)
@@ -94,7 +95,7 @@ def main():
             fails.append((seed, dict(proto=proto, dtype=dtype, op=op, mode=mode, slot=slot, slots=slots, n=n,
                                      bad=bad)))
     stats["seconds"] = round(time.time() - t0, 1)
-    print(json.dumps({"seeds": [lo, hi], **stats}))
+    print(json.dumps({"seeds": [lo, hi], "max_n": max_n, **stats}))
     for f in fails[:40]:
         print("FAIL", f)
 
