@@ -179,7 +179,9 @@ mscclResult_t mscclProgramTouches(mscclProgram_t program, int directPlacement, i
 /* Direct-placement marking the loader computes for rank `rank` of an IR program (reading
  * R15; needs no GPU). For every instruction in (thread block, step) order of that rank,
  * flags[k] = bit 0 DIRECT_SEND (the message is stored into the receiver's destination),
- * bit 1 DIRECT_RECV (the data is already in dst when the head arrives); for a direct send
+ * bit 1 DIRECT_RECV (the data is already in dst when the head arrives), bit 2 PULLED_RECV (the
+ * receive reads the sender's input chunk itself, reading R30), bit 3 PULLED_SEND (its
+ * partner: moves no data); for a direct send
  * rdst[2k], rdst[2k+1] = the receiver's destination buffer (0 i, 1 o, 2 s) and chunk.
  * maxInstr = capacity of flags (rdst: 2*maxInstr); *nInstr = instructions of the rank.
  * Exported so the CPU oracle's race detector (oracle/races.py) can check the marking
@@ -244,9 +246,11 @@ const char* mscclGetLastError(mscclComm_t comm); /* comm may be NULL: last globa
  * launch holds at most 296 / 148 thread blocks); "MSCCL_TIMEOUT_S" watchdog (default 60,
  * <= 0 disables); "MSCCL_DIRECT" direct placement (1); "MSCCL_DIRECT_TILE" one tile per
  * chunk when every message is direct (1; 2 = also across processes, see registration); "MSCCL_DIRECT_HINTS" L2 hints of direct stores, a
- * bit set (default 9: bit 0 terminal direct sends evict_first, bit 3 forwarded direct sends
- * evict_normal; bit 1 demote forwarded lines after reading, bit 2 FIFO stores evict_normal:
- * measured slower, off); "MSCCL_MAX_REGISTRATIONS" (64). All ranks must
+ * bit set (default 25: bit 0 terminal direct sends evict_first, bit 3 forwarded direct sends
+ * evict_normal, bit 4 pulled messages: with every rank in one launch a receive whose message
+ * is a plain send of an input chunk reads that chunk itself, reading R30; bit 1 demote
+ * forwarded lines after reading, bit 2 FIFO stores evict_normal: measured slower, off);
+ * "MSCCL_MAX_REGISTRATIONS" (64). All ranks must
  * use the same values (mscclCommConnect checks). Returns mscclInvalidArgument for an
  * unknown key. */
 mscclResult_t mscclSetParam(const char* key, int64_t value);

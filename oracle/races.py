@@ -158,7 +158,9 @@ def accesses(algo, alias=False, direct=None):
     """Chunk accesses per event: {(q, tb, s): [(rank, buf, chunk, "r"|"w"), ...]}.
 
     direct: None, or {(q, tb, s): ("send", (rank, buf, off, cnt)) | ("recv", None)} -- the
-    direct-placement transformation described in the module docstring."""
+    direct-placement transformation described in the module docstring -- plus, for pulled
+    messages (reading R30), ((q, tb, s), "pulled"): True on the send (it reads nothing) and
+    ((q, tb, s), "pull"): (sender, buf, off, cnt) on the receive (it reads the sender's chunk)."""
     acc = defaultdict(list)
     direct = direct or {}
     for g in algo.gpus:
@@ -174,9 +176,14 @@ def accesses(algo, alias=False, direct=None):
                             if st.writes_all or p == q:
                                 acc[e].append((p, _canon(algo, st.dstbuf, alias), st.dstoff + j, "w"))
                     continue
-                if st.reads_src:
+                if st.reads_src and (e, "pulled") not in direct:   # a pulled send reads nothing (R30)
                     for j in range(st.cnt):
                         acc[e].append((q, _canon(algo, st.srcbuf, alias), st.srcoff + j, "r"))
+                pull = direct.get((e, "pull"))
+                if pull is not None:                   # a pulled receive reads the sender's chunk
+                    (pq, pbuf, poff, pcnt) = pull
+                    for j in range(pcnt):
+                        acc[e].append((pq, _canon(algo, pbuf, alias), poff + j, "r"))
                 if st.op == "re":
                     for j in range(st.cnt):
                         acc[e].append((q, _canon(algo, st.dstbuf, alias), st.dstoff + j, "r"))
@@ -229,7 +236,8 @@ def direct_map(algo, marking):
     """Turn the loader's per-rank marking into the `direct` argument of accesses().
 
     marking: {rank: [(flags, rdst_buf, rdst_chunk), ...]} in (thread block, step) order;
-    flags bit 0 = direct send, bit 1 = direct receive; rdst_buf 0/1/2 = i/o/s.
+    flags bit 0 = direct send, bit 1 = direct receive, bit 2 = pulled receive, bit 3 = pulled
+    send (reading R30); rdst_buf 0/1/2 = i/o/s.
     Raises MarkingError when the two ends of a connection disagree."""
     bufs = ("i", "o", "s")
     flat = {}
@@ -248,6 +256,16 @@ def direct_map(algo, marking):
         for a, b in zip(sends, recvs):
             fa, rb_, ro = flat[a]
             fb = flat[b][0]
+            sp, rp = bool(fa & 8), bool(fb & 4)
+            if sp != rp:
+                raise MarkingError("send %s pulled=%s but its receive %s pulled=%s" % (a, sp, b, rp))
+            if sp:
+                ss = steps[a]
+                if ss.op != "s":
+                    raise MarkingError("pulled send %s is a %s (only a plain send moves a chunk unchanged)"
+                                       % (a, ss.op))
+                out[(a, "pulled")] = True
+                out[(b, "pull")] = (a[0], ss.srcbuf, ss.srcoff, ss.cnt)
             sd, rd = bool(fa & 1), bool(fb & 2)
             if sd != rd:
                 raise MarkingError("send %s direct=%s but its receive %s direct=%s" % (a, sd, b, rd))
@@ -264,6 +282,8 @@ def direct_map(algo, marking):
             prevb = out.get(b)
             out[b] = ("both", prevb[1]) if prevb and prevb[0] == "send" else ("recv", None)
     for e, (f, _, _) in flat.items():
+        if (f & 12) and (e, "pull") not in out and (e, "pulled") not in out:
+            raise MarkingError("%s marked pulled but its connection partner is not" % (e,))
         if (f & 2) and e not in out:
             raise MarkingError("receive %s marked direct but no send on its connection is" % (e,))
     return out

@@ -22,7 +22,11 @@ namespace msccl {
 
 // DI_SEND_TERMINAL: a direct send whose receiving instruction is a plain recv (the data is
 // not forwarded by the receiver's thread block: a cache hint only)
-enum { DI_SEND_DIRECT = 1, DI_RECV_DIRECT = 2, DI_CHAIN_HEAD = 4, DI_SEND_TERMINAL = 8 };
+// DI_RECV_PULL / DI_SEND_PULLED (reading R30): with every rank in the launch (direct == 1) and
+// MSCCL_DIRECT_HINTS bit 4, the receive reads its message from the sender's input chunk pullOff
+// (rank chainLen) and the send moves no data (it still posts its head flag).
+enum { DI_SEND_DIRECT = 1, DI_RECV_DIRECT = 2, DI_CHAIN_HEAD = 4, DI_SEND_TERMINAL = 8, DI_RECV_PULL = 16,
+       DI_SEND_PULLED = 32 };
 
 struct DevInstr {     // 32 bytes
   uint8_t op, srcBuf, dstBuf, nDeps;
@@ -32,8 +36,9 @@ struct DevInstr {     // 32 bytes
   // instead of its FIFO slot. flags: DI_SEND_DIRECT (this send writes peer rdstBuf/rdstOff),
   // DI_RECV_DIRECT (the data of this receive is already in dst when its head arrives).
   uint8_t flags, rdstBuf;
-  uint16_t chainLen;          // DI_CHAIN_HEAD: this and the next chainLen-1 local ops fold into one pass
-  uint32_t rdstOff, pad1;
+  uint16_t chainLen;          // DI_CHAIN_HEAD: this and the next chainLen-1 local ops fold into one pass;
+                              // DI_RECV_PULL: the sender's rank
+  uint32_t rdstOff, pullOff;  // pullOff: DI_RECV_PULL: the sender's input chunk
 };
 
 // One thread block of one rank (= one CTA). Connection pointers are resolved at load time
@@ -113,7 +118,8 @@ struct KernelArgs {
   int32_t direct;
   int32_t directHints;        // L2 hints (interp.cuh HINT_*): bit 0 terminal direct sends evict_first,
                               // bit 1 demote read forwarded lines, bit 2 FIFO stores / bit 3 direct
-                              // forwards evict_normal (default 9)
+                              // forwards evict_normal; bit 4 pulled first hops with direct == 1
+                              // (reading R30) (default 25 = bits 0, 3, 4)
   // multimem ops (reading R23): 0 none; 1 every rank in this launch (slot r = rank r, buffers
   // from the launch arguments, no barrier); 2 cross-launch (group barrier lines publish the
   // ranks' buffer references at the start and completion at the end)

@@ -382,7 +382,8 @@ __device__ __forceinline__ void chunkSpan(const KernelArgs& a, int buf, int64_t 
 // L2 evict_first (reading R15, DI_SEND_TERMINAL)
 // HINT_SRC_DEMOTE: the src lines were stored evict_last by a direct sender (forwarded data):
 // demote them once read. HINT_SEND_NORMAL: store the outgoing lines evict_normal.
-enum { HINT_SEND_FIRST = 1, HINT_SRC_DEMOTE = 2, HINT_SEND_NORMAL = 4 };
+// HINT_NO_DISCARD: the received lines are not a FIFO slot (a pulled input chunk, reading R30).
+enum { HINT_SEND_FIRST = 1, HINT_SRC_DEMOTE = 2, HINT_SEND_NORMAL = 4, HINT_NO_DISCARD = 8 };
 
 template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST, int VB>
 __device__ __forceinline__ int64_t vecLoop(int64_t nvec, const char* rslot, const char* src, char* dst, char* sslot,
@@ -391,7 +392,7 @@ __device__ __forceinline__ int64_t vecLoop(int64_t nvec, const char* rslot, cons
   constexpr int U = ((int)RECV + (int)SRC + (int)REDDST) >= 2 ? MSCCL_UNROLL : MSCCL_UNROLL1;
   const uint64_t pFirst = policyEvictFirst(), pLast0 = policyEvictLast();
   const uint64_t pLast = (hint & HINT_SEND_FIRST) ? pFirst : (hint & HINT_SEND_NORMAL) ? policyEvictNormal() : pLast0;
-  const bool canDiscard = RECV && ((((uintptr_t)rslot) & 127) == 0);
+  const bool canDiscard = RECV && !(hint & HINT_NO_DISCARD) && ((((uintptr_t)rslot) & 127) == 0);
   const int lane = ti & 31, warp = ti >> 5, nw = nt >> 5;
   // Full blocks of U x 32 vectors, one block per warp-iteration (warp-uniform trip count,
   // so the __syncwarp below is reached by every lane); each u-row is 32 x VB contiguous bytes.
@@ -782,18 +783,30 @@ __device__ __forceinline__ bool sendIsDirect(const Ctx& c, const DevInstr& in) {
 __device__ __forceinline__ bool recvIsDirect(const Ctx& c, const DevInstr& in) {
   return (in.flags & DI_RECV_DIRECT) && c.a->direct && ((c.ra->directMask >> in.dstBuf) & 1);
 }
+// reading R30: every rank in this launch and MSCCL_DIRECT_HINTS bit 4 (both ends see the same
+// launch arguments, so they agree)
+__device__ __forceinline__ bool pullOn(const Ctx& c) { return c.a->direct == 1 && (c.a->directHints & 16); }
 
 template <int DT, int OP, bool RECV, bool SEND, bool SRC, bool DST, bool REDDST>
 __device__ __noinline__ void movePiecesSimple(const Ctx& c, const DevTB& tb, const DevInstr& in, int t,
                                               const char* rslot, char* sslot) {
   MSCCL_PIECE_GEOM
+  if (SEND && !RECV && (in.flags & DI_SEND_PULLED) && pullOn(c)) return;  // the receiver reads the chunk
   const bool sdirect = SEND && sendIsDirect(c, in);
   const bool rdirect = RECV && recvIsDirect(c, in);
+  const bool rpull = RECV && (in.flags & DI_RECV_PULL) && pullOn(c);
   for (int j = 0; j < in.cnt; j++) {
     const char* src;
     char* dst;
     int64_t m = pieceGeom<DT, SRC, DST, REDDST>(c, in, t, j, src, dst);
     char* so = SEND ? sslot + j * a.T * w : nullptr;
+    const char* ri = RECV ? rslot + j * a.T * w : nullptr;
+    if (rpull) {  // reading R30: the message is the sender's input chunk, unchanged for the launch
+      int64_t ps, pl;
+      chunkSpan(a, 0, (int64_t)in.pullOff + j, ps, pl);  // buffer 0 = in
+      ri = a.rank[in.chainLen].buf[0] + (ps + a0) * w;
+      if (pl - a0 < m) m = pl - a0;
+    }
     if (sdirect) {  // reading R15: write straight into the receiver's destination chunk
       int64_t rs, rl;
       chunkSpan(a, in.rdstBuf, (int64_t)in.rdstOff + j, rs, rl);
@@ -811,8 +824,8 @@ __device__ __noinline__ void movePiecesSimple(const Ctx& c, const DevTB& tb, con
                                                              hint | (a.directHints & HINT_SRC_DEMOTE));
       continue;
     }
-    pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, RECV ? rslot + j * a.T * w : nullptr, src, dst, so, c.tid, c.nt,
-                                                      hint);
+    pieceSimple<DT, OP, RECV, SEND, SRC, DST, REDDST>(m, ri, src, dst, so, c.tid, c.nt,
+                                                      rpull ? hint | HINT_NO_DISCARD : hint);
   }
 }
 
@@ -883,7 +896,8 @@ __device__ __noinline__ bool runOp(const Ctx& c, const DevTB& tb, const DevInstr
       __syncthreads();                         // c.peerDst visible to every thread
       c.readyDone = true;
     }
-    if (SEND && c.tid == 32 && sent + 1 > (uint64_t)a.slots && !sendIsDirect(c, in))
+    if (SEND && c.tid == 32 && sent + 1 > (uint64_t)a.slots && !sendIsDirect(c, in) &&
+        !((in.flags & DI_SEND_PULLED) && pullOn(c)))
       ok = ok && waitGE(tb.sendAck, sent + 1 - (uint64_t)a.slots, sys, c);
     if (!ok) *sAbort = 1;
     if (RECV || SEND) {

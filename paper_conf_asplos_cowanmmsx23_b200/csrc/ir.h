@@ -86,9 +86,11 @@ void deadlockCheckIR(const Algo& a, int slots, int iters);
 // receive may find its data already in its destination (op r / rcs whose destination
 // chunks no other instruction of the rank touches unless ordered after it);
 // sendDirect[tb][step] = the matching receive on the peer is direct (+ its dst buf/off).
+// recvPull[tb][step] = the receive may read its message from the sender's input chunk
+// pullOff (reading R30); sendPulled[tb][step] = the matching receive on the peer pulls.
 struct DirectInfo {
-  std::vector<std::vector<char>> recvDirect, sendDirect;
-  std::vector<std::vector<int>> rdstBuf, rdstOff, rterminal;
+  std::vector<std::vector<char>> recvDirect, sendDirect, recvPull, sendPulled;
+  std::vector<std::vector<int>> rdstBuf, rdstOff, rterminal, pullOff;
 };
 DirectInfo directPlacement(const Algo& a, int rank);
 

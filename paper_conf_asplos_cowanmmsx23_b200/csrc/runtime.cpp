@@ -31,7 +31,7 @@ namespace {
 // threads per CTA (2 CTAs per SM), direct placement on. LL / LL128 have their own FIFO slots.
 struct Params {
   int64_t slots = 4, slotBytes = 262144, llSlotBytes = 65536, ll128SlotBytes = 262144, maxChannels = 32,
-          threads = 256, timeoutS = 60, direct = 1, directTile = 1, directHints = 9, regMax = 64,
+          threads = 256, timeoutS = 60, direct = 1, directTile = 1, directHints = 25, regMax = 64,
           crossLaunch = 0;
 };
 
@@ -1092,7 +1092,8 @@ mscclResult_t mscclDebugDirectPlacement(const char* ir, size_t irBytes, int rank
     for (size_t t = 0; t < g.tbs.size(); t++)
       for (size_t s = 0; s < g.tbs[t].steps.size(); s++, k++) {
         if (k >= maxInstr || !flags) continue;
-        flags[k] = (di.sendDirect[t][s] ? 1 : 0) | (di.recvDirect[t][s] ? 2 : 0);
+        flags[k] = (di.sendDirect[t][s] ? 1 : 0) | (di.recvDirect[t][s] ? 2 : 0) | (di.recvPull[t][s] ? 4 : 0) |
+                   (di.sendPulled[t][s] ? 8 : 0);
         if (rdst) {
           rdst[2 * k] = di.sendDirect[t][s] ? di.rdstBuf[t][s] : -1;
           rdst[2 * k + 1] = di.sendDirect[t][s] ? di.rdstOff[t][s] : -1;
@@ -1404,6 +1405,12 @@ mscclResult_t mscclLoadProgram(mscclComm_t c, const char* ir, size_t irBytes, si
         deps.push_back(((uint64_t)dp.first << 48) | ((uint64_t)dp.second << 32) |
                        (uint64_t)(uint32_t)g.tbs[dp.first].steps.size());
       if (dinfo.recvDirect[t][si]) di.flags |= DI_RECV_DIRECT;
+      if (dinfo.recvPull[t][si]) {  // reading R30
+        di.flags |= DI_RECV_PULL;
+        di.chainLen = (uint16_t)tb.recv;
+        di.pullOff = (uint32_t)dinfo.pullOff[t][si];
+      }
+      if (dinfo.sendPulled[t][si]) di.flags |= DI_SEND_PULLED;
       const bool sends = in.op == OP_SEND || in.op == OP_RRS || in.op == OP_RRCS || in.op == OP_RCS;
       if (sends && !dinfo.sendDirect[t][si]) p->allDirect = false;
       if (dinfo.sendDirect[t][si]) {

@@ -266,6 +266,41 @@ bool recvCanBeDirect(const Algo& a, int g, int tb, int s) {
   return true;
 }
 
+// may receive step (tb, s) of rank g read its message straight from the sender's input chunk
+// (reading R30)? The matching send is a plain `s` of an input chunk, the program is out of
+// place and the sender's rank writes no input chunk, so the chunk holds the same data from the
+// start of the launch to its end; Simple protocol only; a receive that is already direct keeps
+// that. Every piece of the receive must have the length of the sender's chunk: its non-scratch
+// chunks sit at the sender's chunk position in their block, and it has at least one.
+bool recvCanPull(const Algo& a, int g, int tb, int s) {
+  if (a.proto != PROTO_SIMPLE || a.inplace) return false;
+  const ThreadBlock& rt = a.gpus[g].tbs[tb];
+  const Instr& q = rt.steps[s];
+  const Instr* snd = matchingSend(a, g, tb, s);
+  if (!snd || snd->op != OP_SEND || snd->srcBuf != BUF_IN || snd->cnt != q.cnt) return false;
+  if (recvCanBeDirect(a, g, tb, s)) return false;
+  for (auto& t : a.gpus[rt.recv].tbs)
+    for (auto& x : t.steps)
+      if (opRole(x.op).dst && x.dstBuf == BUF_IN) return false;
+  const int cb = a.gpus[0].iChunks / blocksOf(a.coll, BUF_IN, a.ngpus);
+  if (cb <= 0) return false;
+  const OpRole ro = opRole(q.op);
+  for (int j = 0; j < q.cnt; j++) {
+    const int want = (snd->srcOff + j) % cb;
+    bool anchored = false;
+    if (ro.src && q.srcBuf != BUF_SC) {
+      if ((q.srcOff + j) % cb != want) return false;
+      anchored = true;
+    }
+    if (ro.dst && q.dstBuf != BUF_SC) {
+      if ((q.dstOff + j) % cb != want) return false;
+      anchored = true;
+    }
+    if (!anchored) return false;
+  }
+  return true;
+}
+
 }  // namespace
 
 DirectInfo directPlacement(const Algo& a, int rank) {
@@ -276,6 +311,9 @@ DirectInfo directPlacement(const Algo& a, int rank) {
   di.rdstBuf.resize(g.tbs.size());
   di.rdstOff.resize(g.tbs.size());
   di.rterminal.resize(g.tbs.size());
+  di.recvPull.resize(g.tbs.size());
+  di.pullOff.resize(g.tbs.size());
+  di.sendPulled.resize(g.tbs.size());
   for (size_t t = 0; t < g.tbs.size(); t++) {
     const ThreadBlock& tb = g.tbs[t];
     di.recvDirect[t].assign(tb.steps.size(), 0);
@@ -283,8 +321,17 @@ DirectInfo directPlacement(const Algo& a, int rank) {
     di.rdstBuf[t].assign(tb.steps.size(), 0);
     di.rdstOff[t].assign(tb.steps.size(), 0);
     di.rterminal[t].assign(tb.steps.size(), 0);
+    di.recvPull[t].assign(tb.steps.size(), 0);
+    di.pullOff[t].assign(tb.steps.size(), 0);
+    di.sendPulled[t].assign(tb.steps.size(), 0);
     for (size_t s = 0; s < tb.steps.size(); s++)
-      if (opRole(tb.steps[s].op).recv) di.recvDirect[t][s] = recvCanBeDirect(a, rank, (int)t, (int)s);
+      if (opRole(tb.steps[s].op).recv) {
+        di.recvDirect[t][s] = recvCanBeDirect(a, rank, (int)t, (int)s);
+        if (recvCanPull(a, rank, (int)t, (int)s)) {
+          di.recvPull[t][s] = 1;
+          di.pullOff[t][s] = matchingSend(a, rank, (int)t, (int)s)->srcOff;
+        }
+      }
     if (tb.send < 0) continue;
     // pair the k-th send of (rank -> peer, chan) with the k-th receive of the peer's receiving tb
     const GpuProgram& pg = a.gpus[tb.send];
@@ -306,6 +353,7 @@ DirectInfo directPlacement(const Algo& a, int rank) {
           di.rdstOff[t][s] = rt->steps[rs].dstOff;
           di.rterminal[t][s] = rt->steps[rs].op == OP_RECV ? 1 : 0;
         }
+        if (recvCanPull(a, tb.send, rt->id, rs)) di.sendPulled[t][s] = 1;
       }
       k++;
     }

@@ -111,7 +111,8 @@ def validate(ir_text, nranks, slots=0, max_tbs=0):
 def direct_placement(ir_text, rank):
     """The loader's direct-placement marking for `rank` (mscclDebugDirectPlacement, no GPU):
     a list, in (thread block, step) order, of (flags, rdst_buf, rdst_chunk) with flags bit 0 =
-    direct send, bit 1 = direct receive (reading R15)."""
+    direct send, bit 1 = direct receive (reading R15), bit 2 = pulled receive, bit 3 = pulled send
+    (reading R30)."""
     b = ir_text.encode() if isinstance(ir_text, str) else ir_text
     n = _i()
     _check(lib.mscclDebugDirectPlacement(b, len(b), rank, None, None, 0, _c.byref(n)))

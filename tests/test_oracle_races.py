@@ -88,7 +88,10 @@ def test_every_loader_marked_receive_is_individually_safe():
         al = irparse.parse(ir)
         mk = _marking(ir, R)
         full = races.direct_map(al, mk)
-        for e, (kind, tgt) in full.items():
+        for e, v in full.items():
+            if len(e) != 3:   # pulled-message entries (reading R30)
+                continue
+            kind, tgt = v
             if kind not in ("send", "both"):
                 continue
             one = {e: ("send", tgt)}
@@ -180,8 +183,8 @@ def test_hand_marked_direct_receive_with_earlier_reader_is_flagged():
     assert rs and rs[0].loc == (1, "o", 0), rs
     # the loader does not mark it
     from paper_conf_asplos_cowanmmsx23_b200 import runtime
-    assert all(f == 0 for f, _, _ in runtime.direct_placement(ir, 1))
-    assert all(f == 0 for f, _, _ in runtime.direct_placement(ir, 0))
+    assert all(f & 3 == 0 for f, _, _ in runtime.direct_placement(ir, 1))
+    assert all(f & 3 == 0 for f, _, _ in runtime.direct_placement(ir, 0))
 
 
 def test_unordered_reader_of_a_receive_destination_is_flagged():
@@ -272,3 +275,43 @@ def test_validator_v10():
     ir = _direct_hazard_ir(dep=True)
     with pytest.raises(validate.ValidationError, match="^V10"):
         validate.validate(irparse.parse(ir), marking={0: [(1, 1, 0)], 1: [(0, -1, -1), (2, -1, -1), (0, -1, -1)]})
+
+
+def test_pulled_messages_marked_where_expected():
+    """Reading R30: the loader pulls the first hop of every ReduceScatter chain (a plain send of
+    an input chunk) in out-of-place Simple rings, on both ends of the connection, and nowhere
+    in in-place or LL programs."""
+    for algo, R, want in ((P.ring_allreduce(8), 8, 8), (P.ring_reducescatter(8, 1, 2), 8, 16),
+                          (P.ring_allreduce(4, instances=2), 4, 8)):
+        mk = _marking(algo.to_xml(), R)
+        assert sum(1 for q in mk for f, _, _ in mk[q] if f & 8) == want
+        assert sum(1 for q in mk for f, _, _ in mk[q] if f & 4) == want
+    for algo, R in ((P.ring_allreduce(8, inplace=True), 8), (P.ring_allreduce(8, protocol="LL128"), 8),
+                    (P.ring_allgather(8, 1, 1), 8)):
+        mk = _marking(algo.to_xml(), R)
+        assert not any(f & 12 for q in mk for f, _, _ in mk[q])
+
+
+def test_a_pull_of_a_chunk_the_sender_rewrites_is_a_race():
+    """The race checker models a pulled message as a read of the sender's input chunk at the
+    receive: a hand-marked pull of a chunk the sender overwrites after its send (an in-place
+    program, which the loader never pulls) is reported; the loader's own marking is race free."""
+    from paper_conf_asplos_cowanmmsx23_b200.dsl import Collective, Program, chunk
+    with Program("pull_war", Collective(2, 2, 2, inplace=True), protocol="Simple") as p:
+        chunk(0, "in", 0).copy(1, "sc", 0)
+        chunk(0, "in", 1).copy(0, "in", 0)
+        chunk(1, "sc", 0).copy(1, "in", 1)
+    ir = p.lower().to_xml()
+    al = irparse.parse(ir)
+    mk = _marking(ir, 2)
+    assert not any(f & 12 for q in mk for f, _, _ in mk[q])
+    assert races.check_direct(al, mk) == []
+    forced = {q: list(v) for q, v in mk.items()}
+    for q in (0, 1):
+        for k, (f, b, o) in enumerate(forced[q]):
+            st = [s for tb in al.gpus[q].tbs for s in tb.steps][k]
+            if st.op == "s":
+                forced[q][k] = (f | 8, b, o)
+            elif st.op in ("r", "rcs", "rrc", "rrs", "rrcs"):
+                forced[q][k] = (f | 4, b, o)
+    assert races.check_direct(al, forced) != []
