@@ -20,7 +20,7 @@ DTYPES = ["int32", "bfloat16", "float32"]
 def small_slots():
     from paper_conf_asplos_cowanmmsx23_b200 import runtime
     keys = ("MSCCL_SLOT_BYTES", "MSCCL_LL_SLOT_BYTES", "MSCCL_LL128_SLOT_BYTES", "MSCCL_TIMEOUT_S", "MSCCL_DIRECT",
-            "MSCCL_CROSS_LAUNCH")
+            "MSCCL_CROSS_LAUNCH", "MSCCL_DIRECT_HINTS")
     old = {k: runtime.get_param(k) for k in keys}
     for k in keys[:3]:
         runtime.set_param(k, 4096)     # several tiles per chunk at these sizes
@@ -30,13 +30,16 @@ def small_slots():
         runtime.set_param(k, v)
 
 
-@pytest.mark.parametrize("mode", ["direct", "fifo", "cross"])
+@pytest.mark.parametrize("mode", ["direct", "nopull", "fifo", "cross"])
 @pytest.mark.parametrize("block", range(6))
 def test_random_programs_bit_exact_vs_oracle(small_slots, mode, block):
+    """Modes: direct placement with pulled first hops (the default, readings R15 / R30), direct
+    placement without pulls (MSCCL_DIRECT_HINTS 9), FIFO only, the cross-launch protocol."""
     import gpu_util
     runtime = small_slots
     runtime.set_param("MSCCL_DIRECT", 0 if mode == "fifo" else 1)
     runtime.set_param("MSCCL_CROSS_LAUNCH", 1 if mode == "cross" else 0)
+    runtime.set_param("MSCCL_DIRECT_HINTS", 9 if mode == "nopull" else 25)
     direct = mode
     for seed in range(block * 50, (block + 1) * 50):
         proto = PROTOS[seed % 3]
@@ -86,7 +89,7 @@ def test_random_programs_other_reductions(small_slots, op):
             assert np.array_equal(a, b), (seed, proto, dtype, op, r, k)
 
 
-@pytest.mark.parametrize("mode", ["direct", "fifo"])
+@pytest.mark.parametrize("mode", ["direct", "nopull", "fifo"])
 def test_random_programs_ragged_sizes_whole_buffers(small_slots, mode):
     """Ragged counts (chunks of unequal length, reading R1 / R2; LL / LL128 partial lines): every
     output chunk the program writes, over its whole span, bit-exact with the simulator."""
@@ -95,6 +98,7 @@ def test_random_programs_ragged_sizes_whole_buffers(small_slots, mode):
     runtime = small_slots
     runtime.set_param("MSCCL_DIRECT", 0 if mode == "fifo" else 1)
     runtime.set_param("MSCCL_CROSS_LAUNCH", 0)
+    runtime.set_param("MSCCL_DIRECT_HINTS", 9 if mode == "nopull" else 25)
     for seed in range(1000, 1100):
         proto = PROTOS[seed % 3]
         dtype = DTYPES[(seed // 3) % 3]

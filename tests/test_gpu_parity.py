@@ -187,3 +187,32 @@ def test_one_rank_programs(name):
     xs = synth.inputs(1, n, "float32", "uniform")
     got = _gpu().run_program(build().to_xml(), xs, n, "float32", "sum")
     assert _bits_equal(got[0][:n], xs[0][:n])
+
+
+@pytest.mark.gpu
+@pytest.mark.parametrize("hints", [25, 9])
+@pytest.mark.parametrize("name", ["ring_allreduce", "ring_reducescatter"])
+def test_pulled_first_hops_bit_exact(name, hints):
+    """Reading R30: the ring's first hops read the sender's input chunk (MSCCL_DIRECT_HINTS
+    bit 4, the default) or go through the FIFO (9); both bit-exact with the oracle at a ragged
+    count over several tiles, bf16 and int32."""
+    import gpu_util
+    from paper_conf_asplos_cowanmmsx23_b200 import runtime
+    old = runtime.get_param("MSCCL_DIRECT_HINTS"), runtime.get_param("MSCCL_SLOT_BYTES")
+    runtime.set_param("MSCCL_DIRECT_HINTS", hints)
+    runtime.set_param("MSCCL_SLOT_BYTES", 8192)
+    try:
+        R = 8
+        algo = P.ring_allreduce(R, instances=2) if name == "ring_allreduce" else P.ring_reducescatter(R, 1, 2)
+        text = algo.to_xml()
+        for dtype in ("bfloat16", "int32"):
+            cnt = R * 2 * 3001 + 5 if name == "ring_allreduce" else 2 * 3001 + 5   # ragged chunks (R1)
+            n_in = cnt if name == "ring_allreduce" else R * cnt
+            xs = synth.inputs(R, n_in, dtype, "int" if dtype == "int32" else "uniform", seed=hints)
+            want = sim.simulate(irparse.parse(text), xs, cnt, dtype, "sum")
+            got = gpu_util.run_program(text, xs, cnt, dtype, "sum", out_elems=cnt)
+            for r in range(R):
+                assert np.array_equal(got[r][:cnt].view(np.uint8), want[r][:cnt].view(np.uint8)), (name, hints, dtype, r)
+    finally:
+        runtime.set_param("MSCCL_DIRECT_HINTS", old[0])
+        runtime.set_param("MSCCL_SLOT_BYTES", old[1])
