@@ -173,7 +173,9 @@ mscclResult_t mscclProgramInfo(mscclProgram_t program, int* nThreadBlocks, int* 
  * pass (bytes per launch = touches * chunk bytes): each instruction reads/writes its
  * operands once per chunk — send 2, recv 2, copy 2, reduce 3, rrc 3, rrs 3, rrcs 4, rcs 3 —
  * and with direct placement (directPlacement != 0, reading R15) a direct recv costs 0 and
- * a direct rcs 2 (the data arrived in dst). */
+ * a direct rcs 2 (the data arrived in dst); with every rank in one launch (directPlacement
+ * == 1; 2 = cross-launch) and MSCCL_DIRECT_HINTS bit 4, a pulled send costs 0 (reading R30:
+ * its receive reads the input chunk instead of the FIFO slot, same count). */
 mscclResult_t mscclProgramTouches(mscclProgram_t program, int directPlacement, int64_t* touches);
 
 /* Direct-placement marking the loader computes for rank `rank` of an IR program (reading

@@ -1542,6 +1542,7 @@ mscclResult_t mscclProgramTouches(mscclProgram_t p, int direct, int64_t* touches
       const Instr& in = g.tbs[t].steps[s];
       int c = cost[in.op];
       if (direct && di.recvDirect[t][s]) c = in.op == OP_RCS ? 2 : 0;
+      if (direct == 1 && (p->comm->prm.directHints & 16) && di.sendPulled[t][s]) c = 0;  // reading R30
       n += (int64_t)c * in.cnt;
     }
   *touches = n;
