@@ -1053,7 +1053,7 @@ def main():
                    "peak": l2peak, "frac": round(achieved / l2peak, 4) if l2peak else None,
                    "peak_source": l2src,
                    "note": "touched = the program's per-instruction operand bytes (send 2, recv 2, copy 2, "
-                           "reduce/rrc/rrs 3, rrcs 4, rcs 3 chunks; a direct recv 0, a direct rcs 2), i.e. "
+                           "reduce/rrc/rrs 3, rrcs 4, rcs 3 chunks; a direct recv 0, a direct rcs 2, a pulled send 0), i.e. "
                            "the L2-level traffic of the interpreter; FIFO slots live mostly in L2"},
             "direct_placement": res.get("direct")}
         out["nccl"] = {"note": "skipped: one GPU (NCCL cannot run 8 ranks on one device); the NCCL arm runs "
